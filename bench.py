@@ -1,0 +1,338 @@
+#!/usr/bin/env python3
+"""Benchmark: PCIAM tile-pair translations/sec on the paper's headline 42x59 grid.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config 3] [--impl ours|reference]
+
+A "step" is one pass of the whole hot path (forward
+R2C FFT of every tile, NCPS + inverse FFT + argmax + 4-candidate CCF + selection
+for every west/north pair) over the synthetic grid of BASELINE.json configs[2]
+(42x59 tiles of 1392x1040 uint16).  `value` is pairs/s
+with the tiles resident in HBM; `e2e` is the same through the C ABI from pinned
+host buffers (H2D of the tiles + D2H of the results inside the timed region).
+Inputs (7.2 GB of tiles, 14.5 GB of spectra) are far larger than the 126 MB L2.
+
+N > 1 (torchrun): row-band partition of the grid, one rank per GPU; each rank
+owns tiles [k*nt/N, (k+1)*nt/N) and keeps the preceding tile row resident (halo,
+recomputed locally); the per-step time is the max over ranks (all_reduce MAX).
+
+--impl reference: the reference arm is the oracle (oracle/, plain C, fp64),
+timed as it stands on the host cores on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import synthgrid  # noqa: E402
+
+PAPER_PAIRS_PER_S = 4855 / 49.7   # Pipelined-GPU, 1x Tesla C2070, Table II: context
+REASON_BITS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
+               0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
+               0x40: "hw_thermal_slowdown", 0x80: "hw_power_brake_slowdown",
+               0x100: "display_clock_setting"}
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f), "measured"
+    except OSError:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0}, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device),
+                 "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active",
+                 "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 3:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx = float(parts[1])
+                bits = int(parts[2], 16)
+            except ValueError:
+                continue
+            for b, name in REASON_BITS.items():
+                if bits & b and name != "gpu_idle":
+                    reasons.add(name)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": mx, "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def band(rank: int, world: int, n: int, m: int):
+    nt = n * m
+    b, e = rank * nt // world, (rank + 1) * nt // world
+    halo = max(0, b - m)
+    return b, e, halo
+
+
+def cpu_baseline(cfg: dict, sub_rows: int = 3, sub_cols: int = 4):
+    """The oracle as it stands, on a bounded sample (a sub_rows x sub_cols corner of the
+    workload's grid: same tiles, same pair kinds), all host cores."""
+    import oracle
+    g = synthgrid.make_grid(sub_rows, sub_cols, cfg["H"], cfg["W"], overlap=cfg["overlap"],
+                            delta=cfg["delta"])
+    cores = os.cpu_count() or 1
+    t = time.perf_counter()
+    oracle.grid(g.tiles, threads=cores)
+    dt = time.perf_counter() - t
+    pairs = 2 * sub_rows * sub_cols - sub_rows - sub_cols
+    return {"value": pairs / dt, "unit": "pairs/s", "cores": cores, "kind": "oracle",
+            "sample": f"{sub_rows}x{sub_cols} corner of the {cfg['name']} grid ({pairs} pairs, "
+                      f"{sub_rows * sub_cols} tiles), oracle.grid fp64, {dt:.1f} s wall"}
+
+
+def run_reference(args, cfg):
+    """Reference arm: the oracle timed on the host cores, bounded sample per step."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    sub = (2, 3)
+    g = synthgrid.make_grid(sub[0], sub[1], cfg["H"], cfg["W"], overlap=cfg["overlap"],
+                            delta=cfg["delta"])
+    pairs = 2 * sub[0] * sub[1] - sub[0] - sub[1]
+    cores = os.cpu_count() or 1
+    for _ in range(args.warmup):
+        oracle.grid(g.tiles, threads=cores)
+    t = time.perf_counter()
+    for _ in range(args.steps):
+        oracle.grid(g.tiles, threads=cores)
+    dt = time.perf_counter() - t
+    value = pairs * args.steps / dt
+    line = {
+        "impl": "reference", "metric": f"tile-pair translations/sec ({cfg['name']} grid)",
+        "value": value, "unit": "pairs/s", "n_gpus": args.gpus, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+        "config": {"workload": cfg["name"], "sample": f"{sub[0]}x{sub[1]} sub-grid per step"},
+        "cpu_baseline": {"value": value, "unit": "pairs/s", "cores": cores, "kind": "oracle",
+                         "sample": f"{sub[0]}x{sub[1]} corner of the {cfg['name']} grid "
+                                   f"({pairs} pairs) per step"},
+        "e2e": {"value": value, "unit": "pairs/s", "h2d_bytes_per_step": 0,
+                "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--chunk-pairs", type=int, default=0)
+    ap.add_argument("--chunk-tiles", type=int, default=0)
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    args = ap.parse_args()
+    cfg = dict(synthgrid.CONFIGS[args.config])
+    if args.impl == "reference":
+        return run_reference(args, cfg)
+
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world != args.gpus:
+        raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+
+    n, m, H, W = cfg["n"], cfg["m"], cfg["H"], cfg["W"]
+    b, e, halo = band(rank, world, n, m)
+    r0, r1 = halo // m, (e - 1) // m + 1            # tile rows this rank holds
+    # host tiles of the rows this rank needs, in pinned memory (the e2e source buffer)
+    host = torch.empty((r1 - r0, m, H, W), dtype=torch.uint16, pin_memory=True)
+    synthgrid.make_grid(n, m, H, W, overlap=cfg["overlap"], delta=cfg["delta"],
+                        out=host.numpy().view(np.uint16), rows=(r0, r1))
+    first = r0 * m
+
+    pg = PciamGrid(n, m, H, W, device=local, tile_begin=b, tile_end=e,
+                   chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles)
+    stream = torch.cuda.current_stream()
+    pg.load_tiles(host, first)
+    pg.synchronize()
+    pairs_local = pg.npairs
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    # ---- warm-up, then K timed steps with tiles resident in HBM ----------------------------
+    for _ in range(args.warmup):
+        pg.compute_translations_async()
+    barrier()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    launches = 0
+    with ClockSampler(local) as clk:
+        barrier()
+        ev0.record(stream)
+        for _ in range(args.steps):
+            pg.compute_translations_async()
+            launches += pg.last_counts()["launches"]
+        ev1.record(stream)
+        barrier()
+    dev_ms = ev0.elapsed_time(ev1) / args.steps
+    ms = max_over_ranks(dev_ms)
+    total_pairs = sum_over_ranks(pairs_local)
+    value = total_pairs / (ms / 1e3)
+    clocks = clk.summary()
+
+    # ---- per-kernel durations (timing mode 2: an event after every launch) ---------------
+    pg.set_timing(2)
+    kt_sum = {}
+    for _ in range(max(1, min(args.steps, 5))):
+        pg.compute_translations_async()
+        pg.synchronize()
+        for k, v in pg.kernel_timings().items():
+            s = kt_sum.setdefault(k, {"ms": 0.0, "launches": 0})
+            s["ms"] += v["ms"]
+            s["launches"] += v["launches"]
+    pg.set_timing(0)
+    step_kernel_ms = sum(v["ms"] for v in kt_sum.values())
+    dom = max(kt_sum, key=lambda k: kt_sum[k]["ms"])
+    S = H * (W // 2 + 1) * 8          # algorithmic fp32 half spectrum bytes
+    T = H * W * 2                     # raw tile bytes
+    alg_bytes_per_unit = {            # SURVEY 8(d) per-unit byte model
+        "k1_fwd_rows": T + S, "k2_fwd_cols": 2 * S, "k3_pair_cols": 3 * S,
+        "k4_pair_rows": S, "k5_ccf_moments": 2 * T, "k6_finalize": 8 + 160 + 64}
+    units_per_launch = {
+        "k1_fwd_rows": pg.cfg.chunk_tiles or 8, "k2_fwd_cols": pg.cfg.chunk_tiles or 8,
+        "k3_pair_cols": pg.cfg.chunk_pairs or 8, "k4_pair_rows": pg.cfg.chunk_pairs or 8}
+    kd = kt_sum[dom]
+    nsteps_k = max(1, min(args.steps, 5))
+    units_total = {"k1_fwd_rows": (e - halo), "k2_fwd_cols": (e - halo),
+                   "k3_pair_cols": pairs_local, "k4_pair_rows": pairs_local,
+                   "k5_ccf_moments": pairs_local, "k6_finalize": pairs_local}
+    bytes_per_launch = alg_bytes_per_unit[dom] * units_total[dom] / (kd["launches"] / nsteps_k)
+    avg_launch_ms = kd["ms"] / kd["launches"]
+    pk, pk_kind = peaks()
+    achieved = bytes_per_launch / (avg_launch_ms / 1e3) / 1e9
+    roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": pk["hbm_gbs"],
+                "unit": "GB/s", "frac": achieved / pk["hbm_gbs"], "traffic": None,
+                "peak_source": pk_kind, "avg_launch_ms": avg_launch_ms,
+                "alg_bytes_per_launch": bytes_per_launch,
+                "share_of_step": kd["ms"] / step_kernel_ms,
+                "kernels_ms_per_step": {k: v["ms"] / nsteps_k for k, v in kt_sum.items()}}
+    grid_alg_bytes = ((e - halo) * (T + 3 * S) + pairs_local * (4 * S + 2 * T))
+    roofline["step_alg_GBps"] = grid_alg_bytes / (dev_ms / 1e3) / 1e9
+    traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(traffic_path):
+        with open(traffic_path) as f:
+            tr = json.load(f).get(dom)
+        if tr:
+            roofline["traffic"] = tr.get("bytes_per_launch")
+
+    # ---- e2e: through the C ABI from pinned host buffers ------------------------------
+    e2e_steps = max(1, args.e2e_steps)
+    barrier()
+    t0 = time.perf_counter()
+    for _ in range(e2e_steps):
+        pg.load_tiles(host, first)
+        west, north = pg.compute_translations()     # D2H of the results, synchronous
+    torch.cuda.synchronize()
+    e2e_s = max_over_ranks((time.perf_counter() - t0) / e2e_steps)
+    h2d = (e - halo) * T
+    d2h = pairs_local * 64
+
+    # ---- oracle on the host cores (rank 0, N = 1 only) ----------------------------------
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        cpu = cpu_baseline(cfg)
+
+    if rank == 0:
+        line = {
+            "metric": f"tile-pair translations/sec ({cfg['name']} grid; grid wall time in config)",
+            "value": value, "unit": "pairs/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": value / PAPER_PAIRS_PER_S,
+            "vs_baseline_ref": "paper Pipelined-GPU 1xC2070, 42x59 in 49.7 s (Table II, P:L1208)"
+                               " = 97.7 pairs/s; other hardware, end-to-end incl. TIFF reads",
+            "dtype": "f32", "data": "synthetic",
+            "config": {"workload": f"{cfg['name']} (BASELINE.json configs[{args.config - 1}])",
+                       "grid": f"{n}x{m}", "tile": f"{W}x{H} uint16", "pairs": int(total_pairs),
+                       "tiles": n * m, "grid_wall_ms": ms, "parallelism": f"row-bands x{world}",
+                       "l2": "inputs larger than L2 (7.2 GB tiles, 14.5 GB spectra vs 126 MB)",
+                       "overlap": cfg["overlap"], "seed": synthgrid.SEED},
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": {"value": total_pairs / e2e_s, "unit": "pairs/s", "h2d_bytes_per_step": h2d,
+                    "d2h_bytes_per_step": d2h, "grid_wall_ms": e2e_s * 1e3},
+            "gpu_launches": launches,
+            "clocks": clocks,
+        }
+        print(json.dumps(line), flush=True)
+    pg.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

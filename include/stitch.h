@@ -1,0 +1,186 @@
+/*
+ * stitch.h — C ABI of the B200-native PCIAM tile-pair translation engine.
+ *
+ * Computes phase 1 of the stitching method of Blattner et al., ICPP 2014
+ * (§III): the relative displacement (translation) of every
+ * west and north neighbour pair of a grid of overlapping 16-bit tiles, by
+ * Fourier phase correlation (PCIAM, Fig. 1 steps 1-7; Fig. 2
+ * pciam(); Fig. 3 ccf(); Fig. 4 grid).
+ *
+ * Every step runs in hand-written sm_100a CUDA kernels behind this ABI (no
+ * cuFFT, no CPU fallback).  Arguments are plain pointers and sizes; no torch
+ * or CUDA types appear in the signatures (streams / device memory are passed
+ * as void*).  All functions return a stitch_status; no C++ exception crosses
+ * the boundary.  On error the contents of output arrays are unspecified and
+ * stitch_last_error(ctx) holds a message.
+ *
+ * Conventions
+ *  - Tile layout: uint16 [H][W] row-major, W (x) contiguous.  A grid is
+ *    [n][m][H][W]: n tile rows, m tile columns, tile t = r*m + c.
+ *  - Pair (A, B) = (west or north neighbour, tile) (reading C1);
+ *    the translation (dx, dy) is the origin of B in A's frame, chosen among
+ *    the four candidates {x, W-x} x {y, H-y} of the correlation peak
+ *    (Fig. 2 l.8-12).
+ *  - A context covers the tile range [tile_begin, tile_end) of the grid (a
+ *    row band under multi-GPU partitioning) and computes the pairs whose
+ *    tile B lies in that range; it keeps the tile row before the range (the
+ *    halo) resident too.
+ *  - A context is not thread-safe.  Work is enqueued on the context's stream.
+ */
+#ifndef STITCH_H
+#define STITCH_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct stitch_ctx stitch_ctx; /* opaque, owned by the library */
+
+typedef enum {
+    STITCH_OK = 0,
+    STITCH_ERR_INVALID_ARG = 1, /* null pointer, bad size, bad range */
+    STITCH_ERR_UNSUPPORTED = 2, /* tile size without a compiled FFT plan */
+    STITCH_ERR_OUT_OF_MEMORY = 3,
+    STITCH_ERR_CUDA = 4,        /* a CUDA runtime error; see stitch_last_error */
+    STITCH_ERR_STATE = 6        /* e.g. compute before load */
+} stitch_status;
+
+typedef struct {
+    int32_t tile_width;   /* W (x, contiguous). Compiled plans: 1392x1040, 256x192, 48x40, 58x26 */
+    int32_t tile_height;  /* H (y) */
+    int32_t grid_rows;    /* n >= 1 */
+    int32_t grid_cols;    /* m >= 1 */
+    int32_t device;       /* CUDA ordinal */
+    int32_t tile_begin;   /* first owned tile (row-major index); 0 for the whole grid */
+    int32_t tile_end;     /* one past the last owned tile; 0 => n*m */
+    int32_t chunk_pairs;  /* pairs per inverse-transform chunk (L2-resident intermediate); 0 => default */
+    int32_t chunk_tiles;  /* tiles per forward-transform chunk; 0 => default */
+    int32_t reserved;
+    void* stream;         /* cudaStream_t to enqueue on (e.g. torch's current stream); NULL => library-created */
+    void* workspace;      /* caller-owned device memory of >= stitch_workspace_size bytes (e.g. a torch
+                             tensor), 256-byte aligned; NULL => the library allocates with cudaMalloc */
+    size_t workspace_bytes;
+} stitch_config;
+
+/*
+ * One pair's result (Fig. 2 output "max correlation, x-disp & y-disp", P:L528;
+ * Fig. 4 output "2 arrays of tuples ([correlation, x, y])"), 64 bytes.
+ */
+typedef struct {
+    int32_t dx, dy;        /* chosen translation: origin of tile B in tile A's frame */
+    double ccf;            /* CCF (Fig. 3) of the chosen candidate; NaN if absent / none valid */
+    int32_t candidate;     /* 1..4 in Fig. 2 order (c1..c4); 0 = absent or no valid candidate */
+    int32_t peak_x, peak_y;/* argmax of |iFFT2(NCC)| in [0,W) x [0,H) (step 5) */
+    float peak;            /* max |iFFT2(NCC)| / (W*H) */
+    double ccf_k[4];       /* CCF of each candidate c1..c4 (NaN if invalid: empty region or zero variance) */
+} stitch_pair;
+
+/* Static message for a status code. */
+const char* stitch_status_string(stitch_status s);
+
+/* Bytes of device workspace a context with this config needs (for config.workspace). */
+stitch_status stitch_workspace_size(const stitch_config* cfg, size_t* bytes);
+
+/* Number of pairs the context computes for this config (Fig. 4 order, tile B in range). */
+stitch_status stitch_pair_count(const stitch_config* cfg, int64_t* count);
+
+/*
+ * Create a context: validates the config, selects the compiled FFT plan,
+ * carves / allocates device memory, uploads twiddle tables and the pair list.
+ * Errors: INVALID_ARG (null, n/m < 1, bad tile range, workspace too small),
+ * UNSUPPORTED (tile size), OUT_OF_MEMORY, CUDA.  *out is NULL on error.
+ */
+stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out);
+
+/*
+ * Step 1 (the paper's read + copier stages): copy the
+ * tiles this context needs — rows [halo_begin, tile_end) where halo_begin =
+ * max(0, tile_begin - m) — from the caller's host grid into device memory.
+ * host_grid points at the WHOLE grid [n][m][H][W] (n_bytes = n*m*H*W*2).
+ * Pinned host memory gives asynchronous DMA; the call returns after the copy
+ * has been enqueued and the host buffer may be reused only after the next
+ * stitch_synchronize / compute call returns.
+ */
+stitch_status stitch_load_grid(stitch_ctx* ctx, const uint16_t* host_grid, size_t n_bytes);
+
+/*
+ * Partial load: `tiles` points at tile `first_tile` of a [count][H][W] run of
+ * consecutive row-major tiles that must cover the resident range
+ * [halo_begin, tile_end) (see stitch_resident_range).  on_device != 0 => the
+ * pointer is device memory.  Lets each rank of a row-band partition hold only
+ * its own rows on the host.  Errors: INVALID_ARG if the run does not cover the range.
+ */
+stitch_status stitch_load_tiles(stitch_ctx* ctx, const uint16_t* tiles, int32_t first_tile,
+                                int32_t count, int32_t on_device);
+
+/* Resident tile range of the context: halo_begin = max(0, tile_begin - m). */
+stitch_status stitch_resident_range(stitch_ctx* ctx, int32_t* halo_begin, int32_t* tile_begin,
+                                    int32_t* tile_end);
+
+/* Same from device memory (e.g. a torch CUDA tensor holding the whole grid). */
+stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid, size_t n_bytes);
+
+/*
+ * Steps 2-7 for every pair of the range (Fig. 4), results left on the device;
+ * asynchronous on the context stream (no host synchronisation).
+ * Errors: STATE if no grid was loaded; CUDA.
+ */
+stitch_status stitch_compute_translations_async(stitch_ctx* ctx);
+
+/*
+ * Steps 2-7 and copy-out: fills west[t] / north[t] for every owned tile t
+ * (arrays of n*m entries indexed by row-major tile index; entries outside
+ * the owned range are left untouched; a tile with no west (c = 0) or north
+ * (r = 0) neighbour gets candidate 0, ccf NaN).  Synchronous.
+ */
+stitch_status stitch_compute_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north);
+
+/* Copy the results of the last compute to the host (same layout as above). Synchronous. */
+stitch_status stitch_get_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north);
+
+/* Forward transforms only (step 2) for all resident tiles; asynchronous. */
+stitch_status stitch_forward_async(stitch_ctx* ctx);
+
+/*
+ * Test hook: copy tile t's resident half spectrum F(ky, kx), ky in [0,H),
+ * kx in [0, W/2] (complex64, [H][W/2+1][2] floats) to the host.  Valid after
+ * stitch_forward_async / compute.  Synchronous.
+ */
+stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_out);
+
+/* Wait for all work enqueued on the context stream. */
+stitch_status stitch_synchronize(stitch_ctx* ctx);
+
+/*
+ * Counters of the last compute: kernel launches issued by the library, and
+ * the Table I operation counts: forward transforms, pairs
+ * (= NCC products, inverse transforms, max reductions, CCF1..4 evaluations).
+ */
+stitch_status stitch_last_counts(stitch_ctx* ctx, int64_t* launches, int64_t* forward_ffts,
+                                 int64_t* pairs);
+
+/* Device time of the last compute per stage, milliseconds (CUDA events):
+ * ms[0] forward (K1+K2), ms[1] pair transforms (K3+K4), ms[2] CCF (K5+K6), ms[3] total. */
+stitch_status stitch_last_timings(stitch_ctx* ctx, float* ms4);
+
+/* Event timing mode: 0 off (default), 1 per-stage events, 2 per-stage + one event after
+ * every kernel launch (for per-kernel durations; perturbs the timeline slightly). */
+stitch_status stitch_set_timing(stitch_ctx* ctx, int enabled);
+
+/* Mode-2 timings of the last compute per kernel K1..K6: summed device ms and launch counts.
+ * Valid after stitch_synchronize / stitch_get_translations. */
+stitch_status stitch_kernel_timings(stitch_ctx* ctx, float* ms6, int64_t* launches6);
+
+/* Message for the last error on ctx (valid until the next call on ctx). */
+const char* stitch_last_error(stitch_ctx* ctx);
+
+/* Release everything the context owns.  NULL-safe. */
+void stitch_destroy(stitch_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* STITCH_H */

@@ -1,0 +1,279 @@
+"""B200-native PCIAM tile-pair translation engine (Blattner et al., ICPP 2014, phase 1).
+
+Thin Python binding of the C ABI in ``include/stitch.h`` (``libstitch_b200.so``):
+argument marshalling only -- every step of the path runs in the library's
+sm_100a kernels.  PyTorch is used for plumbing only (device workspace, the
+current CUDA stream, torch.distributed in ``parallel.py``).
+
+    from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid
+    g = PciamGrid(n, m, H, W)
+    g.load_grid(tiles)                      # uint16 [n, m, H, W], host or CUDA
+    west, north = g.compute_translations()  # PAIR_DTYPE [n, m] each (Fig. 4 output)
+
+There is no CPU fallback: if the CUDA library is missing this import fails.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libstitch_b200.so")
+
+STATUS = {0: "STITCH_OK", 1: "STITCH_ERR_INVALID_ARG", 2: "STITCH_ERR_UNSUPPORTED",
+          3: "STITCH_ERR_OUT_OF_MEMORY", 4: "STITCH_ERR_CUDA", 6: "STITCH_ERR_STATE"}
+
+# stitch_pair (include/stitch.h), 64 bytes
+PAIR_DTYPE = np.dtype([
+    ("dx", np.int32), ("dy", np.int32), ("ccf", np.float64), ("candidate", np.int32),
+    ("peak_x", np.int32), ("peak_y", np.int32), ("peak", np.float32), ("ccf_k", np.float64, (4,)),
+], align=True)
+assert PAIR_DTYPE.itemsize == 64
+
+# Tile sizes with a compiled FFT plan (stitch_api.cu plan table)
+SUPPORTED_TILES = {(1392, 1040), (256, 192), (48, 40), (58, 26)}
+
+
+class StitchError(RuntimeError):
+    def __init__(self, status: int, msg: str = ""):
+        self.status = status
+        super().__init__(f"{STATUS.get(status, status)}: {msg}")
+
+
+class Config(ctypes.Structure):
+    _fields_ = [("tile_width", ctypes.c_int32), ("tile_height", ctypes.c_int32),
+                ("grid_rows", ctypes.c_int32), ("grid_cols", ctypes.c_int32),
+                ("device", ctypes.c_int32), ("tile_begin", ctypes.c_int32),
+                ("tile_end", ctypes.c_int32), ("chunk_pairs", ctypes.c_int32),
+                ("chunk_tiles", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("stream", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
+                ("workspace_bytes", ctypes.c_size_t)]
+
+
+EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count", "stitch_init",
+           "stitch_load_grid", "stitch_load_grid_device", "stitch_compute_translations_async",
+           "stitch_compute_translations", "stitch_get_translations", "stitch_forward_async",
+           "stitch_debug_spectrum", "stitch_synchronize", "stitch_last_counts",
+           "stitch_last_timings", "stitch_set_timing", "stitch_last_error", "stitch_destroy",
+           "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings"]
+
+_lib = None
+
+
+def load_library():
+    """Load libstitch_b200.so (raises if it has not been built: no fallback path)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise ImportError(f"{LIB_PATH} not built; run __graft_entry__.build() "
+                          "(python -m paper_conf_icpp_blattnerkcsbz14_b200.build)")
+    lib = ctypes.CDLL(LIB_PATH)
+    P, vp, i32, i64 = ctypes.POINTER, ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+    C = P(Config)
+    sig = {
+        "stitch_status_string": (ctypes.c_char_p, [ctypes.c_int]),
+        "stitch_workspace_size": (ctypes.c_int, [C, P(ctypes.c_size_t)]),
+        "stitch_pair_count": (ctypes.c_int, [C, P(i64)]),
+        "stitch_init": (ctypes.c_int, [C, P(vp)]),
+        "stitch_load_grid": (ctypes.c_int, [vp, vp, ctypes.c_size_t]),
+        "stitch_load_grid_device": (ctypes.c_int, [vp, vp, ctypes.c_size_t]),
+        "stitch_compute_translations_async": (ctypes.c_int, [vp]),
+        "stitch_compute_translations": (ctypes.c_int, [vp, vp, vp]),
+        "stitch_get_translations": (ctypes.c_int, [vp, vp, vp]),
+        "stitch_forward_async": (ctypes.c_int, [vp]),
+        "stitch_debug_spectrum": (ctypes.c_int, [vp, i32, vp]),
+        "stitch_synchronize": (ctypes.c_int, [vp]),
+        "stitch_last_counts": (ctypes.c_int, [vp, P(i64), P(i64), P(i64)]),
+        "stitch_last_timings": (ctypes.c_int, [vp, P(ctypes.c_float)]),
+        "stitch_set_timing": (ctypes.c_int, [vp, ctypes.c_int]),
+        "stitch_last_error": (ctypes.c_char_p, [vp]),
+        "stitch_destroy": (None, [vp]),
+        "stitch_load_tiles": (ctypes.c_int, [vp, vp, i32, i32, i32]),
+        "stitch_resident_range": (ctypes.c_int, [vp, P(i32), P(i32), P(i32)]),
+        "stitch_kernel_timings": (ctypes.c_int, [vp, P(ctypes.c_float), P(i64)]),
+    }
+    for name, (res, args) in sig.items():
+        f = getattr(lib, name)
+        f.restype = res
+        f.argtypes = args
+    _lib = lib
+    return lib
+
+
+def make_config(n, m, H, W, device=0, tile_begin=0, tile_end=0, chunk_pairs=0, chunk_tiles=0,
+                stream=None, workspace=None, workspace_bytes=0) -> Config:
+    return Config(W, H, n, m, device, tile_begin, tile_end, chunk_pairs, chunk_tiles, 0,
+                  stream, workspace, workspace_bytes)
+
+
+def workspace_size(cfg: Config) -> int:
+    b = ctypes.c_size_t(0)
+    st = load_library().stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b))
+    if st:
+        raise StitchError(st, "stitch_workspace_size")
+    return b.value
+
+
+def pair_count(cfg: Config) -> int:
+    c = ctypes.c_int64(0)
+    st = load_library().stitch_pair_count(ctypes.byref(cfg), ctypes.byref(c))
+    if st:
+        raise StitchError(st, "stitch_pair_count")
+    return c.value
+
+
+class PciamGrid:
+    """One context over an n x m grid of H x W uint16 tiles (or the row band
+    [tile_begin, tile_end) of it, for multi-GPU row-band partitioning)."""
+
+    def __init__(self, n: int, m: int, H: int, W: int, device: int = 0, tile_begin: int = 0,
+                 tile_end: int = 0, chunk_pairs: int = 0, chunk_tiles: int = 0,
+                 use_torch: bool = True):
+        self.lib = load_library()
+        self.n, self.m, self.H, self.W = n, m, H, W
+        self.device = device
+        self._ctx = ctypes.c_void_p(None)
+        self._ws = None
+        stream = None
+        cfg = make_config(n, m, H, W, device, tile_begin, tile_end, chunk_pairs, chunk_tiles)
+        if use_torch:
+            import torch
+            dev = torch.device("cuda", device)
+            stream = torch.cuda.current_stream(dev).cuda_stream
+            nbytes = workspace_size(cfg)
+            self._ws = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+            cfg.stream = stream
+            cfg.workspace = self._ws.data_ptr()
+            cfg.workspace_bytes = nbytes
+        self.cfg = cfg
+        self.npairs = pair_count(cfg)
+        self.tile_begin = tile_begin
+        self.tile_end = tile_end if tile_end else n * m
+        self._check(self.lib.stitch_init(ctypes.byref(cfg), ctypes.byref(self._ctx)), "init")
+
+    def _check(self, st: int, what: str):
+        if st:
+            msg = self.lib.stitch_last_error(self._ctx).decode() if self._ctx else ""
+            raise StitchError(st, f"{what}: {msg}")
+
+    # -- step 1: load --------------------------------------------------------
+    def load_grid(self, tiles) -> None:
+        """tiles: uint16 [n, m, H, W] numpy array (host) or torch tensor (host or CUDA)."""
+        nbytes = self.n * self.m * self.H * self.W * 2
+        if isinstance(tiles, np.ndarray):
+            if tiles.dtype != np.uint16 or not tiles.flags.c_contiguous or tiles.nbytes != nbytes:
+                raise ValueError("tiles must be a C-contiguous uint16 [n, m, H, W] array")
+            self._keep = tiles
+            self._check(self.lib.stitch_load_grid(self._ctx, tiles.ctypes.data, nbytes), "load")
+            return
+        import torch
+        if tiles.dtype != torch.uint16 or not tiles.is_contiguous() or \
+                tiles.numel() * 2 != nbytes:
+            raise ValueError("tiles must be a contiguous torch.uint16 [n, m, H, W] tensor")
+        self._keep = tiles
+        if tiles.is_cuda:
+            self._check(self.lib.stitch_load_grid_device(self._ctx, tiles.data_ptr(), nbytes),
+                        "load")
+        else:
+            self._check(self.lib.stitch_load_grid(self._ctx, tiles.data_ptr(), nbytes), "load")
+
+    def resident_range(self) -> tuple[int, int, int]:
+        """(halo_begin, tile_begin, tile_end): tiles this context keeps in HBM."""
+        a, b, c = ctypes.c_int32(), ctypes.c_int32(), ctypes.c_int32()
+        self._check(self.lib.stitch_resident_range(self._ctx, ctypes.byref(a), ctypes.byref(b),
+                                                   ctypes.byref(c)), "range")
+        return a.value, b.value, c.value
+
+    def load_tiles(self, tiles, first_tile: int) -> None:
+        """Load a run of consecutive tiles starting at `first_tile` (numpy or torch, [k, H, W]
+        or [rows, m, H, W]) covering resident_range()."""
+        count = (tiles.size if isinstance(tiles, np.ndarray) else tiles.numel()) // (self.H * self.W)
+        self._keep = tiles
+        if isinstance(tiles, np.ndarray):
+            if tiles.dtype != np.uint16 or not tiles.flags.c_contiguous:
+                raise ValueError("tiles must be C-contiguous uint16")
+            ptr, dev = tiles.ctypes.data, 0
+        else:
+            import torch
+            if tiles.dtype != torch.uint16 or not tiles.is_contiguous():
+                raise ValueError("tiles must be a contiguous torch.uint16 tensor")
+            ptr, dev = tiles.data_ptr(), int(tiles.is_cuda)
+        self._check(self.lib.stitch_load_tiles(self._ctx, ptr, first_tile, count, dev), "load")
+
+    # -- steps 2-7 -------------------------------------------------------------
+    def compute_translations_async(self) -> None:
+        self._check(self.lib.stitch_compute_translations_async(self._ctx), "compute")
+
+    def forward_async(self) -> None:
+        self._check(self.lib.stitch_forward_async(self._ctx), "forward")
+
+    def get_translations(self, west: np.ndarray | None = None, north: np.ndarray | None = None):
+        if west is None:
+            west = np.zeros(self.n * self.m, PAIR_DTYPE)
+        if north is None:
+            north = np.zeros(self.n * self.m, PAIR_DTYPE)
+        self._check(self.lib.stitch_get_translations(self._ctx, west.ctypes.data,
+                                                     north.ctypes.data), "get")
+        return west.reshape(self.n, self.m), north.reshape(self.n, self.m)
+
+    def compute_translations(self):
+        """Fig. 4: (west, north) arrays of PAIR_DTYPE, shape [n, m] (owned tiles filled)."""
+        west = np.zeros(self.n * self.m, PAIR_DTYPE)
+        north = np.zeros(self.n * self.m, PAIR_DTYPE)
+        self._check(self.lib.stitch_compute_translations(self._ctx, west.ctypes.data,
+                                                         north.ctypes.data), "compute")
+        return west.reshape(self.n, self.m), north.reshape(self.n, self.m)
+
+    def spectrum(self, tile: int) -> np.ndarray:
+        """Resident half spectrum of a tile, complex64 [H, W//2 + 1] (test hook)."""
+        out = np.empty((self.H, self.W // 2 + 1), np.complex64)
+        self._check(self.lib.stitch_debug_spectrum(self._ctx, tile, out.ctypes.data), "spectrum")
+        return out
+
+    def synchronize(self) -> None:
+        self._check(self.lib.stitch_synchronize(self._ctx), "synchronize")
+
+    def last_counts(self) -> dict:
+        a, b, c = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_int64()
+        self._check(self.lib.stitch_last_counts(self._ctx, ctypes.byref(a), ctypes.byref(b),
+                                                ctypes.byref(c)), "counts")
+        return {"launches": a.value, "forward_ffts": b.value, "pairs": c.value}
+
+    def set_timing(self, mode: int) -> None:
+        """0 off, 1 per-stage events, 2 per-stage + per-launch events."""
+        self._check(self.lib.stitch_set_timing(self._ctx, int(mode)), "timing")
+
+    def kernel_timings(self) -> dict:
+        """Mode-2 per-kernel (K1..K6) summed device ms and launch counts of the last compute."""
+        ms = (ctypes.c_float * 6)()
+        cnt = (ctypes.c_int64 * 6)()
+        self._check(self.lib.stitch_kernel_timings(self._ctx, ms, cnt), "kernel timings")
+        names = ["k1_fwd_rows", "k2_fwd_cols", "k3_pair_cols", "k4_pair_rows",
+                 "k5_ccf_moments", "k6_finalize"]
+        return {n: {"ms": ms[i], "launches": cnt[i]} for i, n in enumerate(names)}
+
+    def last_timings(self) -> dict:
+        ms = (ctypes.c_float * 4)()
+        self._check(self.lib.stitch_last_timings(self._ctx, ms), "timings")
+        return {"forward_ms": ms[0], "pairs_ms": ms[1], "ccf_ms": ms[2], "total_ms": ms[3]}
+
+    def close(self) -> None:
+        if self._ctx:
+            self.lib.stitch_destroy(self._ctx)
+            self._ctx = ctypes.c_void_p(None)
+        self._ws = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

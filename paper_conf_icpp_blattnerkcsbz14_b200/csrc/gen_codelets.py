@@ -1,0 +1,175 @@
+#!/usr/bin/env python3
+"""Generate straight-line fp32 DFT codelets (codelets.cuh) for the CUDA FFT engine.
+
+Each codelet computes, in registers, an unnormalised length-R DFT
+    X[k] = sum_j x[j] exp(SIGN * 2 pi i j k / R),   SIGN = -1 (forward) or +1 (inverse)
+in place on a float2[R] array.  Primes use the symmetric (x_j +- x_{R-j}) form,
+composites a Cooley-Tukey split R = R1*R2 with constant twiddles (trivial ones --
+multiples of pi/4 -- special-cased).  Constants are computed in double here and
+rounded once to float literals.
+
+This is part of the CUDA product path only (it shares nothing with oracle/).
+Run:  python gen_codelets.py > codelets.cuh
+"""
+import math
+import sys
+
+RADICES = [2, 3, 4, 5, 6, 8, 10, 12, 13, 16, 20, 24, 26, 29, 40]
+
+
+def flit(x: float) -> str:
+    if x == 0.0:
+        return "0.0f"
+    s = repr(float(x))
+    if "e" not in s and "." not in s:
+        s += ".0"
+    return f"({s}f)"
+
+
+class Em:
+    def __init__(self):
+        self.lines = []
+        self.n = 0
+
+    def let(self, expr: str) -> str:
+        self.n += 1
+        name = f"t{self.n}"
+        self.lines.append(f"    const float {name} = {expr};")
+        return name
+
+
+def cadd(e, a, b):
+    return (e.let(f"{a[0]} + {b[0]}"), e.let(f"{a[1]} + {b[1]}"))
+
+
+def csub(e, a, b):
+    return (e.let(f"{a[0]} - {b[0]}"), e.let(f"{a[1]} - {b[1]}"))
+
+
+def twiddle(e, a, num, den, sign):
+    """a * exp(sign * 2 pi i num / den)."""
+    num %= den
+    if num == 0:
+        return a
+    g = math.gcd(num, den)
+    num //= g
+    den //= g
+    if den == 2:                       # -1
+        return (e.let(f"-{a[0]}"), e.let(f"-{a[1]}"))
+    if den == 4:                       # (sign i)^num
+        q = num if sign > 0 else (4 - num) % 4   # exponent of +i
+        if q == 1:                     # i * a = (-a.im, a.re)
+            return (e.let(f"-{a[1]}"), a[0])
+        if q == 3:                     # -i * a = (a.im, -a.re)
+            return (a[1], e.let(f"-{a[0]}"))
+    ang = sign * 2.0 * math.pi * num / den
+    c, s = math.cos(ang), math.sin(ang)
+    if den == 8:                       # (+-1 +- i)/sqrt2
+        h = flit(math.sqrt(0.5))
+        cs, ss = (1 if c > 0 else -1), (1 if s > 0 else -1)
+        # re = a.re*c - a.im*s ; im = a.re*s + a.im*c
+        re = e.let(f"{h} * ({'' if cs > 0 else '-'}{a[0]} {'-' if ss > 0 else '+'} {a[1]})")
+        im = e.let(f"{h} * ({'' if ss > 0 else '-'}{a[0]} {'+' if cs > 0 else '-'} {a[1]})")
+        return (re, im)
+    re = e.let(f"fmaf({a[0]}, {flit(c)}, -({a[1]} * {flit(s)}))")
+    im = e.let(f"fmaf({a[0]}, {flit(s)}, {a[1]} * {flit(c)})")
+    return (re, im)
+
+
+def split(n):
+    if n % 4 == 0 and n != 4:
+        return 4, n // 4
+    for p in range(2, n):
+        if n % p == 0:
+            return p, n // p
+    return None
+
+
+def gen(e, xs, sign):
+    n = len(xs)
+    if n == 1:
+        return list(xs)
+    if n == 2:
+        return [cadd(e, xs[0], xs[1]), csub(e, xs[0], xs[1])]
+    sp = split(n)
+    if sp is None:                     # prime: symmetric form
+        h = (n - 1) // 2
+        s = [None] + [cadd(e, xs[j], xs[n - j]) for j in range(1, h + 1)]
+        d = [None] + [csub(e, xs[j], xs[n - j]) for j in range(1, h + 1)]
+        out = [None] * n
+        acc = xs[0]
+        for j in range(1, h + 1):
+            acc = cadd(e, acc, s[j])
+        out[0] = acc
+        for k in range(1, h + 1):
+            ar, ai = xs[0]
+            br, bi = None, None
+            for j in range(1, h + 1):
+                m = (j * k) % n
+                c = math.cos(2.0 * math.pi * m / n)
+                sn = math.sin(2.0 * math.pi * m / n)
+                ar = e.let(f"fmaf({s[j][0]}, {flit(c)}, {ar})")
+                ai = e.let(f"fmaf({s[j][1]}, {flit(c)}, {ai})")
+                if br is None:
+                    br = e.let(f"{d[j][0]} * {flit(sn)}")
+                    bi = e.let(f"{d[j][1]} * {flit(sn)}")
+                else:
+                    br = e.let(f"fmaf({d[j][0]}, {flit(sn)}, {br})")
+                    bi = e.let(f"fmaf({d[j][1]}, {flit(sn)}, {bi})")
+            # X_k = A + sign*i*B ; X_{n-k} = A - sign*i*B ; i*B = (-bi, br)
+            if sign < 0:
+                out[k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
+                out[n - k] = (e.let(f"{ar} - {bi}"), e.let(f"{ai} + {br}"))
+            else:
+                out[k] = (e.let(f"{ar} - {bi}"), e.let(f"{ai} + {br}"))
+                out[n - k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
+        return out
+    n1, n2 = sp
+    # x index j = n2*a + b ; X index k = k1 + n1*k2
+    Z = []
+    for b in range(n2):
+        Y = gen(e, [xs[n2 * a + b] for a in range(n1)], sign)
+        Z.append([twiddle(e, Y[k1], b * k1, n, sign) for k1 in range(n1)])
+    out = [None] * n
+    for k1 in range(n1):
+        X = gen(e, [Z[b][k1] for b in range(n2)], sign)
+        for k2 in range(n2):
+            out[k1 + n1 * k2] = X[k2]
+    return out
+
+
+def codelet(n, sign):
+    e = Em()
+    xs = []
+    for j in range(n):
+        xs.append((f"x{j}r", f"x{j}i"))
+    outs = gen(e, xs, sign)
+    tag = "m" if sign < 0 else "p"
+    lines = [f"__device__ __forceinline__ void dft{n}{tag}(float2* __restrict__ v) {{"]
+    for j in range(n):
+        lines.append(f"    const float x{j}r = v[{j}].x, x{j}i = v[{j}].y;")
+    lines += e.lines
+    for k in range(n):
+        lines.append(f"    v[{k}] = make_float2({outs[k][0]}, {outs[k][1]});")
+    lines.append("}")
+    return "\n".join(lines)
+
+
+def main():
+    out = ["// GENERATED by gen_codelets.py -- do not edit.",
+           "// Straight-line fp32 DFT codelets: v[k] <- sum_j v[j] exp(SIGN 2 pi i j k / R).",
+           "#pragma once", "", "namespace stitch {", "",
+           "template <int R, int SIGN> struct Dft;", ""]
+    for r in RADICES:
+        for sign in (-1, 1):
+            out.append(codelet(r, sign))
+            tag = "m" if sign < 0 else "p"
+            out.append(f"template <> struct Dft<{r}, {sign}> {{ static __device__ __forceinline__ "
+                       f"void run(float2* v) {{ dft{r}{tag}(v); }} }};")
+            out.append("")
+    out.append("}  // namespace stitch")
+    sys.stdout.write("\n".join(out) + "\n")
+
+
+if __name__ == "__main__":
+    main()

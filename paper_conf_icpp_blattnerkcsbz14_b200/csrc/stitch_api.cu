@@ -1,0 +1,583 @@
+// stitch_api.cu — host side of the C ABI declared in include/stitch.h.
+//
+// Owns the device memory plan, the pair list (Fig. 4 order), the
+// launch schedule of K1..K6 (pciam_kernels.cuh) and the copy-in / copy-out.
+// The runtime is deliberately small: one stream, chunked launches sized so the
+// per-chunk intermediates (K1->K2 spectra, K3->K4 Q) stay in the 126 MB L2.
+#include <cuda_runtime.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/stitch.h"
+#include "pciam_kernels.cuh"
+
+using namespace stitch;
+
+namespace {
+
+// ------------------------------------------------------------ plan table ---
+// Compiled tile-size plans (Radix lists: the row transform is W/2 complex).
+//            W     H     row radices            column radices        rowL rowT colP colT
+using P1392 = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 16, 416>;
+using P256 = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 16, 256>;
+using P48 = Plan<48, 40, Radix<24, 24>, Radix<40, 40>, 8, 64, 16, 64>;
+using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 64, 16, 64>;
+
+struct PlanOps {
+    int W, H, M, WC, WP, row_l, col_p;
+    cudaError_t (*setup)();
+    void (*k1)(const uint16_t*, float2*, int, int, const float2*, const float2*, cudaStream_t);
+    void (*k2)(float2*, int, int, const float2*, cudaStream_t);
+    void (*k3)(const float2*, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
+    void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
+               cudaStream_t);
+};
+
+template <class PL>
+cudaError_t plan_setup() {
+    cudaError_t e;
+    if ((e = cudaFuncSetAttribute(k1_fwd_rows<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)PL::ROW_SMEM)) != cudaSuccess) return e;
+    if ((e = cudaFuncSetAttribute(k4_pair_rows<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)PL::ROW_SMEM)) != cudaSuccess) return e;
+    if ((e = cudaFuncSetAttribute(k2_fwd_cols<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)PL::COL_SMEM)) != cudaSuccess) return e;
+    return cudaFuncSetAttribute(k3_pair_cols<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)PL::COL_SMEM);
+}
+
+template <class PL>
+void launch_k1(const uint16_t* raw, float2* spec, int t0, int nt, const float2* twM,
+               const float2* twW, cudaStream_t s) {
+    k1_fwd_rows<PL><<<dim3(PL::H / PL::ROW_L, nt), PL::ROW_T, PL::ROW_SMEM, s>>>(raw, spec, t0,
+                                                                                 twM, twW);
+}
+template <class PL>
+void launch_k2(float2* spec, int t0, int nt, const float2* twH, cudaStream_t s) {
+    k2_fwd_cols<PL><<<dim3(PL::WP / PL::COL_P, nt), PL::COL_T, PL::COL_SMEM, s>>>(spec, t0, twH);
+}
+template <class PL>
+void launch_k3(const float2* spec, float2* Q, const PairIdx* pairs, int p0, int np,
+               const float2* twH, cudaStream_t s) {
+    k3_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(spec, Q, pairs,
+                                                                                   p0, twH);
+}
+template <class PL>
+void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const float2* twM,
+               const float2* twW, cudaStream_t s) {
+    k4_pair_rows<PL><<<dim3(PL::H / PL::ROW_L, np), PL::ROW_T, PL::ROW_SMEM, s>>>(Q, keys, p0,
+                                                                                  twM, twW);
+}
+
+template <class PL>
+PlanOps make_ops() {
+    return PlanOps{PL::W,      PL::H,        PL::M,        PL::WC,       PL::WP,
+                   PL::ROW_L,  PL::COL_P,    plan_setup<PL>, launch_k1<PL>, launch_k2<PL>,
+                   launch_k3<PL>, launch_k4<PL>};
+}
+
+const PlanOps* find_plan(int W, int H) {
+    static const PlanOps ops[] = {make_ops<P1392>(), make_ops<P256>(), make_ops<P48>(),
+                                  make_ops<P58>()};
+    for (const auto& o : ops)
+        if (o.W == W && o.H == H) return &o;
+    return nullptr;
+}
+
+size_t align256(size_t x) { return (x + 255) / 256 * 256; }
+
+struct Layout {
+    int h_begin, t_begin, t_end, nlocal;
+    int64_t npairs;
+    int chunk_pairs, chunk_tiles;
+    size_t off_raw, off_spec, off_q, off_pairs, off_keys, off_mom, off_res, off_tw, total;
+};
+
+stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L) {
+    const int n = c->grid_rows, m = c->grid_cols;
+    const int64_t nt = (int64_t)n * m;
+    L->t_begin = c->tile_begin;
+    L->t_end = c->tile_end ? c->tile_end : (int)nt;
+    if (L->t_begin < 0 || L->t_end > nt || L->t_begin >= L->t_end) return STITCH_ERR_INVALID_ARG;
+    L->h_begin = L->t_begin - m > 0 ? L->t_begin - m : 0;
+    L->nlocal = L->t_end - L->h_begin;
+    int64_t np = 0;
+    for (int t = L->t_begin; t < L->t_end; ++t) np += (t % m >= 1) + (t / m >= 1);
+    L->npairs = np;
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 8;
+    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 8;
+    if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
+    const size_t H = ops->H, W = ops->W, WP = ops->WP;
+    size_t o = 0;
+    L->off_raw = o;   o += align256((size_t)L->nlocal * H * W * sizeof(uint16_t));
+    L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * sizeof(float2));
+    L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * sizeof(float2));
+    L->off_pairs = o; o += align256((size_t)(np > 0 ? np : 1) * sizeof(PairIdx));
+    L->off_keys = o;  o += align256((size_t)(np > 0 ? np : 1) * sizeof(unsigned long long));
+    L->off_mom = o;   o += align256((size_t)(np > 0 ? np : 1) * 20 * sizeof(unsigned long long));
+    L->off_res = o;   o += align256((size_t)(np > 0 ? np : 1) * sizeof(stitch_pair));
+    L->off_tw = o;    o += align256((size_t)(ops->M + ops->H + ops->W) * sizeof(float2));
+    L->total = o;
+    return STITCH_OK;
+}
+
+stitch_status check_config(const stitch_config* c, const PlanOps** ops) {
+    if (!c) return STITCH_ERR_INVALID_ARG;
+    if (c->grid_rows < 1 || c->grid_cols < 1 || c->tile_width < 2 || c->tile_height < 1)
+        return STITCH_ERR_INVALID_ARG;
+    if ((int64_t)c->grid_rows * c->grid_cols > (1 << 30)) return STITCH_ERR_INVALID_ARG;
+    *ops = find_plan(c->tile_width, c->tile_height);
+    if (!*ops) return STITCH_ERR_UNSUPPORTED;
+    if ((int64_t)c->tile_width * c->tile_height > 0x7FFFFFFF) return STITCH_ERR_UNSUPPORTED;
+    return STITCH_OK;
+}
+
+}  // namespace
+
+struct stitch_ctx {
+    stitch_config cfg;
+    const PlanOps* ops;
+    Layout L;
+    int n, m, H, W;
+    cudaStream_t stream = nullptr;
+    bool own_stream = false;
+    char* mem = nullptr;
+    bool own_mem = false;
+    uint16_t* raw;
+    float2 *spec, *Q, *twM, *twH, *twW;
+    PairIdx* pairs;
+    unsigned long long *keys, *mom;
+    stitch_pair* res;
+    std::vector<int32_t> pair_tile;   // global tile index (B) of each pair
+    std::vector<int8_t> pair_kind;    // 0 west, 1 north
+    std::vector<stitch_pair> res_h;
+    bool loaded = false, computed = false;
+    int64_t launches = 0;
+    int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events
+    cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
+    float ms[4] = {0, 0, 0, 0};
+    std::vector<cudaEvent_t> kev;     // per-launch events (timing == 2)
+    std::vector<int8_t> kkind;        // kernel id of each recorded launch
+    float kms[6] = {0, 0, 0, 0, 0, 0};
+    int64_t kcount[6] = {0, 0, 0, 0, 0, 0};
+    std::string err;
+};
+
+// Per-launch event (timing mode 2): kid 0..5 = K1..K6.
+static cudaError_t mark(stitch_ctx* ctx, int kid) {
+    if (ctx->timing < 2) return cudaSuccess;
+    const size_t i = ctx->kkind.size();
+    if (i + 1 >= ctx->kev.size()) {
+        const size_t old = ctx->kev.size();
+        ctx->kev.resize(old ? old * 2 : 1024, nullptr);
+        for (size_t j = old; j < ctx->kev.size(); ++j) {
+            cudaError_t e = cudaEventCreate(&ctx->kev[j]);
+            if (e != cudaSuccess) return e;
+        }
+    }
+    ctx->kkind.push_back((int8_t)kid);
+    return cudaEventRecord(ctx->kev[i + 1], ctx->stream);
+}
+
+static stitch_status fail(stitch_ctx* ctx, stitch_status s, const std::string& msg) {
+    if (ctx) ctx->err = msg;
+    return s;
+}
+
+static stitch_status cuda_fail(stitch_ctx* ctx, cudaError_t e, const char* where) {
+    return fail(ctx, e == cudaErrorMemoryAllocation ? STITCH_ERR_OUT_OF_MEMORY : STITCH_ERR_CUDA,
+                std::string(where) + ": " + cudaGetErrorString(e));
+}
+
+#define CK(call, where)                                   \
+    do {                                                  \
+        cudaError_t e_ = (call);                          \
+        if (e_ != cudaSuccess) return cuda_fail(ctx, e_, where); \
+    } while (0)
+
+extern "C" {
+
+const char* stitch_status_string(stitch_status s) {
+    switch (s) {
+        case STITCH_OK: return "ok";
+        case STITCH_ERR_INVALID_ARG: return "invalid argument";
+        case STITCH_ERR_UNSUPPORTED: return "unsupported tile size";
+        case STITCH_ERR_OUT_OF_MEMORY: return "out of device memory";
+        case STITCH_ERR_CUDA: return "CUDA error";
+        case STITCH_ERR_STATE: return "invalid call order";
+    }
+    return "unknown status";
+}
+
+stitch_status stitch_workspace_size(const stitch_config* cfg, size_t* bytes) {
+    const PlanOps* ops;
+    if (!bytes) return STITCH_ERR_INVALID_ARG;
+    stitch_status s = check_config(cfg, &ops);
+    if (s != STITCH_OK) return s;
+    Layout L;
+    if ((s = make_layout(cfg, ops, &L)) != STITCH_OK) return s;
+    *bytes = L.total;
+    return STITCH_OK;
+}
+
+stitch_status stitch_pair_count(const stitch_config* cfg, int64_t* count) {
+    const PlanOps* ops;
+    if (!count) return STITCH_ERR_INVALID_ARG;
+    stitch_status s = check_config(cfg, &ops);
+    if (s != STITCH_OK) return s;
+    Layout L;
+    if ((s = make_layout(cfg, ops, &L)) != STITCH_OK) return s;
+    *count = L.npairs;
+    return STITCH_OK;
+}
+
+void stitch_destroy(stitch_ctx* ctx) {
+    if (!ctx) return;
+    if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    for (auto& e : ctx->ev)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : ctx->kev)
+        if (e) cudaEventDestroy(e);
+    if (ctx->own_mem && ctx->mem) cudaFree(ctx->mem);
+    if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
+    delete ctx;
+}
+
+stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
+    if (!out) return STITCH_ERR_INVALID_ARG;
+    *out = nullptr;
+    const PlanOps* ops;
+    stitch_status s = check_config(cfg, &ops);
+    if (s != STITCH_OK) return s;
+    Layout L;
+    if ((s = make_layout(cfg, ops, &L)) != STITCH_OK) return s;
+    if (cfg->workspace && cfg->workspace_bytes < L.total) return STITCH_ERR_INVALID_ARG;
+    if (cfg->workspace && (reinterpret_cast<uintptr_t>(cfg->workspace) & 255))
+        return STITCH_ERR_INVALID_ARG;
+
+    stitch_ctx* ctx = new (std::nothrow) stitch_ctx();
+    if (!ctx) return STITCH_ERR_OUT_OF_MEMORY;
+    ctx->cfg = *cfg;
+    ctx->ops = ops;
+    ctx->L = L;
+    ctx->n = cfg->grid_rows;
+    ctx->m = cfg->grid_cols;
+    ctx->H = ops->H;
+    ctx->W = ops->W;
+    auto bail = [&](stitch_status st) {
+        stitch_destroy(ctx);
+        return st;
+    };
+    cudaError_t e = cudaSetDevice(cfg->device);
+    if (e != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if ((e = ops->setup()) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if (cfg->stream) {
+        ctx->stream = (cudaStream_t)cfg->stream;
+    } else {
+        if (cudaStreamCreateWithFlags(&ctx->stream, cudaStreamNonBlocking) != cudaSuccess)
+            return bail(STITCH_ERR_CUDA);
+        ctx->own_stream = true;
+    }
+    if (cfg->workspace) {
+        ctx->mem = (char*)cfg->workspace;
+    } else {
+        e = cudaMalloc(&ctx->mem, L.total);
+        if (e != cudaSuccess)
+            return bail(e == cudaErrorMemoryAllocation ? STITCH_ERR_OUT_OF_MEMORY : STITCH_ERR_CUDA);
+        ctx->own_mem = true;
+    }
+    char* b = ctx->mem;
+    ctx->raw = (uint16_t*)(b + L.off_raw);
+    ctx->spec = (float2*)(b + L.off_spec);
+    ctx->Q = (float2*)(b + L.off_q);
+    ctx->pairs = (PairIdx*)(b + L.off_pairs);
+    ctx->keys = (unsigned long long*)(b + L.off_keys);
+    ctx->mom = (unsigned long long*)(b + L.off_mom);
+    ctx->res = (stitch_pair*)(b + L.off_res);
+    ctx->twM = (float2*)(b + L.off_tw);
+    ctx->twH = ctx->twM + ops->M;
+    ctx->twW = ctx->twH + ops->H;
+
+    // Twiddle tables w_N^e = exp(-2 pi i e / N), computed in double, rounded once.
+    std::vector<float2> tw((size_t)ops->M + ops->H + ops->W);
+    auto fill = [&](float2* dst, int N) {
+        for (int k = 0; k < N; ++k) {
+            const double a = -2.0 * M_PI * (double)k / (double)N;
+            dst[k] = make_float2((float)std::cos(a), (float)std::sin(a));
+        }
+    };
+    fill(tw.data(), ops->M);
+    fill(tw.data() + ops->M, ops->H);
+    fill(tw.data() + ops->M + ops->H, ops->W);
+
+    // Pair list, Fig. 4 order: for each owned tile, west then north, as (neighbour, tile).
+    std::vector<PairIdx> pl;
+    pl.reserve((size_t)L.npairs);
+    for (int t = L.t_begin; t < L.t_end; ++t) {
+        const int r = t / ctx->m, c = t % ctx->m;
+        if (c >= 1) {
+            pl.push_back(PairIdx{t - 1 - L.h_begin, t - L.h_begin});
+            ctx->pair_tile.push_back(t);
+            ctx->pair_kind.push_back(0);
+        }
+        if (r >= 1) {
+            pl.push_back(PairIdx{t - ctx->m - L.h_begin, t - L.h_begin});
+            ctx->pair_tile.push_back(t);
+            ctx->pair_kind.push_back(1);
+        }
+    }
+    ctx->res_h.resize((size_t)L.npairs);
+    if ((e = cudaMemcpyAsync(ctx->twM, tw.data(), tw.size() * sizeof(float2),
+                             cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
+        return bail(STITCH_ERR_CUDA);
+    if (!pl.empty() &&
+        (e = cudaMemcpyAsync(ctx->pairs, pl.data(), pl.size() * sizeof(PairIdx),
+                             cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
+        return bail(STITCH_ERR_CUDA);
+    for (auto& ev : ctx->ev)
+        if (cudaEventCreate(&ev) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if ((e = cudaStreamSynchronize(ctx->stream)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    *out = ctx;
+    return STITCH_OK;
+}
+
+static stitch_status load_common(stitch_ctx* ctx, const uint16_t* src, size_t n_bytes,
+                                 cudaMemcpyKind kind) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!src) return fail(ctx, STITCH_ERR_INVALID_ARG, "null grid pointer");
+    const size_t tile = (size_t)ctx->H * ctx->W;
+    if (n_bytes != (size_t)ctx->n * ctx->m * tile * sizeof(uint16_t))
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "n_bytes != n*m*H*W*2");
+    CK(cudaMemcpyAsync(ctx->raw, src + (size_t)ctx->L.h_begin * tile,
+                       (size_t)ctx->L.nlocal * tile * sizeof(uint16_t), kind, ctx->stream),
+       "load grid");
+    ctx->loaded = true;
+    ctx->computed = false;
+    return STITCH_OK;
+}
+
+stitch_status stitch_load_tiles(stitch_ctx* ctx, const uint16_t* tiles, int32_t first_tile,
+                                int32_t count, int32_t on_device) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!tiles) return fail(ctx, STITCH_ERR_INVALID_ARG, "null tiles pointer");
+    if (first_tile > ctx->L.h_begin || first_tile + (int64_t)count < ctx->L.t_end || first_tile < 0)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range does not cover [halo_begin, tile_end)");
+    const size_t tile = (size_t)ctx->H * ctx->W;
+    CK(cudaMemcpyAsync(ctx->raw, tiles + (size_t)(ctx->L.h_begin - first_tile) * tile,
+                       (size_t)ctx->L.nlocal * tile * sizeof(uint16_t),
+                       on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->stream),
+       "load tiles");
+    ctx->loaded = true;
+    ctx->computed = false;
+    return STITCH_OK;
+}
+
+stitch_status stitch_resident_range(stitch_ctx* ctx, int32_t* halo_begin, int32_t* tile_begin,
+                                    int32_t* tile_end) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (halo_begin) *halo_begin = ctx->L.h_begin;
+    if (tile_begin) *tile_begin = ctx->L.t_begin;
+    if (tile_end) *tile_end = ctx->L.t_end;
+    return STITCH_OK;
+}
+
+stitch_status stitch_load_grid(stitch_ctx* ctx, const uint16_t* host_grid, size_t n_bytes) {
+    return load_common(ctx, host_grid, n_bytes, cudaMemcpyHostToDevice);
+}
+
+stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid, size_t n_bytes) {
+    return load_common(ctx, dev_grid, n_bytes, cudaMemcpyDeviceToDevice);
+}
+
+static stitch_status forward_impl(stitch_ctx* ctx) {
+    const PlanOps* o = ctx->ops;
+    const int nl = ctx->L.nlocal, ct = ctx->L.chunk_tiles;
+    for (int t0 = 0; t0 < nl; t0 += ct) {
+        const int nt = nl - t0 < ct ? nl - t0 : ct;
+        o->k1(ctx->raw, ctx->spec, t0, nt, ctx->twM, ctx->twW, ctx->stream);
+        CK(mark(ctx, 0), "event");
+        o->k2(ctx->spec, t0, nt, ctx->twH, ctx->stream);
+        CK(mark(ctx, 1), "event");
+        ctx->launches += 2;
+    }
+    CK(cudaGetLastError(), "forward launch");
+    return STITCH_OK;
+}
+
+stitch_status stitch_forward_async(stitch_ctx* ctx) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
+    ctx->launches = 0;
+    return forward_impl(ctx);
+}
+
+stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "compute before load");
+    const PlanOps* o = ctx->ops;
+    cudaStream_t s = ctx->stream;
+    const int64_t np = ctx->L.npairs;
+    ctx->launches = 0;
+    ctx->kkind.clear();
+    if (ctx->timing >= 2) {
+        if (ctx->kev.empty()) {
+            ctx->kev.resize(1024, nullptr);
+            for (auto& e : ctx->kev) CK(cudaEventCreate(&e), "event create");
+        }
+        CK(cudaEventRecord(ctx->kev[0], s), "event");
+    }
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[0], s), "event");
+    stitch_status st = forward_impl(ctx);
+    if (st != STITCH_OK) return st;
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], s), "event");
+    if (np > 0) {
+        CK(cudaMemsetAsync(ctx->keys, 0, (size_t)np * sizeof(unsigned long long), s), "memset");
+        CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), s), "memset");
+        if (ctx->timing >= 2) CK(mark(ctx, -1), "event");
+        const int cp = ctx->L.chunk_pairs;
+        for (int64_t p0 = 0; p0 < np; p0 += cp) {
+            const int npc = (int)(np - p0 < cp ? np - p0 : cp);
+            o->k3(ctx->spec, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
+            CK(mark(ctx, 2), "event");
+            o->k4(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, s);
+            CK(mark(ctx, 3), "event");
+            ctx->launches += 2;
+        }
+        CK(cudaGetLastError(), "pair launch");
+    }
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[2], s), "event");
+    if (np > 0) {
+        const int rows = (2 * ctx->H + CCF_ROWS - 1) / CCF_ROWS;
+        for (int64_t p0 = 0; p0 < np; p0 += 65535) {
+            const int npc = (int)(np - p0 < 65535 ? np - p0 : 65535);
+            k5_ccf_moments<<<dim3(rows, npc), CCF_T, 0, s>>>(ctx->raw, ctx->pairs, ctx->keys,
+                                                            ctx->mom, ctx->H, ctx->W, (int)p0);
+            CK(mark(ctx, 4), "event");
+            ctx->launches += 1;
+        }
+        k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, s>>>(ctx->keys, ctx->mom, ctx->res,
+                                                                 ctx->H, ctx->W, (int)np);
+        CK(mark(ctx, 5), "event");
+        ctx->launches += 1;
+        CK(cudaGetLastError(), "ccf launch");
+    }
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[3], s), "event");
+    ctx->computed = true;
+    return STITCH_OK;
+}
+
+static cudaError_t collect_timings(stitch_ctx* ctx) {
+    cudaError_t e = cudaSuccess;
+    if (ctx->timing) {
+        for (int i = 0; i < 3; ++i)
+            if ((e = cudaEventElapsedTime(&ctx->ms[i], ctx->ev[i], ctx->ev[i + 1])) != cudaSuccess)
+                return e;
+        if ((e = cudaEventElapsedTime(&ctx->ms[3], ctx->ev[0], ctx->ev[3])) != cudaSuccess) return e;
+    }
+    if (ctx->timing >= 2) {
+        for (int k = 0; k < 6; ++k) { ctx->kms[k] = 0.f; ctx->kcount[k] = 0; }
+        for (size_t i = 0; i < ctx->kkind.size(); ++i) {
+            float t = 0.f;
+            if ((e = cudaEventElapsedTime(&t, ctx->kev[i], ctx->kev[i + 1])) != cudaSuccess) return e;
+            const int k = ctx->kkind[i];
+            if (k >= 0) { ctx->kms[k] += t; ctx->kcount[k] += 1; }
+        }
+    }
+    return cudaSuccess;
+}
+
+stitch_status stitch_get_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!west || !north) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output array");
+    if (!ctx->computed) return fail(ctx, STITCH_ERR_STATE, "no computed translations");
+    const int64_t np = ctx->L.npairs;
+    if (np > 0)
+        CK(cudaMemcpyAsync(ctx->res_h.data(), ctx->res, (size_t)np * sizeof(stitch_pair),
+                           cudaMemcpyDeviceToHost, ctx->stream),
+           "copy results");
+    CK(cudaStreamSynchronize(ctx->stream), "synchronize");
+    CK(collect_timings(ctx), "event timing");
+    stitch_pair absent;
+    std::memset(&absent, 0, sizeof(absent));
+    absent.ccf = NAN;
+    for (int k = 0; k < 4; ++k) absent.ccf_k[k] = NAN;
+    for (int t = ctx->L.t_begin; t < ctx->L.t_end; ++t) {
+        west[t] = absent;
+        north[t] = absent;
+    }
+    for (int64_t p = 0; p < np; ++p) {
+        stitch_pair* dst = ctx->pair_kind[p] == 0 ? west : north;
+        dst[ctx->pair_tile[p]] = ctx->res_h[p];
+    }
+    return STITCH_OK;
+}
+
+stitch_status stitch_compute_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!west || !north) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output array");
+    stitch_status s = stitch_compute_translations_async(ctx);
+    if (s != STITCH_OK) return s;
+    return stitch_get_translations(ctx, west, north);
+}
+
+stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_out) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!host_out) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output");
+    if (tile < ctx->L.h_begin || tile >= ctx->L.t_end)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
+    const int lt = tile - ctx->L.h_begin;
+    const float2* src = ctx->spec + (size_t)lt * ctx->H * ctx->ops->WP;
+    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), src,
+                         ctx->ops->WP * sizeof(float2), ctx->ops->WC * sizeof(float2), ctx->H,
+                         cudaMemcpyDeviceToHost, ctx->stream),
+       "copy spectrum");
+    CK(cudaStreamSynchronize(ctx->stream), "synchronize");
+    return STITCH_OK;
+}
+
+stitch_status stitch_synchronize(stitch_ctx* ctx) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    CK(cudaStreamSynchronize(ctx->stream), "synchronize");
+    if (ctx->computed) CK(collect_timings(ctx), "event timing");
+    return STITCH_OK;
+}
+
+stitch_status stitch_kernel_timings(stitch_ctx* ctx, float* ms6, int64_t* launches6) {
+    if (!ctx || !ms6 || !launches6) return STITCH_ERR_INVALID_ARG;
+    for (int k = 0; k < 6; ++k) {
+        ms6[k] = ctx->kms[k];
+        launches6[k] = ctx->kcount[k];
+    }
+    return STITCH_OK;
+}
+
+stitch_status stitch_last_counts(stitch_ctx* ctx, int64_t* launches, int64_t* forward_ffts,
+                                 int64_t* pairs) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (launches) *launches = ctx->launches;
+    if (forward_ffts) *forward_ffts = ctx->L.nlocal;
+    if (pairs) *pairs = ctx->L.npairs;
+    return STITCH_OK;
+}
+
+stitch_status stitch_last_timings(stitch_ctx* ctx, float* ms4) {
+    if (!ctx || !ms4) return STITCH_ERR_INVALID_ARG;
+    for (int i = 0; i < 4; ++i) ms4[i] = ctx->ms[i];
+    return STITCH_OK;
+}
+
+stitch_status stitch_set_timing(stitch_ctx* ctx, int enabled) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (enabled < 0 || enabled > 2) return fail(ctx, STITCH_ERR_INVALID_ARG, "timing mode 0..2");
+    ctx->timing = enabled;
+    return STITCH_OK;
+}
+
+const char* stitch_last_error(stitch_ctx* ctx) { return ctx ? ctx->err.c_str() : "null context"; }
+
+}  // extern "C"
