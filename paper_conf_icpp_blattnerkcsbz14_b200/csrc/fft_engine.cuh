@@ -1,17 +1,20 @@
 // fft_engine.cuh — batched in-CTA mixed-radix Stockham FFT for sm_100a.
 //
-// A CTA transforms L lines of length N.  Each stage of radix R (Stockham
-// autosort, NS = product of the radices already applied) gives every thread
-// whole radix-R butterflies held in registers:
-//     inputs   n = b + j*(N/R),                 j < R
-//     twiddle  v[j] *= w_N^{SIGN * j*k*(N/(NS*R))},  k = b mod NS
-//     DFT_R    straight-line codelet (codelets.cuh)
-//     outputs  n = (b/NS)*NS*R + k + j*NS
-// The first stage reads from a caller "source" functor (global memory with
-// the producer's arithmetic fused in: uint16->fp32, NCPS, C2R pre-twiddle)
-// and the last stage writes to a "destination" functor (global memory or the
-// fused argmax epilogue), so a two-stage transform makes exactly one shared-
-// memory round trip.  No cuFFT, no tensor cores: the path is HBM/FP32-bound.
+// A CTA transforms L lines of length N = R0 * R1 (one or two radix stages).
+// Stockham autosort, two stages:
+//   stage 1 (radix R0, butterfly b < R1):  in  n = b + j*R1          (j < R0)
+//                                           out (u = j, v = b)        n = b*R0 + j
+//   stage 2 (radix R1, butterfly b < R0):  in  (u = b, v = j)        n = b + j*R0 (j < R1)
+//                                           twiddle w_N^{SIGN j b}
+//                                           out n = b + j*R0
+// so the exchange buffer is an R1 x R0 matrix written at (u=j, v=b) and read at
+// (u=b, v=j): one shared-memory round trip per transform.  Each thread owns whole
+// radix-R butterflies in registers (straight-line codelets, codelets.cuh).
+// The first stage reads from a caller "source" functor (global memory with the
+// producer's arithmetic fused in: uint16->fp32, NCPS, C2R pre-twiddle) and the
+// second writes to a "destination" functor (global memory, shared memory, or the
+// argmax epilogue).  Every address inside a butterfly is base + constant offset.
+// No cuFFT, no tensor cores: the path is HBM- / FP32-issue-bound.
 #pragma once
 #include <cuda_runtime.h>
 #include <stdint.h>
@@ -23,25 +26,9 @@ namespace stitch {
 __device__ __forceinline__ float2 cmul(float2 a, float2 b) {
     return make_float2(fmaf(a.x, b.x, -a.y * b.y), fmaf(a.x, b.y, a.y * b.x));
 }
-
-// Shared-memory line storage, line-major with one float2 of padding per 16
-// elements so stride-R Stockham writes spread over the 32 banks.
-template <int STRIDE>
-struct RowSmem {
-    float2* s;
-    static __host__ __device__ constexpr int phys(int n) { return n + (n >> 4); }
-    __device__ __forceinline__ float2 load(int line, int n) const { return s[line * STRIDE + phys(n)]; }
-    __device__ __forceinline__ void store(int line, int n, float2 v) const { s[line * STRIDE + phys(n)] = v; }
-};
-
-// Column-panel storage: element n of line (column) c at n*P + c, so 16
-// consecutive threads touch 16 consecutive columns (one 128-byte wavefront).
-template <int P>
-struct ColSmem {
-    float2* s;
-    __device__ __forceinline__ float2 load(int line, int n) const { return s[n * P + line]; }
-    __device__ __forceinline__ void store(int line, int n, float2 v) const { s[n * P + line] = v; }
-};
+__device__ __forceinline__ float2 cmulc(float2 a, float2 b) {  // a * conj(b)
+    return make_float2(fmaf(a.x, b.x, a.y * b.y), fmaf(a.y, b.x, -a.x * b.y));
+}
 
 // Butterfly id g -> (line, b).  Row map: consecutive threads walk one line.
 struct RowMap {
@@ -60,114 +47,164 @@ struct ColMap {
     }
 };
 
-template <int N, int R, int NS, int SIGN>
-__device__ __forceinline__ void butterfly(float2 (&v)[R], int b, const float2* __restrict__ tw) {
-    if constexpr (NS > 1) {
-        const int k = b % NS;
-        constexpr int TS = N / (NS * R);
-#pragma unroll
-        for (int j = 1; j < R; ++j) {
-            float2 w = __ldg(&tw[j * k * TS]);
-            if constexpr (SIGN > 0) w.y = -w.y;
-            v[j] = cmul(v[j], w);
-        }
+// Exchange buffer for row lines: line-major, each line an R1 x (R0+PAD) matrix.
+template <int R0, int R1, int PAD>
+struct RowXchg {
+    float2* s;
+    static constexpr int LSTRIDE = R1 * (R0 + PAD);
+    __device__ __forceinline__ float2& at(int line, int u, int v) const {
+        return s[line * LSTRIDE + v * (R0 + PAD) + u];
     }
-    Dft<R, SIGN>::run(v);
-}
-
-// One Stockham stage.  INPLACE: src and dst alias the same shared memory, so
-// every thread loads all of its butterflies before a barrier, then stores.
-template <int N, int R, int NS, int SIGN, int L, int T, class Map, bool INPLACE, class Src,
-          class Dst>
-__device__ __forceinline__ void fft_stage(const Src& src, Dst& dst, const float2* __restrict__ tw) {
-    static_assert(N % R == 0, "radix must divide N");
-    constexpr int NB = N / R;
-    constexpr int TOTAL = L * NB;
-    constexpr int ITER = (TOTAL + T - 1) / T;
-    if constexpr (INPLACE) {
-        float2 v[ITER][R];
-#pragma unroll
-        for (int it = 0; it < ITER; ++it) {
-            const int g = threadIdx.x + it * T;
-            if (TOTAL % T == 0 || g < TOTAL) {
-                int line, b;
-                Map::template map<NB, L>(g, line, b);
-#pragma unroll
-                for (int j = 0; j < R; ++j) v[it][j] = src.load(line, b + j * NB);
-            }
-        }
-        __syncthreads();
-#pragma unroll
-        for (int it = 0; it < ITER; ++it) {
-            const int g = threadIdx.x + it * T;
-            if (TOTAL % T == 0 || g < TOTAL) {
-                int line, b;
-                Map::template map<NB, L>(g, line, b);
-                butterfly<N, R, NS, SIGN>(v[it], b, tw);
-                const int base = (b / NS) * (NS * R) + (b % NS);
-#pragma unroll
-                for (int j = 0; j < R; ++j) dst.store(line, base + j * NS, v[it][j]);
-            }
-        }
-    } else {
-#pragma unroll
-        for (int it = 0; it < ITER; ++it) {
-            const int g = threadIdx.x + it * T;
-            if (TOTAL % T == 0 || g < TOTAL) {
-                int line, b;
-                Map::template map<NB, L>(g, line, b);
-                float2 v[R];
-#pragma unroll
-                for (int j = 0; j < R; ++j) v[j] = src.load(line, b + j * NB);
-                butterfly<N, R, NS, SIGN>(v, b, tw);
-                const int base = (b / NS) * (NS * R) + (b % NS);
-#pragma unroll
-                for (int j = 0; j < R; ++j) dst.store(line, base + j * NS, v[j]);
-            }
-        }
+    // element n of the transform in natural order: the slot stage 2 read it from
+    // (u = n mod R0, v = n / R0), so stage 2 may write its outputs back in place
+    __device__ __forceinline__ float2& nat(int line, int n) const { return at(line, n % R0, n / R0); }
+    __device__ __forceinline__ void store(int line, int n, float2 v) const { nat(line, n) = v; }
+};
+// Exchange buffer for a panel of P columns: element (u, v) of column c at
+// (v*(R0+PAD) + u)*P + c, so a warp's 8-byte accesses span all 32 banks.
+template <int R0, int R1, int PAD, int P>
+struct ColXchg {
+    float2* s;
+    __device__ __forceinline__ float2& at(int line, int u, int v) const {
+        return s[(v * (R0 + PAD) + u) * P + line];
     }
-}
+};
 
-// A length-N transform as a list of radices (applied left to right).
+// Stage-2 twiddle table layout: tw2[b*(R1-1) + (j-1)] = w_N^{-j b}, b < R0, 1 <= j < R1.
+template <int R0, int R1>
+struct Tw2 {
+    static constexpr int SIZE = R0 * (R1 - 1);
+};
+
+struct NoMid {
+    __device__ __forceinline__ void operator()() const {}
+};
+
 template <int N_, int... Rs>
 struct Radix {
     static constexpr int N = N_;
     static constexpr int count = sizeof...(Rs);
 };
 
-template <class RX, int SIGN, int L, int T, class Map, bool LAST_INPLACE>
+template <class RX, int SIGN, int L, int T, class Map, bool TW_SMEM = false>
 struct FftRun;
 
-template <int N, int R0, int SIGN, int L, int T, class Map, bool LAST_INPLACE>
-struct FftRun<Radix<N, R0>, SIGN, L, T, Map, LAST_INPLACE> {
-    template <class Src, class Sm, class Dst>
-    static __device__ __forceinline__ void run(const Src& src, Sm& sm, Dst& dst, const float2* tw) {
-        static_assert(N == R0, "single-stage plan");
-        fft_stage<N, R0, 1, SIGN, L, T, Map, false>(src, dst, tw);
+// One stage: N = R0, no twiddles, source -> destination.
+template <int N, int R0, int SIGN, int L, int T, class Map, bool TW_SMEM>
+struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM> {
+    static_assert(N == R0, "single-stage plan");
+    static constexpr int R1 = 1;
+    template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid>
+    static __device__ __forceinline__ void run(const Src& src, const Xc&, Dst& dst,
+                                               const float2* __restrict__, const Mid& mid = Mid()) {
+        // one butterfly per line (the source is consumed inside the loop; `mid` runs after it)
+        constexpr int TOTAL = L;
+        constexpr int ITER = (TOTAL + T - 1) / T;
+#pragma unroll
+        for (int it = 0; it < ITER; ++it) {
+            const int g = threadIdx.x + it * T;
+            if (TOTAL % T == 0 || g < TOTAL) {
+                const int line = g;
+                float2 v[R0];
+#pragma unroll
+                for (int j = 0; j < R0; ++j) v[j] = src.load(line, j);
+                Dft<R0, SIGN>::run(v);
+#pragma unroll
+                for (int j = 0; j < R0; ++j) dst.store(line, j, v[j]);
+            }
+        }
+        __syncthreads();
+        mid();
     }
 };
 
-template <int N, int R0, int R1, int SIGN, int L, int T, class Map, bool LAST_INPLACE>
-struct FftRun<Radix<N, R0, R1>, SIGN, L, T, Map, LAST_INPLACE> {
-    template <class Src, class Sm, class Dst>
-    static __device__ __forceinline__ void run(const Src& src, Sm& sm, Dst& dst, const float2* tw) {
-        static_assert(N == R0 * R1, "radices must multiply to N");
-        fft_stage<N, R0, 1, SIGN, L, T, Map, false>(src, sm, tw);
-        __syncthreads();
-        fft_stage<N, R1, R0, SIGN, L, T, Map, LAST_INPLACE>(sm, dst, tw);
+// Two stages: N = R0 * R1, one exchange through shared memory.
+template <int N, int R0_, int R1_, int SIGN, int L, int T, class Map, bool TW_SMEM>
+struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
+    static constexpr int R0 = R0_, R1 = R1_;
+    static_assert(N == R0 * R1, "radices must multiply to N");
+    // Stage 1: radix R0 over R1 butterflies per line, source -> exchange.  IN_PLACE: the
+    // source is the exchange buffer itself (a landing buffer reused as the exchange), so
+    // every thread loads all of its butterflies before a barrier, then computes and stores.
+    template <bool IN_PLACE, class Src, class Xc>
+    static __device__ __forceinline__ void stage1(const Src& src, const Xc& xc) {
+        constexpr int TOTAL = L * R1;
+        constexpr int ITER = (TOTAL + T - 1) / T;
+        if constexpr (IN_PLACE) {
+            float2 v[ITER][R0];
+#pragma unroll
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    int line, b;
+                    Map::template map<R1, L>(g, line, b);
+#pragma unroll
+                    for (int j = 0; j < R0; ++j) v[it][j] = src.load(line, b + j * R1);
+                }
+            }
+            __syncthreads();
+#pragma unroll
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    int line, b;
+                    Map::template map<R1, L>(g, line, b);
+                    Dft<R0, SIGN>::run(v[it]);
+#pragma unroll
+                    for (int j = 0; j < R0; ++j) xc.at(line, j, b) = v[it][j];
+                }
+            }
+        } else {
+#pragma unroll
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    int line, b;
+                    Map::template map<R1, L>(g, line, b);
+                    float2 v[R0];
+#pragma unroll
+                    for (int j = 0; j < R0; ++j) v[j] = src.load(line, b + j * R1);
+                    Dft<R0, SIGN>::run(v);
+#pragma unroll
+                    for (int j = 0; j < R0; ++j) xc.at(line, j, b) = v[j];
+                }
+            }
+        }
     }
-};
 
-template <int N, int R0, int R1, int R2, int SIGN, int L, int T, class Map, bool LAST_INPLACE>
-struct FftRun<Radix<N, R0, R1, R2>, SIGN, L, T, Map, LAST_INPLACE> {
-    template <class Src, class Sm, class Dst>
-    static __device__ __forceinline__ void run(const Src& src, Sm& sm, Dst& dst, const float2* tw) {
-        static_assert(N == R0 * R1 * R2, "radices must multiply to N");
-        fft_stage<N, R0, 1, SIGN, L, T, Map, false>(src, sm, tw);
+    // `mid` runs (in every thread) after the barrier that ends stage 1, i.e. once the
+    // source has been fully consumed: persistent kernels prefetch their next input there.
+    template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid>
+    static __device__ __forceinline__ void run(const Src& src, const Xc& xc, Dst& dst,
+                                               const float2* __restrict__ tw2,
+                                               const Mid& mid = Mid()) {
+        stage1<IN_PLACE>(src, xc);
         __syncthreads();
-        fft_stage<N, R1, R0, SIGN, L, T, Map, true>(sm, sm, tw);
-        __syncthreads();
-        fft_stage<N, R2, R0 * R1, SIGN, L, T, Map, LAST_INPLACE>(sm, dst, tw);
+        mid();
+        {   // stage 2: radix R1 over R0 butterflies per line, exchange -> destination
+            constexpr int TOTAL = L * R0;
+            constexpr int ITER = (TOTAL + T - 1) / T;
+#pragma unroll
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    int line, b;
+                    Map::template map<R0, L>(g, line, b);
+                    float2 v[R1];
+#pragma unroll
+                    for (int j = 0; j < R1; ++j) v[j] = xc.at(line, b, j);
+                    const float2* tw = tw2 + b * (R1 - 1);
+#pragma unroll
+                    for (int j = 1; j < R1; ++j) {
+                        const float2 w = TW_SMEM ? tw[j - 1] : __ldg(tw + (j - 1));
+                        v[j] = SIGN < 0 ? cmul(v[j], w) : cmulc(v[j], w);
+                    }
+                    Dft<R1, SIGN>::run(v);
+#pragma unroll
+                    for (int j = 0; j < R1; ++j) dst.store(line, b + j * R0, v[j]);
+                }
+            }
+        }
     }
 };
 

@@ -2,27 +2,32 @@
 //
 // Data layout in HBM:
 //   raw   uint16 [tiles][H][W]           W contiguous (the caller's tile layout)
-//   spec  float2 [tiles][H][WP]          half spectrum kx in [0, W/2], WP = pad16(W/2+1),
-//                                        resident for reuse by <= 4 pairs
+//   G     float2 [chunk][H][WP]          row-transformed tiles of a forward chunk (L2-sized)
+//   spec  u32    [tiles][H][WP]          resident half spectrum kx in [0, W/2] (WP = pad16(W/2+1))
+//                                        stored as its phase code (31-bit turn + nonzero flag),
+//                                        reused by <= 4 pairs
 //   Q     float2 [chunk][H][WP]          per-pair column-inverse intermediate (L2-sized chunk)
 //   keys  u64    [pairs]                 packed (|c| bits << 32 | ~index) argmax per pair
 //   mom   u64    [pairs][4][5]           exact integer CCF moments per candidate
 //
 // Kernels (one launch covers a chunk of tiles or pairs):
-//   K1 fwd_rows   raw -> spec   R2C along x: length-W real row as a W/2 complex FFT + post-twiddle
+//   K1 fwd_rows   raw -> G      R2C along x: length-W real row as a W/2 complex FFT + post-twiddle
 //                               (step 2 first half; uint16->fp32 fused into the load)
-//   K2 fwd_cols   spec -> spec  C2C along y, in place on column panels (step 2 second half)
-//   K3 pair_cols  2 spec -> Q   NCPS F_A conj(F_B)/|..| fused into the loads (step 3), then the
-//                               inverse C2C along y (step 4 first half)
+//   K2 fwd_cols   G -> spec     C2C along y on TMA-landed column panels (step 2 second half),
+//                               epilogue: phase code
+//   K3 pair_cols  2 spec -> Q   NCPS exp(i(phi_A - phi_B)) from two TMA-landed phase panels
+//                               (step 3), then the inverse C2C along y (step 4 first half)
 //   K4 pair_rows  Q -> keys     C2R along x (step 4 second half) with |.| + argmax fused in the
 //                               epilogue; the real correlation surface is never stored (step 5)
 //   K5 ccf_mom    raw -> mom    integer moments of the 4 candidate overlaps (step 6, Fig. 3)
 //   K6 finalize   mom -> pairs  CCF in fp64 from exact int128 moments, candidate selection (step 7)
 #pragma once
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>
 
+#include "async_copy.cuh"
 #include "fft_engine.cuh"
 #include "../../include/stitch.h"
 
@@ -30,9 +35,18 @@ namespace stitch {
 
 constexpr int pad16(int x) { return (x + 15) / 16 * 16; }
 
+template <class RX> struct RadixInfo;
+template <int N, int R0_> struct RadixInfo<Radix<N, R0_>> {
+    static constexpr int R0 = R0_, R1 = 1, STAGES = 1;
+};
+template <int N, int R0_, int R1_> struct RadixInfo<Radix<N, R0_, R1_>> {
+    static constexpr int R0 = R0_, R1 = R1_, STAGES = 2;
+};
+
 // A compiled tile-size plan: row transform (length W/2 complex) and column
-// transform (length H) radices, CTA shapes.
-template <int W_, int H_, class RowRX, class ColRX, int ROW_L_, int ROW_T_, int COL_P_, int COL_T_>
+// transform (length H) radices, CTA shapes, exchange-buffer padding.
+template <int W_, int H_, class RowRX, class ColRX, int ROW_L_, int ROW_T_, int COL_P_, int COL_T_,
+          int ROW_PAD_, int COL_PAD_>
 struct Plan {
     static constexpr int W = W_, H = H_;
     static constexpr int M = W / 2;           // complex row length
@@ -40,11 +54,37 @@ struct Plan {
     static constexpr int WP = pad16(WC);      // row pitch of spectra (float2)
     using Row = RowRX;
     using Col = ColRX;
+    using RI = RadixInfo<RowRX>;
+    using CI = RadixInfo<ColRX>;
     static constexpr int ROW_L = ROW_L_, ROW_T = ROW_T_;
     static constexpr int COL_P = COL_P_, COL_T = COL_T_;
-    static constexpr int ROW_STRIDE = WC + (WC >> 4) + 1;   // padded smem line (RowSmem)
-    static constexpr size_t ROW_SMEM = sizeof(float2) * ROW_L * ROW_STRIDE;
-    static constexpr size_t COL_SMEM = sizeof(float2) * COL_P * H;
+    static constexpr int ROW_PAD = ROW_PAD_, COL_PAD = COL_PAD_;
+    using RowX = RowXchg<RI::R0, RI::R1, ROW_PAD>;
+    using ColX = ColXchg<CI::R0, CI::R1, COL_PAD, COL_P>;
+    static constexpr size_t ROW_SMEM = sizeof(float2) * ROW_L * RowX::LSTRIDE;
+    // column kernels: a TMA landing panel [H][COL_P] (complex, or two phase panels), reused
+    // in place as the stage exchange buffer once stage 1 has read it into registers
+    // K3 lands two phase panels: the second starts 128-byte aligned (TMA destination rule)
+    static constexpr size_t COL_PHASE_B = (sizeof(uint32_t) * COL_P * H + 127) / 128 * 128;
+    static constexpr size_t COL_LAND_C = sizeof(float2) * COL_P * H;
+    static constexpr size_t COL_LAND_P = COL_PHASE_B + sizeof(uint32_t) * COL_P * H;
+    static constexpr size_t COL_LAND = COL_LAND_C > COL_LAND_P ? COL_LAND_C : COL_LAND_P;
+    static constexpr size_t COL_XCH =
+        CI::STAGES == 1 ? 0 : sizeof(float2) * COL_P * CI::R1 * (CI::R0 + COL_PAD);
+    static constexpr size_t COL_SMEM = COL_LAND > COL_XCH ? COL_LAND : COL_XCH;
+    static constexpr int BOXH = H / ((H + 255) / 256);   // TMA box rows (<= 256)
+    static_assert(H % BOXH == 0, "H must split into equal TMA boxes of <= 256 rows");
+    static_assert((BOXH * COL_P * 4) % 128 == 0 || H == BOXH, "TMA boxes must land 128-B aligned");
+    // CTAs per SM the column kernels are register-budgeted for (shared memory allows this many)
+    static constexpr int COL_MINB_RAW = (int)((220 * 1024) / (COL_SMEM + 1024));
+    static constexpr int COL_MINB = COL_MINB_RAW > 3 ? 3 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
+    // register cap so COL_MINB CTAs of COL_T threads fit the 64K-register file (8-register units)
+    static constexpr int COL_WARPS = (COL_T + 31) / 32;
+    static constexpr int COL_MAXREG_RAW = (65536 / (COL_MINB * COL_WARPS * 32)) / 8 * 8;
+    static constexpr int COL_MAXREG = COL_MAXREG_RAW > 255 ? 255 : COL_MAXREG_RAW;
+    // stage-2 twiddle tables (w_N^{-j b}, see fft_engine.cuh)
+    static constexpr int ROW_TW2 = RI::R0 * (RI::R1 - 1);
+    static constexpr int COL_TW2 = CI::R0 * (CI::R1 - 1);
     static_assert(W % 2 == 0, "W must be even");
     static_assert(Row::N == M && Col::N == H, "plan radices do not match the tile");
     static_assert(H % ROW_L == 0, "rows per CTA must divide H");
@@ -67,87 +107,178 @@ struct U16RowSrc {  // z[n] = x[2n] + i x[2n+1], straight from the uint16 row
 
 template <class PL>
 __global__ void __launch_bounds__(PL::ROW_T) k1_fwd_rows(const uint16_t* __restrict__ raw,
-                                                         float2* __restrict__ spec, int tile0,
-                                                         const float2* __restrict__ twM,
+                                                         float2* __restrict__ G, int tile0,
+                                                         const float2* __restrict__ tw2,
                                                          const float2* __restrict__ twW) {
     extern __shared__ float2 smem[];
     constexpr int L = PL::ROW_L, T = PL::ROW_T, M = PL::M;
     const size_t t = (size_t)tile0 + blockIdx.y;
     const int y0 = blockIdx.x * L;
     U16RowSrc<PL> src{reinterpret_cast<const uint32_t*>(raw + (t * PL::H + y0) * PL::W)};
-    RowSmem<PL::ROW_STRIDE> sm{smem};
-    FftRun<typename PL::Row, -1, L, T, RowMap, true>::run(src, sm, sm, twM);
+    typename PL::RowX xc{smem};
+    // stage 2 writes Z[n] back into the slot it read it from (in place, per thread)
+    FftRun<typename PL::Row, -1, L, T, RowMap>::run(src, xc, xc, tw2);
     __syncthreads();
     // Real-to-complex post-processing, q in [0, M] (Z[M] == Z[0]):
     //   E = (Z[q] + conj Z[M-q]) / 2,  O = (Z[q] - conj Z[M-q]) / (2i),  X[q] = E + w_W^q O
-    float2* out = spec + (t * PL::H + y0) * PL::WP;
-    for (int i = threadIdx.x; i < L * PL::WP; i += T) {
-        const int line = i / PL::WP, q = i - line * PL::WP;
-        float2 X = make_float2(0.f, 0.f);
-        if (q <= M) {
-            const float2 zq = sm.load(line, q == M ? 0 : q);
-            const float2 zm = sm.load(line, q == 0 ? 0 : M - q);
-            const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
-            const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
-            const float2 w = __ldg(&twW[q]);
-            const float2 wo = cmul(w, O);
-            X = make_float2(E.x + wo.x, E.y + wo.y);
+#pragma unroll 1
+    for (int line = 0; line < L; ++line) {
+        float2* out = G + ((size_t)blockIdx.y * PL::H + y0 + line) * PL::WP;
+        for (int q = threadIdx.x; q < PL::WP; q += T) {
+            float2 X = make_float2(0.f, 0.f);
+            if (q <= M) {
+                const float2 zq = xc.nat(line, q == M ? 0 : q);
+                const float2 zm = xc.nat(line, q == 0 ? 0 : M - q);
+                const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
+                const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
+                const float2 wo = cmul(__ldg(&twW[q]), O);
+                X = make_float2(E.x + wo.x, E.y + wo.y);
+            }
+            out[q] = X;
         }
-        out[(size_t)line * PL::WP + q] = X;
     }
 }
 
 // ------------------------------------------------------------------ K2 ----
 template <class PL>
-struct PanelIO {  // a panel of COL_P columns of one [H][WP] array
+struct PanelIO {  // a panel of COL_P columns of one [H][WP] complex array
     float2* p;
     __device__ __forceinline__ float2 load(int line, int n) const { return p[(size_t)n * PL::WP + line]; }
     __device__ __forceinline__ void store(int line, int n, float2 v) const { p[(size_t)n * PL::WP + line] = v; }
 };
 
 template <class PL>
-__global__ void __launch_bounds__(PL::COL_T) k2_fwd_cols(float2* __restrict__ spec, int tile0,
-                                                         const float2* __restrict__ twH) {
-    extern __shared__ float2 smem[];
-    const size_t t = (size_t)tile0 + blockIdx.y;
-    PanelIO<PL> io{spec + t * PL::H * PL::WP + blockIdx.x * PL::COL_P};
-    ColSmem<PL::COL_P> sm{smem};
-    FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, false>::run(io, sm, io, twH);
+struct LandSrc {  // a landed complex panel [H][COL_P] in shared memory
+    const float2* s;
+    __device__ __forceinline__ float2 load(int line, int n) const { return s[n * PL::COL_P + line]; }
+};
+
+// Resident spectrum code: the phase of F in 31-bit fixed point (top bits, 2^32 per turn)
+// plus a nonzero flag (bit 0).  Step 3 needs only phases: F_A conj(F_B) / |F_A conj(F_B)|
+// = exp(i (phi_A - phi_B)), and 0 where F_A or F_B vanishes (reading C4).
+// atan2(y, x) / pi in (-1, 1]: octant reduction + a degree-8 polynomial in t^2 for
+// atan(t)/pi on [0, 1] (coefficients fitted in double, max error 1.6e-7 rad in fp32;
+// the fp32 spectrum's own phase error is ~1e-6 rad).
+__device__ __forceinline__ float atan2_halfturns(float y, float x) {
+    const float ax = fabsf(x), ay = fabsf(y);
+    const float mx = fmaxf(ax, ay), mn = fminf(ax, ay);
+    const float t = mx > 0.f ? __fdividef(mn, mx) : 0.f;
+    const float s = t * t;
+    float p = 0.0009368208120577037f;
+    p = fmaf(p, s, -0.00521085737273097f);
+    p = fmaf(p, s, 0.013704856857657433f);
+    p = fmaf(p, s, -0.023946231231093407f);
+    p = fmaf(p, s, 0.03387756645679474f);
+    p = fmaf(p, s, -0.045206326991319656f);
+    p = fmaf(p, s, 0.06363658607006073f);
+    p = fmaf(p, s, -0.10610226541757584f);
+    p = fmaf(p, s, 0.31830987334251404f);
+    float r = p * t;                       // atan(mn/mx) / pi in [0, 1/4]
+    if (ay > ax) r = 0.5f - r;
+    if (x < 0.f) r = 1.0f - r;
+    return y < 0.f ? -r : r;
 }
 
-// ------------------------------------------------------------------ K3 ----
+__device__ __forceinline__ uint32_t phase_code(float2 v) {
+    const float t = atan2_halfturns(v.y, v.x);                       // [-1, 1]
+    const int32_t q = __float2int_rn(t * 2147483648.0f);            // saturates at t = 1
+    return ((uint32_t)q & ~1u) | ((v.x != 0.f || v.y != 0.f) ? 1u : 0u);
+}
+
 template <class PL>
-struct NcpsSrc {  // step 3: NCC = F_A conj(F_B) / |F_A conj(F_B)|, 0 where it vanishes
-    const float2* a;
-    const float2* b;
-    __device__ __forceinline__ float2 load(int line, int n) const {
-        const float2 fa = a[(size_t)n * PL::WP + line];
-        const float2 fb = b[(size_t)n * PL::WP + line];
-        // |F_A conj F_B| = |F_A| |F_B|: normalise each factor first so no
-        // intermediate exceeds |F|^2 (<= ~1e22, safely inside fp32).
-        const float ma = fmaf(fa.x, fa.x, fa.y * fa.y);
-        const float mb = fmaf(fb.x, fb.x, fb.y * fb.y);
-        const float ra = ma > 0.f ? rsqrtf(ma) : 0.f;
-        const float rb = mb > 0.f ? rsqrtf(mb) : 0.f;
-        const float ax = fa.x * ra, ay = fa.y * ra, bx = fb.x * rb, by = fb.y * rb;
-        return make_float2(fmaf(ax, bx, ay * by), fmaf(ay, bx, -ax * by));
+struct PhaseDst {  // K2 output: phase codes of a panel of the resident spectrum
+    uint32_t* p;
+    __device__ __forceinline__ void store(int line, int n, float2 v) const {
+        p[(size_t)n * PL::WP + line] = phase_code(v);
     }
 };
 
 template <class PL>
-__global__ void __launch_bounds__(PL::COL_T) k3_pair_cols(const float2* __restrict__ spec,
-                                                          float2* __restrict__ Q,
-                                                          const PairIdx* __restrict__ pairs,
-                                                          int pair0,
-                                                          const float2* __restrict__ twH) {
-    extern __shared__ float2 smem[];
+__device__ __forceinline__ void tma_panel(void* land, const CUtensorMap* map, int x, int row0,
+                                          int elem_bytes, uint64_t* bar) {
+    // one panel = H rows of COL_P elements, in boxes of BOXH rows
+    char* d = reinterpret_cast<char*>(land);
+#pragma unroll 1
+    for (int y = 0; y < PL::H; y += PL::BOXH)
+        tma_load_2d(d + (size_t)y * PL::COL_P * elem_bytes, map, x, row0 + y, bar);
+}
+
+// K2: column FFT of a chunk of row-transformed tiles (G, complex, L2-resident), panel of
+// COL_P columns landed by TMA; writes the resident phase spectrum (or, for the test hook,
+// the complex spectrum back into G).
+template <class PL, bool PHASE_OUT>
+__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
+    k2t_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
+                 uint32_t* __restrict__ spec, int tile0, const float2* __restrict__ tw2) {
+    extern __shared__ __align__(128) unsigned char csmem[];
+    __shared__ uint64_t bar;
+    const int tl = blockIdx.y, c0 = blockIdx.x * PL::COL_P;
+    if (threadIdx.x == 0) {
+        prefetch_tensormap(&tmG);
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C);
+        tma_panel<PL>(csmem, &tmG, 2 * c0, tl * PL::H, 8, &bar);
+    }
+    mbar_wait(&bar, 0);
+    LandSrc<PL> src{reinterpret_cast<const float2*>(csmem)};
+    typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
+    if constexpr (PHASE_OUT) {
+        PhaseDst<PL> dst{spec + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
+        FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap>::template run<true>(src, xc, dst,
+                                                                                       tw2);
+    } else {
+        PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
+        FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap>::template run<true>(src, xc, dst,
+                                                                                       tw2);
+    }
+}
+
+// ------------------------------------------------------------------ K3 ----
+template <class PL>
+struct NcpsPhaseSrc {  // step 3 from two landed phase panels: exp(i (phi_A - phi_B)) or 0
+    const uint32_t* a;
+    const uint32_t* b;
+    __device__ __forceinline__ float2 load(int line, int n) const {
+        const uint32_t ua = a[n * PL::COL_P + line], ub = b[n * PL::COL_P + line];
+        const uint32_t d = ua - ub;   // phase difference, wraps mod one turn (flag bits cancel)
+        const float x = (float)(int32_t)d * 1.46291807926715968e-9f;   // 2 pi / 2^32, [-pi, pi)
+        float sn, cs;
+        __sincosf(x, &sn, &cs);
+        return (ua & ub & 1u) ? make_float2(cs, sn) : make_float2(0.f, 0.f);
+    }
+};
+
+template <class PL>
+__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
+    k3t_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
+                  const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2) {
+    extern __shared__ __align__(128) unsigned char csmem[];
+    __shared__ uint64_t bar;
     const PairIdx pr = pairs[pair0 + blockIdx.y];
     const int c0 = blockIdx.x * PL::COL_P;
-    const size_t img = (size_t)PL::H * PL::WP;
-    NcpsSrc<PL> src{spec + pr.a * img + c0, spec + pr.b * img + c0};
-    PanelIO<PL> dst{Q + blockIdx.y * img + c0};
-    ColSmem<PL::COL_P> sm{smem};
-    FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, false>::run(src, sm, dst, twH);
+    uint32_t* la = reinterpret_cast<uint32_t*>(csmem);
+    uint32_t* lb = reinterpret_cast<uint32_t*>(csmem + PL::COL_PHASE_B);
+    if (threadIdx.x == 0) {
+        prefetch_tensormap(&tmS);
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        mbar_arrive_expect_tx(&bar, (uint32_t)(2 * PL::H * PL::COL_P * 4));
+        tma_panel<PL>(la, &tmS, c0, pr.a * PL::H, 4, &bar);
+        tma_panel<PL>(lb, &tmS, c0, pr.b * PL::H, 4, &bar);
+    }
+    mbar_wait(&bar, 0);
+    NcpsPhaseSrc<PL> src{la, lb};
+    PanelIO<PL> dst{Q + (size_t)blockIdx.y * PL::H * PL::WP + c0};
+    typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
+    FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap>::template run<true>(src, xc, dst,
+                                                                                   tw2);
 }
 
 // ------------------------------------------------------------------ K4 ----
@@ -162,35 +293,44 @@ struct C2RSrc {  // complex-to-real pre-processing of row X[0..M] into Z[0..M)
         // E = X[n] + conj X[M-n];  O = (X[n] - conj X[M-n]) e^{+2 pi i n / W};  Z = E + i O
         const float2 w = __ldg(&twW[n]);
         const float2 d = make_float2(xn.x - xm.x, xn.y + xm.y);
-        const float2 o = make_float2(fmaf(d.x, w.x, d.y * w.y), fmaf(d.y, w.x, -d.x * w.y));
+        const float2 o = cmulc(d, w);
         return make_float2(xn.x + xm.x - o.y, xn.y - xm.y + o.x);
     }
 };
 
 struct ArgmaxDst {  // step 5: running max of |x| with its row-major index, never stored
-    unsigned long long best;
-    int row_base;  // (y0 + line) * W added per line
+    float best_v;      // largest |x| seen by this thread (>= 0; -1 before the first value)
+    uint32_t best_i;   // its row-major index y*W + x (smallest index among equal values)
+    int row_base;      // y0 of the CTA's first line
     int W;
+    __device__ __forceinline__ void take(float a, uint32_t idx) {
+        if (a > best_v || (a == best_v && idx < best_i)) {
+            best_v = a;
+            best_i = idx;
+        }
+    }
     __device__ __forceinline__ void store(int line, int n, float2 v) {
         const uint32_t idx = (uint32_t)((row_base + line) * W + 2 * n);
-        const unsigned long long k0 =
-            ((unsigned long long)__float_as_uint(fabsf(v.x)) << 32) | (0xFFFFFFFFu - idx);
-        const unsigned long long k1 =
-            ((unsigned long long)__float_as_uint(fabsf(v.y)) << 32) | (0xFFFFFFFFu - (idx + 1));
-        best = max(best, max(k0, k1));
+        take(fabsf(v.x), idx);       // x[2n]
+        take(fabsf(v.y), idx + 1);   // x[2n+1]
+    }
+    // packed key: larger |x| wins, then the smaller index (reading C6)
+    __device__ __forceinline__ unsigned long long key() const {
+        if (best_v < 0.f) return 0ull;
+        return ((unsigned long long)__float_as_uint(best_v) << 32) | (0xFFFFFFFFu - best_i);
     }
 };
 
 template <int T>
 __device__ __forceinline__ unsigned long long block_max_u64(unsigned long long v) {
-    __shared__ unsigned long long red[T / 32];
+    __shared__ unsigned long long red[(T + 31) / 32];
 #pragma unroll
     for (int o = 16; o > 0; o >>= 1) v = max(v, __shfl_xor_sync(0xFFFFFFFFu, v, o));
     const int w = threadIdx.x >> 5;
     if ((threadIdx.x & 31) == 0) red[w] = v;
     __syncthreads();
     if (threadIdx.x < 32) {
-        v = threadIdx.x < T / 32 ? red[threadIdx.x] : 0ull;
+        v = threadIdx.x < (T + 31) / 32 ? red[threadIdx.x] : 0ull;
 #pragma unroll
         for (int o = 16; o > 0; o >>= 1) v = max(v, __shfl_xor_sync(0xFFFFFFFFu, v, o));
     }
@@ -201,24 +341,210 @@ template <class PL>
 __global__ void __launch_bounds__(PL::ROW_T) k4_pair_rows(const float2* __restrict__ Q,
                                                           unsigned long long* __restrict__ keys,
                                                           int pair0,
-                                                          const float2* __restrict__ twM,
+                                                          const float2* __restrict__ tw2,
                                                           const float2* __restrict__ twW) {
     extern __shared__ float2 smem[];
     constexpr int L = PL::ROW_L, T = PL::ROW_T;
     const int y0 = blockIdx.x * L;
     C2RSrc<PL> src{Q + ((size_t)blockIdx.y * PL::H + y0) * PL::WP, twW};
-    ArgmaxDst dst{0ull, y0, PL::W};
-    RowSmem<PL::ROW_STRIDE> sm{smem};
-    FftRun<typename PL::Row, +1, L, T, RowMap, false>::run(src, sm, dst, twM);
-    const unsigned long long best = block_max_u64<T>(dst.best);
+    ArgmaxDst dst{-1.f, 0xFFFFFFFFu, y0, PL::W};
+    typename PL::RowX xc{smem};
+    FftRun<typename PL::Row, +1, L, T, RowMap>::run(src, xc, dst, tw2);
+    const unsigned long long best = block_max_u64<T>(dst.key());
     if (threadIdx.x == 0) atomicMax(&keys[pair0 + blockIdx.y], best);
 }
 
+// ------------------------------------------------ persistent row kernels ----
+// K1p / K4p: persistent CTAs walk the row blocks of a chunk (static round robin).  A
+// block's input rows land in shared memory by TMA bulk copy (cp.async.bulk + mbarrier);
+// the copy for block k+1 is issued as soon as stage 1 of block k has consumed the
+// landing buffer, so it overlaps stage 2 / the epilogue of block k and the other CTAs
+// on the SM.  Stage-2 twiddle tables live in shared memory.
+template <class PL>
+struct RowPersist {
+    static constexpr int L = PL::ROW_L;
+    static constexpr int LP = PL::WP + 8;            // padded landing pitch (float2), 16-B rows
+    static constexpr int RAWB = L * PL::W * 2;       // raw landing bytes per block (K1)
+    static constexpr int QB = L * PL::WP * 8;        // Q landing bytes per block (K4, copied row by row)
+    static constexpr int XCH = L * PL::RowX::LSTRIDE;  // exchange float2
+    static constexpr int TW2 = PL::ROW_TW2 > 0 ? PL::ROW_TW2 : 1;
+    static constexpr int TWW = PL::M + 1;
+    // byte offsets in dynamic shared memory
+    static constexpr size_t OFF_BAR = 0;                              // 2 x u64
+    static constexpr size_t OFF_TW2 = 16;
+    static constexpr size_t OFF_TWW = OFF_TW2 + (size_t)TW2 * 8;
+    static constexpr size_t OFF_XCH = (OFF_TWW + (size_t)TWW * 8 + 15) / 16 * 16;
+    static constexpr size_t OFF_LAND = OFF_XCH + (size_t)XCH * 8;
+    static constexpr size_t LAND_K1 = ((size_t)RAWB + 15) / 16 * 16;
+    static constexpr size_t LAND_K4 = (size_t)L * LP * 8;
+    static constexpr size_t SMEM_K1 = OFF_LAND + LAND_K1;
+    // K4 keeps w_W in global memory (L1) so three CTAs fit an SM
+    static constexpr size_t OFF_XCH4 = (OFF_TW2 + (size_t)TW2 * 8 + 15) / 16 * 16;
+    static constexpr size_t OFF_LAND4 = OFF_XCH4 + (size_t)XCH * 8;
+    static constexpr size_t SMEM_K4 = OFF_LAND4 + LAND_K4;
+    static constexpr bool K1_BULK = (PL::W * 2) % 16 == 0;   // raw rows 16-byte aligned
+};
+
+template <class PL>
+__device__ __forceinline__ void load_row_tables(float2* tw2s, float2* twWs, const float2* tw2,
+                                                const float2* twW) {
+    for (int i = threadIdx.x; i < PL::ROW_TW2; i += PL::ROW_T) tw2s[i] = __ldg(tw2 + i);
+    for (int i = threadIdx.x; i <= PL::M; i += PL::ROW_T) twWs[i] = __ldg(twW + i);
+}
+
+template <class PL>
+struct U16SmemSrc {  // z[n] = x[2n] + i x[2n+1] from a landed raw row block
+    const uint32_t* p;
+    __device__ __forceinline__ float2 load(int line, int n) const {
+        const uint32_t u = p[line * (PL::W / 2) + n];
+        return make_float2((float)(u & 0xFFFFu), (float)(u >> 16));
+    }
+};
+
+template <class PL>
+__global__ void __launch_bounds__(PL::ROW_T) k1p_fwd_rows(const uint16_t* __restrict__ raw,
+                                                          float2* __restrict__ G, int tile0,
+                                                          int ntiles,
+                                                          const float2* __restrict__ tw2,
+                                                          const float2* __restrict__ twW) {
+    using RP = RowPersist<PL>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    constexpr int L = PL::ROW_L, T = PL::ROW_T, M = PL::M, BPT = PL::H / L;
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + RP::OFF_BAR);
+    float2* tw2s = reinterpret_cast<float2*>(smem_raw + RP::OFF_TW2);
+    float2* twWs = reinterpret_cast<float2*>(smem_raw + RP::OFF_TWW);
+    typename PL::RowX xc{reinterpret_cast<float2*>(smem_raw + RP::OFF_XCH)};
+    unsigned char* land = smem_raw + RP::OFF_LAND;
+    const int nblk = ntiles * BPT;
+    auto issue = [&](int blk, int buf) {
+        const int tl = blk / BPT, y0 = (blk - tl * BPT) * L;
+        const uint16_t* src = raw + ((size_t)(tile0 + tl) * PL::H + y0) * PL::W;
+        mbar_arrive_expect_tx(&bar[buf], RP::RAWB);
+        bulk_g2s(land, src, RP::RAWB, &bar[buf]);
+    };
+    if (threadIdx.x == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        fence_mbar_init();
+    }
+    load_row_tables<PL>(tw2s, twWs, tw2, twW);
+    __syncthreads();
+    // One landing buffer: block k+1's rows are fetched (TMA bulk copy) as soon as stage 1
+    // of block k has consumed them, overlapping stage 2 + post-processing of block k.
+    if (threadIdx.x == 0 && (int)blockIdx.x < nblk) issue(blockIdx.x, 0);
+    int k = 0;
+    for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++k) {
+        mbar_wait(&bar[0], k & 1);
+        const int tl = blk / BPT, y0 = (blk - tl * BPT) * L;
+        const int nxt = blk + gridDim.x;
+        U16SmemSrc<PL> src{reinterpret_cast<const uint32_t*>(land)};
+        auto prefetch = [&]() {
+            if (threadIdx.x == 0 && nxt < nblk) {
+                fence_proxy_async();
+                issue(nxt, 0);
+            }
+        };
+        FftRun<typename PL::Row, -1, L, T, RowMap, true>::run(src, xc, xc, tw2s, prefetch);
+        __syncthreads();
+        float2* out0 = G + ((size_t)tl * PL::H + y0) * PL::WP;
+#pragma unroll 1
+        for (int line = 0; line < L; ++line) {
+            float2* out = out0 + (size_t)line * PL::WP;
+            for (int q = threadIdx.x; q < PL::WP; q += T) {
+                float2 X = make_float2(0.f, 0.f);
+                if (q <= M) {
+                    const float2 zq = xc.nat(line, q == M ? 0 : q);
+                    const float2 zm = xc.nat(line, q == 0 ? 0 : M - q);
+                    const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
+                    const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
+                    const float2 wo = cmul(twWs[q], O);
+                    X = make_float2(E.x + wo.x, E.y + wo.y);
+                }
+                out[q] = X;
+            }
+        }
+        __syncthreads();   // exchange free
+    }
+}
+
+template <class PL>
+struct C2RSmemSrc {  // C2R pre-processing from a landed Q row block (pitch LP)
+    const float2* rows;
+    const float2* twW;
+    __device__ __forceinline__ float2 load(int line, int n) const {
+        const float2* r = rows + line * RowPersist<PL>::LP;
+        const float2 xn = r[n];
+        const float2 xm = r[PL::M - n];
+        const float2 d = make_float2(xn.x - xm.x, xn.y + xm.y);
+        const float2 o = cmulc(d, __ldg(twW + n));   // global table (L1-resident)
+        return make_float2(xn.x + xm.x - o.y, xn.y - xm.y + o.x);
+    }
+};
+
+template <class PL>
+__global__ void __launch_bounds__(PL::ROW_T) k4p_pair_rows(const float2* __restrict__ Q,
+                                                           unsigned long long* __restrict__ keys,
+                                                           int pair0, int npairs,
+                                                           const float2* __restrict__ tw2,
+                                                           const float2* __restrict__ twW) {
+    using RP = RowPersist<PL>;
+    extern __shared__ __align__(16) unsigned char smem_raw[];
+    constexpr int L = PL::ROW_L, T = PL::ROW_T, BPP = PL::H / L;
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + RP::OFF_BAR);
+    float2* tw2s = reinterpret_cast<float2*>(smem_raw + RP::OFF_TW2);
+    typename PL::RowX xc{reinterpret_cast<float2*>(smem_raw + RP::OFF_XCH4)};
+    float2* land = reinterpret_cast<float2*>(smem_raw + RP::OFF_LAND4);
+    const int nblk = npairs * BPP;
+    auto issue = [&](int blk, int buf) {
+        const int pl = blk / BPP, y0 = (blk - pl * BPP) * L;
+        const float2* src = Q + ((size_t)pl * PL::H + y0) * PL::WP;
+        mbar_arrive_expect_tx(&bar[buf], RP::QB);
+#pragma unroll
+        for (int line = 0; line < L; ++line)
+            bulk_g2s(land + line * RP::LP, src + (size_t)line * PL::WP, PL::WP * 8, &bar[buf]);
+    };
+    if (threadIdx.x == 0) {
+        mbar_init(&bar[0], 1);
+        mbar_init(&bar[1], 1);
+        fence_mbar_init();
+    }
+    for (int i = threadIdx.x; i < PL::ROW_TW2; i += T) tw2s[i] = __ldg(tw2 + i);
+    __syncthreads();
+    // One landing buffer, refilled (TMA bulk copies) as soon as stage 1 consumed it.
+    if (threadIdx.x == 0 && (int)blockIdx.x < nblk) issue(blockIdx.x, 0);
+    int k = 0;
+    for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++k) {
+        mbar_wait(&bar[0], k & 1);
+        const int pl = blk / BPP, y0 = (blk - pl * BPP) * L;
+        const int nxt = blk + gridDim.x;
+        C2RSmemSrc<PL> src{land, twW};
+        ArgmaxDst dst{-1.f, 0xFFFFFFFFu, y0, PL::W};
+        auto prefetch = [&]() {
+            if (threadIdx.x == 0 && nxt < nblk) {
+                fence_proxy_async();
+                issue(nxt, 0);
+            }
+        };
+        FftRun<typename PL::Row, +1, L, T, RowMap, true>::run(src, xc, dst, tw2s, prefetch);
+        const unsigned long long best = block_max_u64<T>(dst.key());
+        if (threadIdx.x == 0) atomicMax(&keys[pair0 + pl], best);
+        __syncthreads();   // exchange and reduction scratch free
+    }
+}
+
 // ------------------------------------------------------------------ K5 ----
-// Rows of the four candidate overlaps of pair p, concatenated (2H rows in all):
-//   c1 (dx,dy)=(x,y): H-y rows | c2 (W-x,y): H-y | c3 (x,H-y): y | c4 (W-x,H-y): y
-// region a = A[dy:H, dx:W], b = B[0:H-dy, 0:W-dx] (Fig. 2 l.8-11 unified, Fig. 3).
-constexpr int CCF_ROWS = 8;
+// Candidate overlaps of pair p (Fig. 2 l.8-11 unified, Fig. 3): candidate (dx, dy) has
+// region a = A[dy:H, dx:W], b = B[0:H-dy, 0:W-dx].  c1 = (x, y) and c2 = (W-x, y) share
+// their rows (dy = y: A rows y.., B rows 0..H-y-1), and so do c3 = (x, H-y) and
+// c4 = (W-x, H-y) (dy = H-y).  Row group g (0: c1/c2, 1: c3/c4) is cut into blocks of
+// CCF_ROWS rows; a CTA stages CCF_BATCH rows of A and B at a time in shared memory
+// (aligned 16-byte loads: each tile row is read once for both candidates) and every
+// B pixel b = B[i][j] is paired with both of its partners
+//   candidate dx = x   : a = A[dy+i][x + j],      j <  W - x
+//   candidate dx = W-x : a = A[dy+i][W - x + j],  j <  x
+// accumulating the exact integer moments Sa, Sb, Saa, Sbb, Sab (u32 / u64 wide MADs).
+constexpr int CCF_ROWS = 64;   // rows of one group per CTA
+constexpr int CCF_BATCH = 8;   // rows staged in shared memory at a time (one warp per row)
 constexpr int CCF_T = 256;
 
 __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v) {
@@ -227,66 +553,106 @@ __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
     return v;
 }
 
+struct Moments {
+    uint32_t sa = 0, sb = 0;  // <= CCF_ROWS/CCF_BATCH * ceil(W/32) * 65535 < 2^32 per lane
+    unsigned long long saa = 0, sbb = 0, sab = 0;
+    __device__ __forceinline__ void add(uint32_t a, uint32_t b) {
+        sa += a;
+        sb += b;
+        saa += (unsigned long long)a * a;
+        sbb += (unsigned long long)b * b;
+        sab += (unsigned long long)a * b;
+    }
+};
+
+// Moments of one candidate over one staged row: a = ar[off + j], b = br[j], j < w.
+// Lane l takes j = l + 32k (conflict-free 2-byte shared loads), unrolled by 4.
+__device__ __forceinline__ void row_moments(Moments& m, const uint16_t* ar, const uint16_t* br,
+                                            int off, int w, int lane) {
+    const uint16_t* a = ar + off + lane;
+    const uint16_t* b = br + lane;
+    const int n = w - lane;                  // elements this lane may touch: j' = 32k < n
+    int k = 0;
+    for (; k + 96 < n; k += 128) {
+        m.add(a[k], b[k]);
+        m.add(a[k + 32], b[k + 32]);
+        m.add(a[k + 64], b[k + 64]);
+        m.add(a[k + 96], b[k + 96]);
+    }
+    for (; k < n; k += 32) m.add(a[k], b[k]);
+}
+
+template <int W, int H>
 __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restrict__ raw,
                                                         const PairIdx* __restrict__ pairs,
                                                         const unsigned long long* __restrict__ keys,
                                                         unsigned long long* __restrict__ mom,
-                                                        int H, int W, int pair0) {
-    __shared__ unsigned long long red[5][CCF_T / 32];
+                                                        int pair0) {
+    extern __shared__ uint4 ccf_smem[];
+    __shared__ unsigned long long red[10][CCF_T / 32];
     const int p = pair0 + blockIdx.y;
     const PairIdx pr = pairs[p];
     const uint32_t lo = 0xFFFFFFFFu - (uint32_t)(keys[p] & 0xFFFFFFFFull);
     const int x = (int)(lo % (uint32_t)W), y = (int)(lo / (uint32_t)W);
-    const uint16_t* A = raw + (size_t)pr.a * H * W;
-    const uint16_t* B = raw + (size_t)pr.b * H * W;
-    const int r0 = blockIdx.x * CCF_ROWS;
-    const int r1 = min(r0 + CCF_ROWS, 2 * H);
-    unsigned long long sa = 0, sb = 0, saa = 0, sbb = 0, sab = 0;
-    int cur = -1;
-    for (int r = r0; r <= r1; ++r) {
-        int k = 4, i = 0;
-        if (r < r1) {
-            const int h12 = H - y;
-            if (r < h12) { k = 0; i = r; }
-            else if (r < 2 * h12) { k = 1; i = r - h12; }
-            else if (r < 2 * h12 + y) { k = 2; i = r - 2 * h12; }
-            else { k = 3; i = r - 2 * h12 - y; }
-        }
-        if (k != cur) {  // block-uniform: flush the previous candidate's partial sums
-            if (cur >= 0) {
-                unsigned long long v[5] = {sa, sb, saa, sbb, sab};
-#pragma unroll
-                for (int q = 0; q < 5; ++q) {
-                    v[q] = warp_sum_u64(v[q]);
-                    if ((threadIdx.x & 31) == 0) red[q][threadIdx.x >> 5] = v[q];
-                }
-                __syncthreads();
-                if (threadIdx.x < 5) {
-                    unsigned long long s = 0;
-                    for (int w = 0; w < CCF_T / 32; ++w) s += red[threadIdx.x][w];
-                    if (s) atomicAdd(&mom[((size_t)p * 4 + cur) * 5 + threadIdx.x], s);
-                }
-                __syncthreads();
+    const int nb0 = (H - y + CCF_ROWS - 1) / CCF_ROWS;
+    int g, i0, hg;
+    if ((int)blockIdx.x < nb0) { g = 0; i0 = blockIdx.x * CCF_ROWS; hg = H - y; }
+    else { g = 1; i0 = (blockIdx.x - nb0) * CCF_ROWS; hg = y; }
+    if (i0 >= hg) return;                      // block-uniform
+    const int dy = g ? H - y : y;
+    const int rows_total = min(CCF_ROWS, hg - i0);
+    const uint16_t* A = raw + (size_t)pr.a * H * W + (size_t)(dy + i0) * W;
+    const uint16_t* B = raw + (size_t)pr.b * H * W + (size_t)i0 * W;
+    uint16_t* sA = reinterpret_cast<uint16_t*>(ccf_smem);
+    uint16_t* sB = sA + CCF_BATCH * W;
+    const int w0 = W - x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    Moments m0, m1;
+    for (int rb = 0; rb < rows_total; rb += CCF_BATCH) {
+        const int rows = min(CCF_BATCH, rows_total - rb);
+        const int n = rows * W;                // a contiguous run of rows in both tiles
+        if (rb) __syncthreads();               // previous batch consumed
+        if constexpr ((W & 7) == 0) {
+            const uint4* A4 = reinterpret_cast<const uint4*>(A + (size_t)rb * W);
+            const uint4* B4 = reinterpret_cast<const uint4*>(B + (size_t)rb * W);
+            uint4* sA4 = reinterpret_cast<uint4*>(sA);
+            uint4* sB4 = reinterpret_cast<uint4*>(sB);
+            for (int q = threadIdx.x; q < n / 8; q += CCF_T) {
+                sA4[q] = __ldg(A4 + q);
+                sB4[q] = __ldg(B4 + q);
             }
-            cur = k;
-            sa = sb = saa = sbb = sab = 0;
+        } else {                               // rows not 16-byte aligned
+            for (int q = threadIdx.x; q < n; q += CCF_T) {
+                sA[q] = __ldg(A + (size_t)rb * W + q);
+                sB[q] = __ldg(B + (size_t)rb * W + q);
+            }
         }
-        if (k == 4) break;
-        const int dx = (k & 1) ? W - x : x;
-        const int dy = (k & 2) ? H - y : y;
-        const int w = W - dx;
-        const uint16_t* ar = A + (size_t)(dy + i) * W + dx;
-        const uint16_t* br = B + (size_t)i * W;
-        for (int j = threadIdx.x; j < w; j += CCF_T) {
-            const uint32_t a = __ldg(ar + j), b = __ldg(br + j);
-            sa += a;
-            sb += b;
-            saa += (unsigned long long)(a * a);
-            sbb += (unsigned long long)(b * b);
-            sab += (unsigned long long)(a * b);
+        __syncthreads();
+        if (warp < rows) {                     // one warp per staged row
+            const uint16_t* ar = sA + warp * W;
+            const uint16_t* br = sB + warp * W;
+            row_moments(m0, ar, br, x, w0, lane);   // candidate dx = x
+            row_moments(m1, ar, br, w0, x, lane);   // candidate dx = W - x
         }
     }
+    unsigned long long v[10] = {m0.sa, m0.sb, m0.saa, m0.sbb, m0.sab,
+                                m1.sa, m1.sb, m1.saa, m1.sbb, m1.sab};
+#pragma unroll
+    for (int q = 0; q < 10; ++q) {
+        v[q] = warp_sum_u64(v[q]);
+        if (lane == 0) red[q][warp] = v[q];
+    }
+    __syncthreads();
+    if (threadIdx.x < 10) {
+        unsigned long long s = 0;
+#pragma unroll
+        for (int w = 0; w < CCF_T / 32; ++w) s += red[threadIdx.x][w];
+        const int c = 2 * g + threadIdx.x / 5;  // candidate index 0..3 (c1..c4)
+        atomicAdd(&mom[((size_t)p * 4 + c) * 5 + threadIdx.x % 5], s);
+    }
 }
+
+inline size_t k5_smem_bytes(int W) { return (size_t)2 * CCF_BATCH * W * sizeof(uint16_t); }
+inline int k5_grid_x(int H) { return H / CCF_ROWS + 2; }
 
 // ------------------------------------------------------------------ K6 ----
 __device__ __forceinline__ double i128_to_double(__int128 v) {

@@ -4,7 +4,9 @@
 // launch schedule of K1..K6 (pciam_kernels.cuh) and the copy-in / copy-out.
 // The runtime is deliberately small: one stream, chunked launches sized so the
 // per-chunk intermediates (K1->K2 spectra, K3->K4 Q) stay in the 126 MB L2.
+#include <cuda.h>
 #include <cuda_runtime.h>
+#include <cudaTypedefs.h>
 
 #include <cmath>
 #include <cstdio>
@@ -22,50 +24,86 @@ namespace {
 
 // ------------------------------------------------------------ plan table ---
 // Compiled tile-size plans (Radix lists: the row transform is W/2 complex).
-//            W     H     row radices            column radices        rowL rowT colP colT
-using P1392 = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 16, 416>;
-using P256 = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 16, 256>;
-using P48 = Plan<48, 40, Radix<24, 24>, Radix<40, 40>, 8, 64, 16, 64>;
-using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 64, 16, 64>;
+//            W     H     row radices          column radices      rowL rowT colP colT rowPad colPad
+using P1392 = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 8, 208, 0, 1>;
+using P256 = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 8, 128, 1, 1>;
+using P48 = Plan<48, 40, Radix<24, 24>, Radix<40, 40>, 8, 32, 8, 32, 0, 0>;
+using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 32, 8, 32, 0, 0>;
 
 struct PlanOps {
     int W, H, M, WC, WP, row_l, col_p;
-    cudaError_t (*setup)();
+    int row_r0, row_r1, col_r0, col_r1;  // stage radices (r1 = 1: single stage)
+    cudaError_t (*setup)(int* grid_k1p, int* grid_k4p);  // persistent grids (0 = not used)
+    void (*k1p)(const uint16_t*, float2*, int, int, const float2*, const float2*, int, cudaStream_t);
+    void (*k4p)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
+                cudaStream_t);
+    void (*k5)(const uint16_t*, const PairIdx*, const unsigned long long*, unsigned long long*, int,
+               int, cudaStream_t);
     void (*k1)(const uint16_t*, float2*, int, int, const float2*, const float2*, cudaStream_t);
-    void (*k2)(float2*, int, int, const float2*, cudaStream_t);
-    void (*k3)(const float2*, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
+    void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, cudaStream_t);
+    void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
                cudaStream_t);
 };
 
-template <class PL>
-cudaError_t plan_setup() {
-    cudaError_t e;
-    if ((e = cudaFuncSetAttribute(k1_fwd_rows<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)PL::ROW_SMEM)) != cudaSuccess) return e;
-    if ((e = cudaFuncSetAttribute(k4_pair_rows<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)PL::ROW_SMEM)) != cudaSuccess) return e;
-    if ((e = cudaFuncSetAttribute(k2_fwd_cols<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)PL::COL_SMEM)) != cudaSuccess) return e;
-    return cudaFuncSetAttribute(k3_pair_cols<PL>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)PL::COL_SMEM);
+template <class K>
+cudaError_t max_smem(K* kernel, size_t bytes) {
+    cudaError_t e = cudaFuncSetAttribute(kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         (int)bytes);
+    if (e != cudaSuccess) return e;
+    return cudaFuncSetAttribute(kernel, cudaFuncAttributePreferredSharedMemoryCarveout,
+                                (int)cudaSharedmemCarveoutMaxShared);
 }
 
 template <class PL>
-void launch_k1(const uint16_t* raw, float2* spec, int t0, int nt, const float2* twM,
+cudaError_t plan_setup(int* grid_k1p, int* grid_k4p) {
+    cudaError_t e;
+    using RP = RowPersist<PL>;
+    int dev = 0, sms = 0, nb = 0;
+    if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+    if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+        return e;
+    *grid_k1p = 0;
+    if (RP::K1_BULK) {
+        if ((e = max_smem(k1p_fwd_rows<PL>, RP::SMEM_K1)) != cudaSuccess) return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1p_fwd_rows<PL>, PL::ROW_T,
+                                                                RP::SMEM_K1)) != cudaSuccess)
+            return e;
+        *grid_k1p = nb * sms;
+    }
+    if ((e = max_smem(k4p_pair_rows<PL>, RP::SMEM_K4)) != cudaSuccess) return e;
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k4p_pair_rows<PL>, PL::ROW_T,
+                                                            RP::SMEM_K4)) != cudaSuccess)
+        return e;
+    *grid_k4p = nb * sms;
+    if ((e = max_smem(k5_ccf_moments<PL::W, PL::H>, k5_smem_bytes(PL::W))) != cudaSuccess) return e;
+    if ((e = max_smem(k1_fwd_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(k4_pair_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(k2t_fwd_cols<PL, false>, PL::COL_SMEM)) != cudaSuccess) return e;
+    return max_smem(k3t_pair_cols<PL>, PL::COL_SMEM);
+}
+
+template <class PL>
+void launch_k1(const uint16_t* raw, float2* G, int t0, int nt, const float2* twM,
                const float2* twW, cudaStream_t s) {
-    k1_fwd_rows<PL><<<dim3(PL::H / PL::ROW_L, nt), PL::ROW_T, PL::ROW_SMEM, s>>>(raw, spec, t0,
+    k1_fwd_rows<PL><<<dim3(PL::H / PL::ROW_L, nt), PL::ROW_T, PL::ROW_SMEM, s>>>(raw, G, t0,
                                                                                  twM, twW);
 }
 template <class PL>
-void launch_k2(float2* spec, int t0, int nt, const float2* twH, cudaStream_t s) {
-    k2_fwd_cols<PL><<<dim3(PL::WP / PL::COL_P, nt), PL::COL_T, PL::COL_SMEM, s>>>(spec, t0, twH);
+void launch_k2(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt, const float2* tw2,
+               bool phase_out, cudaStream_t s) {
+    const dim3 grid(PL::WP / PL::COL_P, nt);
+    if (phase_out)
+        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2);
+    else
+        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2);
 }
 template <class PL>
-void launch_k3(const float2* spec, float2* Q, const PairIdx* pairs, int p0, int np,
-               const float2* twH, cudaStream_t s) {
-    k3_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(spec, Q, pairs,
-                                                                                   p0, twH);
+void launch_k3(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
+               const float2* tw2, cudaStream_t s) {
+    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(tmS, Q, pairs,
+                                                                                    p0, tw2);
 }
 template <class PL>
 void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const float2* twM,
@@ -75,10 +113,33 @@ void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const 
 }
 
 template <class PL>
+void launch_k1p(const uint16_t* raw, float2* G, int t0, int nt, const float2* tw2,
+                const float2* twW, int grid, cudaStream_t s) {
+    const int nblk = nt * (PL::H / PL::ROW_L);
+    k1p_fwd_rows<PL><<<grid < nblk ? grid : nblk, PL::ROW_T, RowPersist<PL>::SMEM_K1, s>>>(
+        raw, G, t0, nt, tw2, twW);
+}
+template <class PL>
+void launch_k4p(const float2* Q, unsigned long long* keys, int p0, int np, const float2* tw2,
+                const float2* twW, int grid, cudaStream_t s) {
+    const int nblk = np * (PL::H / PL::ROW_L);
+    k4p_pair_rows<PL><<<grid < nblk ? grid : nblk, PL::ROW_T, RowPersist<PL>::SMEM_K4, s>>>(
+        Q, keys, p0, np, tw2, twW);
+}
+
+template <class PL>
+void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long long* keys,
+               unsigned long long* mom, int p0, int np, cudaStream_t s) {
+    k5_ccf_moments<PL::W, PL::H><<<dim3(k5_grid_x(PL::H), np), CCF_T, k5_smem_bytes(PL::W), s>>>(
+        raw, pairs, keys, mom, p0);
+}
+
+template <class PL>
 PlanOps make_ops() {
-    return PlanOps{PL::W,      PL::H,        PL::M,        PL::WC,       PL::WP,
-                   PL::ROW_L,  PL::COL_P,    plan_setup<PL>, launch_k1<PL>, launch_k2<PL>,
-                   launch_k3<PL>, launch_k4<PL>};
+    return PlanOps{PL::W,       PL::H,         PL::M,          PL::WC,        PL::WP,
+                   PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
+                   PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
+                   launch_k1<PL>, launch_k2<PL>, launch_k3<PL>, launch_k4<PL>};
 }
 
 const PlanOps* find_plan(int W, int H) {
@@ -91,11 +152,16 @@ const PlanOps* find_plan(int W, int H) {
 
 size_t align256(size_t x) { return (x + 255) / 256 * 256; }
 
+// twiddle tables: row stage-2 [r0*(r1-1)], column stage-2 [c0*(c1-1)], R2C/C2R w_W [W]
+size_t tw_row(const PlanOps* o) { return (size_t)o->row_r0 * (o->row_r1 - 1); }
+size_t tw_col(const PlanOps* o) { return (size_t)o->col_r0 * (o->col_r1 - 1); }
+size_t tw_count(const PlanOps* o) { return tw_row(o) + tw_col(o) + o->W + 2; }
+
 struct Layout {
     int h_begin, t_begin, t_end, nlocal;
     int64_t npairs;
     int chunk_pairs, chunk_tiles;
-    size_t off_raw, off_spec, off_q, off_pairs, off_keys, off_mom, off_res, off_tw, total;
+    size_t off_raw, off_spec, off_g, off_q, off_pairs, off_keys, off_mom, off_res, off_tw, total;
 };
 
 stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L) {
@@ -115,13 +181,14 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     size_t o = 0;
     L->off_raw = o;   o += align256((size_t)L->nlocal * H * W * sizeof(uint16_t));
-    L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * sizeof(float2));
+    L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * sizeof(uint32_t));
+    L->off_g = o;     o += align256((size_t)L->chunk_tiles * H * WP * sizeof(float2));
     L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * sizeof(float2));
     L->off_pairs = o; o += align256((size_t)(np > 0 ? np : 1) * sizeof(PairIdx));
     L->off_keys = o;  o += align256((size_t)(np > 0 ? np : 1) * sizeof(unsigned long long));
     L->off_mom = o;   o += align256((size_t)(np > 0 ? np : 1) * 20 * sizeof(unsigned long long));
     L->off_res = o;   o += align256((size_t)(np > 0 ? np : 1) * sizeof(stitch_pair));
-    L->off_tw = o;    o += align256((size_t)(ops->M + ops->H + ops->W) * sizeof(float2));
+    L->off_tw = o;    o += align256((size_t)(tw_count(ops)) * sizeof(float2));
     L->total = o;
     return STITCH_OK;
 }
@@ -149,7 +216,9 @@ struct stitch_ctx {
     char* mem = nullptr;
     bool own_mem = false;
     uint16_t* raw;
-    float2 *spec, *Q, *twM, *twH, *twW;
+    uint32_t* spec;                   // resident phase spectra [nlocal][H][WP]
+    float2 *G, *Q, *twM, *twH, *twW;  // chunk intermediates, twiddles
+    CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (phase codes)
     PairIdx* pairs;
     unsigned long long *keys, *mom;
     stitch_pair* res;
@@ -158,6 +227,7 @@ struct stitch_ctx {
     std::vector<stitch_pair> res_h;
     bool loaded = false, computed = false;
     int64_t launches = 0;
+    int grid_k1p = 0, grid_k4p = 0;   // persistent-kernel grids (0: use the non-persistent kernel)
     int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     float ms[4] = {0, 0, 0, 0};
@@ -275,7 +345,8 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     };
     cudaError_t e = cudaSetDevice(cfg->device);
     if (e != cudaSuccess) return bail(STITCH_ERR_CUDA);
-    if ((e = ops->setup()) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if ((e = ops->setup(&ctx->grid_k1p, &ctx->grid_k4p)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+
     if (cfg->stream) {
         ctx->stream = (cudaStream_t)cfg->stream;
     } else {
@@ -293,27 +364,64 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     }
     char* b = ctx->mem;
     ctx->raw = (uint16_t*)(b + L.off_raw);
-    ctx->spec = (float2*)(b + L.off_spec);
+    ctx->spec = (uint32_t*)(b + L.off_spec);
+    ctx->G = (float2*)(b + L.off_g);
     ctx->Q = (float2*)(b + L.off_q);
     ctx->pairs = (PairIdx*)(b + L.off_pairs);
     ctx->keys = (unsigned long long*)(b + L.off_keys);
     ctx->mom = (unsigned long long*)(b + L.off_mom);
     ctx->res = (stitch_pair*)(b + L.off_res);
     ctx->twM = (float2*)(b + L.off_tw);
-    ctx->twH = ctx->twM + ops->M;
-    ctx->twW = ctx->twH + ops->H;
+    ctx->twH = ctx->twM + tw_row(ops);
+    ctx->twW = ctx->twH + tw_col(ops);
 
-    // Twiddle tables w_N^e = exp(-2 pi i e / N), computed in double, rounded once.
-    std::vector<float2> tw((size_t)ops->M + ops->H + ops->W);
-    auto fill = [&](float2* dst, int N) {
-        for (int k = 0; k < N; ++k) {
-            const double a = -2.0 * M_PI * (double)k / (double)N;
-            dst[k] = make_float2((float)std::cos(a), (float)std::sin(a));
+    // TMA descriptors (driver entry point through the runtime; no libcuda link needed)
+    {
+        void* fn = nullptr;
+        cudaDriverEntryPointQueryResult q;
+        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) !=
+                cudaSuccess || !fn)
+            return bail(STITCH_ERR_CUDA);
+        auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
+        const cuuint32_t boxh = (cuuint32_t)(ops->H / ((ops->H + 255) / 256));
+        const cuuint32_t estr[2] = {1, 1};
+        {
+            const cuuint64_t dims[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
+            const cuuint64_t strides[1] = {(cuuint64_t)ops->WP * 8};
+            const cuuint32_t box[2] = {(cuuint32_t)2 * ops->col_p, boxh};
+            if (encode(&ctx->tmG, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, dims, strides, box,
+                       estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                       CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                return bail(STITCH_ERR_CUDA);
         }
+        {
+            const cuuint64_t dims[2] = {(cuuint64_t)ops->WP, (cuuint64_t)L.nlocal * ops->H};
+            const cuuint64_t strides[1] = {(cuuint64_t)ops->WP * 4};
+            const cuuint32_t box[2] = {(cuuint32_t)ops->col_p, boxh};
+            if (encode(&ctx->tmS, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->spec, dims, strides, box,
+                       estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                       CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+                return bail(STITCH_ERR_CUDA);
+        }
+    }
+
+    // Twiddles w_N^e = exp(-2 pi i e / N), computed in double, rounded once.
+    //   stage-2 tables: tw2[b*(r1-1) + j-1] = w_N^{j b}, b < r0, 1 <= j < r1 (fft_engine.cuh)
+    std::vector<float2> tw(tw_count(ops));
+    auto w = [](long e, long N) {
+        const double a = -2.0 * M_PI * (double)(e % N) / (double)N;
+        return make_float2((float)std::cos(a), (float)std::sin(a));
     };
-    fill(tw.data(), ops->M);
-    fill(tw.data() + ops->M, ops->H);
-    fill(tw.data() + ops->M + ops->H, ops->W);
+    auto fill2 = [&](float2* dst, int r0, int r1) {
+        const int N = r0 * r1;
+        for (int bb = 0; bb < r0; ++bb)
+            for (int j = 1; j < r1; ++j) dst[(size_t)bb * (r1 - 1) + j - 1] = w((long)j * bb, N);
+    };
+    fill2(tw.data(), ops->row_r0, ops->row_r1);
+    fill2(tw.data() + tw_row(ops), ops->col_r0, ops->col_r1);
+    for (int k = 0; k < ops->W; ++k) tw[tw_row(ops) + tw_col(ops) + k] = w(k, ops->W);
 
     // Pair list, Fig. 4 order: for each owned tile, west then north, as (neighbour, tile).
     std::vector<PairIdx> pl;
@@ -399,9 +507,12 @@ static stitch_status forward_impl(stitch_ctx* ctx) {
     const int nl = ctx->L.nlocal, ct = ctx->L.chunk_tiles;
     for (int t0 = 0; t0 < nl; t0 += ct) {
         const int nt = nl - t0 < ct ? nl - t0 : ct;
-        o->k1(ctx->raw, ctx->spec, t0, nt, ctx->twM, ctx->twW, ctx->stream);
+        if (ctx->grid_k1p > 0)
+            o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, ctx->stream);
+        else
+            o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->stream);
         CK(mark(ctx, 0), "event");
-        o->k2(ctx->spec, t0, nt, ctx->twH, ctx->stream);
+        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->stream);
         CK(mark(ctx, 1), "event");
         ctx->launches += 2;
     }
@@ -442,9 +553,12 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
         const int cp = ctx->L.chunk_pairs;
         for (int64_t p0 = 0; p0 < np; p0 += cp) {
             const int npc = (int)(np - p0 < cp ? np - p0 : cp);
-            o->k3(ctx->spec, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
+            o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
             CK(mark(ctx, 2), "event");
-            o->k4(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, s);
+            if (ctx->grid_k4p > 0)
+                o->k4p(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, ctx->grid_k4p, s);
+            else
+                o->k4(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, s);
             CK(mark(ctx, 3), "event");
             ctx->launches += 2;
         }
@@ -452,11 +566,9 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     }
     if (ctx->timing) CK(cudaEventRecord(ctx->ev[2], s), "event");
     if (np > 0) {
-        const int rows = (2 * ctx->H + CCF_ROWS - 1) / CCF_ROWS;
         for (int64_t p0 = 0; p0 < np; p0 += 65535) {
             const int npc = (int)(np - p0 < 65535 ? np - p0 : 65535);
-            k5_ccf_moments<<<dim3(rows, npc), CCF_T, 0, s>>>(ctx->raw, ctx->pairs, ctx->keys,
-                                                            ctx->mom, ctx->H, ctx->W, (int)p0);
+            o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, s);
             CK(mark(ctx, 4), "event");
             ctx->launches += 1;
         }
@@ -530,9 +642,18 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
     if (!host_out) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output");
     if (tile < ctx->L.h_begin || tile >= ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
+    // The resident store keeps phase codes; recompute the complex spectrum of this tile
+    // with the same K1 + K2 kernels into the chunk buffer G (slot 0) and copy it out.
     const int lt = tile - ctx->L.h_begin;
-    const float2* src = ctx->spec + (size_t)lt * ctx->H * ctx->ops->WP;
-    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), src,
+    const PlanOps* o = ctx->ops;
+    if (ctx->grid_k1p > 0)
+        o->k1p(ctx->raw, ctx->G, lt, 1, ctx->twM, ctx->twW, ctx->grid_k1p, ctx->stream);
+    else
+        o->k1(ctx->raw, ctx->G, lt, 1, ctx->twM, ctx->twW, ctx->stream);
+    o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->twH, false, ctx->stream);
+    CK(cudaGetLastError(), "spectrum launch");
+    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->G,
                          ctx->ops->WP * sizeof(float2), ctx->ops->WC * sizeof(float2), ctx->H,
                          cudaMemcpyDeviceToHost, ctx->stream),
        "copy spectrum");
