@@ -9,7 +9,7 @@ for every west/north pair) over the synthetic grid of BASELINE.json configs[2]
 (42x59 tiles of 1392x1040 uint16).  `value` is pairs/s
 with the tiles resident in HBM; `e2e` is the same through the C ABI from pinned
 host buffers (H2D of the tiles + D2H of the results inside the timed region).
-Inputs (7.2 GB of tiles, 14.5 GB of spectra) are far larger than the 126 MB L2.
+Inputs (7.2 GB of tiles, 7.3 GB of resident phase spectra) are far larger than the 126 MB L2.
 
 N > 1 (torchrun): row-band partition of the grid, one rank per GPU; each rank
 owns tiles [k*nt/N, (k+1)*nt/N) and keeps the preceding tile row resident (halo,
@@ -258,14 +258,18 @@ def main():
     pg.set_timing(0)
     step_kernel_ms = sum(v["ms"] for v in kt_sum.values())
     dom = max(kt_sum, key=lambda k: kt_sum[k]["ms"])
-    S = H * (W // 2 + 1) * 8          # algorithmic fp32 half spectrum bytes
+    S = H * (W // 2 + 1) * 8          # fp32 complex half spectrum (kx in [0, W/2]) bytes
     T = H * W * 2                     # raw tile bytes
-    alg_bytes_per_unit = {            # SURVEY 8(d) per-unit byte model
-        "k1_fwd_rows": T + S, "k2_fwd_cols": 2 * S, "k3_pair_cols": 3 * S,
-        "k4_pair_rows": S, "k5_ccf_moments": 2 * T, "k6_finalize": 8 + 160 + 64}
-    units_per_launch = {
-        "k1_fwd_rows": pg.cfg.chunk_tiles or 8, "k2_fwd_cols": pg.cfg.chunk_tiles or 8,
-        "k3_pair_cols": pg.cfg.chunk_pairs or 8, "k4_pair_rows": pg.cfg.chunk_pairs or 8}
+    # Algorithmic bytes per unit (tile or pair) of each kernel in this design (DESIGN.md
+    # "Roofline"): what it must read + write at least once; the resident spectrum is a
+    # 4-byte phase code per bin (S/2), intermediates G and Q are complex (S).
+    alg_bytes_per_unit = {
+        "k1_fwd_rows": T + S,          # raw in, row-transformed G out
+        "k2_fwd_cols": S + S // 2,     # G in, phase spectrum out
+        "k3_pair_cols": S // 2 * 2 + S,  # two phase spectra in, Q out
+        "k4_pair_rows": S,             # Q in (the surface is never stored)
+        "k5_ccf_moments": 2 * T,       # the four candidate overlaps of A and B (HW pixels each)
+        "k6_finalize": 8 + 160 + 64}
     kd = kt_sum[dom]
     nsteps_k = max(1, min(args.steps, 5))
     units_total = {"k1_fwd_rows": (e - halo), "k2_fwd_cols": (e - halo),
@@ -280,9 +284,15 @@ def main():
                 "peak_source": pk_kind, "avg_launch_ms": avg_launch_ms,
                 "alg_bytes_per_launch": bytes_per_launch,
                 "share_of_step": kd["ms"] / step_kernel_ms,
-                "kernels_ms_per_step": {k: v["ms"] / nsteps_k for k, v in kt_sum.items()}}
-    grid_alg_bytes = ((e - halo) * (T + 3 * S) + pairs_local * (4 * S + 2 * T))
-    roofline["step_alg_GBps"] = grid_alg_bytes / (dev_ms / 1e3) / 1e9
+                "kernels_ms_per_step": {k: v["ms"] / nsteps_k for k, v in kt_sum.items()},
+                "kernels_frac": {k: (alg_bytes_per_unit[k] * units_total[k] / (v["ms"] / nsteps_k
+                                                                              / 1e3) / 1e9)
+                                 / pk["hbm_gbs"] for k, v in kt_sum.items() if v["ms"] > 0}}
+    design_bytes = sum(alg_bytes_per_unit[k] * units_total[k] for k in alg_bytes_per_unit)
+    survey_2pass = (e - halo) * (T + 3 * S) + pairs_local * (4 * S + 2 * T)
+    roofline["step_alg_GBps"] = design_bytes / (dev_ms / 1e3) / 1e9
+    roofline["step_frac"] = roofline["step_alg_GBps"] / pk["hbm_gbs"]
+    roofline["survey_2pass_GBps"] = survey_2pass / (dev_ms / 1e3) / 1e9
     traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(traffic_path):
         with open(traffic_path) as f:
@@ -319,7 +329,7 @@ def main():
             "config": {"workload": f"{cfg['name']} (BASELINE.json configs[{args.config - 1}])",
                        "grid": f"{n}x{m}", "tile": f"{W}x{H} uint16", "pairs": int(total_pairs),
                        "tiles": n * m, "grid_wall_ms": ms, "parallelism": f"row-bands x{world}",
-                       "l2": "inputs larger than L2 (7.2 GB tiles, 14.5 GB spectra vs 126 MB)",
+                       "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)",
                        "overlap": cfg["overlap"], "seed": synthgrid.SEED},
             "roofline": roofline,
             "cpu_baseline": cpu,

@@ -71,16 +71,20 @@ struct Plan {
     static constexpr size_t COL_LAND = COL_LAND_C > COL_LAND_P ? COL_LAND_C : COL_LAND_P;
     static constexpr size_t COL_XCH =
         CI::STAGES == 1 ? 0 : sizeof(float2) * COL_P * CI::R1 * (CI::R0 + COL_PAD);
-    static constexpr size_t COL_SMEM = COL_LAND > COL_XCH ? COL_LAND : COL_XCH;
+    static constexpr size_t COL_BUF = ((COL_LAND > COL_XCH ? COL_LAND : COL_XCH) + 15) / 16 * 16;
+    static constexpr int COL_TW2N = CI::R0 * (CI::R1 - 1);      // stage-2 twiddles in smem
+    static constexpr size_t COL_SMEM = COL_BUF + sizeof(float2) * (COL_TW2N > 0 ? COL_TW2N : 1);
     static constexpr int BOXH = H / ((H + 255) / 256);   // TMA box rows (<= 256)
     static_assert(H % BOXH == 0, "H must split into equal TMA boxes of <= 256 rows");
     static_assert((BOXH * COL_P * 4) % 128 == 0 || H == BOXH, "TMA boxes must land 128-B aligned");
     // CTAs per SM the column kernels are register-budgeted for (shared memory allows this many)
     static constexpr int COL_MINB_RAW = (int)((220 * 1024) / (COL_SMEM + 1024));
     static constexpr int COL_MINB = COL_MINB_RAW > 3 ? 3 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
-    // register cap so COL_MINB CTAs of COL_T threads fit the 64K-register file (8-register units)
+    // register cap so COL_MINB CTAs of COL_T threads fit: the 64K-register file is split
+    // over the 4 SM sub-partitions (16K each) and warps are dealt to them round robin
     static constexpr int COL_WARPS = (COL_T + 31) / 32;
-    static constexpr int COL_MAXREG_RAW = (65536 / (COL_MINB * COL_WARPS * 32)) / 8 * 8;
+    static constexpr int COL_WPS = (COL_MINB * COL_WARPS + 3) / 4;   // warps per sub-partition
+    static constexpr int COL_MAXREG_RAW = (16384 / (COL_WPS * 32)) / 8 * 8;
     static constexpr int COL_MAXREG = COL_MAXREG_RAW > 255 ? 255 : COL_MAXREG_RAW;
     // stage-2 twiddle tables (w_N^{-j b}, see fft_engine.cuh)
     static constexpr int ROW_TW2 = RI::R0 * (RI::R1 - 1);
@@ -223,17 +227,18 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C);
         tma_panel<PL>(csmem, &tmG, 2 * c0, tl * PL::H, 8, &bar);
     }
+    float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
+    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
     mbar_wait(&bar, 0);
     LandSrc<PL> src{reinterpret_cast<const float2*>(csmem)};
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
+    using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, true>;
     if constexpr (PHASE_OUT) {
         PhaseDst<PL> dst{spec + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
-        FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap>::template run<true>(src, xc, dst,
-                                                                                       tw2);
+        Run::template run<true>(src, xc, dst, tws);
     } else {
         PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
-        FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap>::template run<true>(src, xc, dst,
-                                                                                       tw2);
+        Run::template run<true>(src, xc, dst, tws);
     }
 }
 
@@ -273,12 +278,14 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         tma_panel<PL>(la, &tmS, c0, pr.a * PL::H, 4, &bar);
         tma_panel<PL>(lb, &tmS, c0, pr.b * PL::H, 4, &bar);
     }
+    float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
+    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
     mbar_wait(&bar, 0);
     NcpsPhaseSrc<PL> src{la, lb};
     PanelIO<PL> dst{Q + (size_t)blockIdx.y * PL::H * PL::WP + c0};
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
-    FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap>::template run<true>(src, xc, dst,
-                                                                                   tw2);
+    FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, true>::template run<true>(src, xc,
+                                                                                         dst, tws);
 }
 
 // ------------------------------------------------------------------ K4 ----
@@ -303,8 +310,11 @@ struct ArgmaxDst {  // step 5: running max of |x| with its row-major index, neve
     uint32_t best_i;   // its row-major index y*W + x (smallest index among equal values)
     int row_base;      // y0 of the CTA's first line
     int W;
+    // Every thread stores its values in increasing index order (one butterfly per line and
+    // thread in the row plans: n = b + j*R0 with j increasing), so a strict '>' keeps the
+    // smallest index among equal values; across threads the packed key decides (C6).
     __device__ __forceinline__ void take(float a, uint32_t idx) {
-        if (a > best_v || (a == best_v && idx < best_i)) {
+        if (a > best_v) {
             best_v = a;
             best_i = idx;
         }
@@ -588,8 +598,11 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
                                                         const unsigned long long* __restrict__ keys,
                                                         unsigned long long* __restrict__ mom,
                                                         int pair0) {
-    extern __shared__ uint4 ccf_smem[];
+    constexpr bool BULK = (W * 2) % 16 == 0;   // rows 16-byte aligned: TMA bulk copies
+    constexpr int BUFS = BULK ? 2 : 1;
+    extern __shared__ __align__(16) unsigned char ccf_smem[];
     __shared__ unsigned long long red[10][CCF_T / 32];
+    __shared__ uint64_t bar[2];
     const int p = pair0 + blockIdx.y;
     const PairIdx pr = pairs[p];
     const uint32_t lo = 0xFFFFFFFFu - (uint32_t)(keys[p] & 0xFFFFFFFFull);
@@ -601,38 +614,56 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
     if (i0 >= hg) return;                      // block-uniform
     const int dy = g ? H - y : y;
     const int rows_total = min(CCF_ROWS, hg - i0);
+    const int nbatch = (rows_total + CCF_BATCH - 1) / CCF_BATCH;
     const uint16_t* A = raw + (size_t)pr.a * H * W + (size_t)(dy + i0) * W;
     const uint16_t* B = raw + (size_t)pr.b * H * W + (size_t)i0 * W;
-    uint16_t* sA = reinterpret_cast<uint16_t*>(ccf_smem);
-    uint16_t* sB = sA + CCF_BATCH * W;
-    const int w0 = W - x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    Moments m0, m1;
-    for (int rb = 0; rb < rows_total; rb += CCF_BATCH) {
-        const int rows = min(CCF_BATCH, rows_total - rb);
-        const int n = rows * W;                // a contiguous run of rows in both tiles
-        if (rb) __syncthreads();               // previous batch consumed
-        if constexpr ((W & 7) == 0) {
-            const uint4* A4 = reinterpret_cast<const uint4*>(A + (size_t)rb * W);
-            const uint4* B4 = reinterpret_cast<const uint4*>(B + (size_t)rb * W);
-            uint4* sA4 = reinterpret_cast<uint4*>(sA);
-            uint4* sB4 = reinterpret_cast<uint4*>(sB);
-            for (int q = threadIdx.x; q < n / 8; q += CCF_T) {
-                sA4[q] = __ldg(A4 + q);
-                sB4[q] = __ldg(B4 + q);
-            }
-        } else {                               // rows not 16-byte aligned
-            for (int q = threadIdx.x; q < n; q += CCF_T) {
-                sA[q] = __ldg(A + (size_t)rb * W + q);
-                sB[q] = __ldg(B + (size_t)rb * W + q);
-            }
+    auto bufA = [&](int buf) { return reinterpret_cast<uint16_t*>(ccf_smem) + buf * 2 * CCF_BATCH * W; };
+    auto bufB = [&](int buf) { return bufA(buf) + CCF_BATCH * W; };
+    auto issue = [&](int bi) {  // TMA bulk copy of batch bi (A rows and B rows) into buffer bi&1
+        const int rows = min(CCF_BATCH, rows_total - bi * CCF_BATCH);
+        const uint32_t bytes = (uint32_t)(rows * W * 2);
+        uint64_t* br = &bar[bi & 1];
+        mbar_arrive_expect_tx(br, 2 * bytes);
+        bulk_g2s(bufA(bi & 1), A + (size_t)bi * CCF_BATCH * W, bytes, br);
+        bulk_g2s(bufB(bi & 1), B + (size_t)bi * CCF_BATCH * W, bytes, br);
+    };
+    if constexpr (BULK) {
+        if (threadIdx.x == 0) {
+            mbar_init(&bar[0], 1);
+            mbar_init(&bar[1], 1);
+            fence_mbar_init();
+            issue(0);
         }
         __syncthreads();
+    }
+    const int w0 = W - x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    Moments m0, m1;
+    for (int bi = 0; bi < nbatch; ++bi) {
+        const int rows = min(CCF_BATCH, rows_total - bi * CCF_BATCH);
+        const int buf = bi % BUFS;
+        if constexpr (BULK) {
+            // prefetch the next batch into the other buffer (freed by the barrier that
+            // ended batch bi-1), then wait for this one
+            if (threadIdx.x == 0 && bi + 1 < nbatch) {
+                fence_proxy_async();
+                issue(bi + 1);
+            }
+            mbar_wait(&bar[buf], (bi >> 1) & 1);
+        } else {                               // rows not 16-byte aligned: plain staging
+            const int n = rows * W;
+            for (int q = threadIdx.x; q < n; q += CCF_T) {
+                bufA(0)[q] = __ldg(A + (size_t)bi * CCF_BATCH * W + q);
+                bufB(0)[q] = __ldg(B + (size_t)bi * CCF_BATCH * W + q);
+            }
+            __syncthreads();
+        }
         if (warp < rows) {                     // one warp per staged row
-            const uint16_t* ar = sA + warp * W;
-            const uint16_t* br = sB + warp * W;
+            const uint16_t* ar = bufA(buf) + warp * W;
+            const uint16_t* br = bufB(buf) + warp * W;
             row_moments(m0, ar, br, x, w0, lane);   // candidate dx = x
             row_moments(m1, ar, br, w0, x, lane);   // candidate dx = W - x
         }
+        __syncthreads();                       // buffer free for batch bi+2
     }
     unsigned long long v[10] = {m0.sa, m0.sb, m0.saa, m0.sbb, m0.sab,
                                 m1.sa, m1.sb, m1.saa, m1.sbb, m1.sab};
@@ -651,7 +682,9 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
     }
 }
 
-inline size_t k5_smem_bytes(int W) { return (size_t)2 * CCF_BATCH * W * sizeof(uint16_t); }
+inline size_t k5_smem_bytes(int W) {
+    return (size_t)((W * 2) % 16 == 0 ? 2 : 1) * 2 * CCF_BATCH * W * sizeof(uint16_t);
+}
 inline int k5_grid_x(int H) { return H / CCF_ROWS + 2; }
 
 // ------------------------------------------------------------------ K6 ----

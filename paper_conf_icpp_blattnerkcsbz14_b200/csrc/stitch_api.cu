@@ -8,6 +8,7 @@
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
 
+#include <algorithm>
 #include <cmath>
 #include <cstdio>
 #include <cstring>
@@ -175,8 +176,8 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     int64_t np = 0;
     for (int t = L->t_begin; t < L->t_end; ++t) np += (t % m >= 1) + (t / m >= 1);
     L->npairs = np;
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 8;
-    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 8;
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 24;
+    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 16;
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     size_t o = 0;
@@ -423,10 +424,24 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     fill2(tw.data() + tw_row(ops), ops->col_r0, ops->col_r1);
     for (int k = 0; k < ops->W; ++k) tw[tw_row(ops) + tw_col(ops) + k] = w(k, ops->W);
 
-    // Pair list, Fig. 4 order: for each owned tile, west then north, as (neighbour, tile).
+    // Pair list: every owned tile's west and north pair, as (neighbour, tile) (Fig. 4).
+    // Processing order (results do not depend on it): tiles in bands of PAIR_BAND tile
+    // rows, column-major inside a band, so a tile's spectrum and raw pixels are reused by
+    // its <= 4 pairs while still in L2 (the paper's traversal-order idea).
+    constexpr int PAIR_BAND = 8;
+    std::vector<int> order;
+    order.reserve((size_t)(L.t_end - L.t_begin));
+    for (int t = L.t_begin; t < L.t_end; ++t) order.push_back(t);
+    const int mm = ctx->m;
+    std::stable_sort(order.begin(), order.end(), [mm](int a, int b) {
+        const int ra = a / mm, rb = b / mm, ba = ra / PAIR_BAND, bb = rb / PAIR_BAND;
+        if (ba != bb) return ba < bb;
+        if (a % mm != b % mm) return a % mm < b % mm;
+        return ra < rb;
+    });
     std::vector<PairIdx> pl;
     pl.reserve((size_t)L.npairs);
-    for (int t = L.t_begin; t < L.t_end; ++t) {
+    for (const int t : order) {
         const int r = t / ctx->m, c = t % ctx->m;
         if (c >= 1) {
             pl.push_back(PairIdx{t - 1 - L.h_begin, t - L.h_begin});
