@@ -12,8 +12,10 @@ host buffers (H2D of the tiles + D2H of the results inside the timed region).
 Inputs (7.2 GB of tiles, 7.3 GB of resident phase spectra) are far larger than the 126 MB L2.
 
 N > 1 (torchrun): row-band partition of the grid, one rank per GPU; each rank
-owns tiles [k*nt/N, (k+1)*nt/N) and keeps the preceding tile row resident (halo,
-recomputed locally); the per-step time is the max over ranks (all_reduce MAX).
+owns tiles [k*nt/N, (k+1)*nt/N) and keeps the preceding tile row resident (halo):
+the halo's spectra are received from the previous rank (NCCL send/recv over NVLink,
+paper future work P:L1512-1517), its raw pixels are loaded with the band; the per-step
+time is the max over ranks (all_reduce MAX).
 
 --impl reference: the reference arm is the oracle (oracle/, plain C, fp64),
 timed as it stands on the host cores on a bounded sample of the same workload.
@@ -34,6 +36,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 import synthgrid  # noqa: E402
+from paper_conf_icpp_blattnerkcsbz14_b200.parallel import band as parallel_band  # noqa: E402
 
 PAPER_PAIRS_PER_S = 4855 / 49.7   # Pipelined-GPU, 1x Tesla C2070, Table II: context
 REASON_BITS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
@@ -171,6 +174,8 @@ def main():
     ap.add_argument("--chunk-tiles", type=int, default=0)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-exchange", action="store_true",
+                    help="N > 1: recompute the halo row's spectra instead of receiving them")
     args = ap.parse_args()
     cfg = dict(synthgrid.CONFIGS[args.config])
     if args.impl == "reference":
@@ -179,7 +184,7 @@ def main():
     import torch
     import torch.distributed as dist
 
-    from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid
+    from paper_conf_icpp_blattnerkcsbz14_b200.parallel import BandPciam
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -193,14 +198,17 @@ def main():
     n, m, H, W = cfg["n"], cfg["m"], cfg["H"], cfg["W"]
     b, e, halo = band(rank, world, n, m)
     r0, r1 = halo // m, (e - 1) // m + 1            # tile rows this rank holds
+    assert (r0, r1) == (parallel_band(rank, world, n, m).row_begin,
+                        parallel_band(rank, world, n, m).row_end)
     # host tiles of the rows this rank needs, in pinned memory (the e2e source buffer)
     host = torch.empty((r1 - r0, m, H, W), dtype=torch.uint16, pin_memory=True)
     synthgrid.make_grid(n, m, H, W, overlap=cfg["overlap"], delta=cfg["delta"],
                         out=host.numpy().view(np.uint16), rows=(r0, r1))
     first = r0 * m
 
-    pg = PciamGrid(n, m, H, W, device=local, tile_begin=b, tile_end=e,
+    bp = BandPciam(n, m, H, W, rank, world, device=local, exchange=not args.no_exchange,
                    chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles)
+    pg = bp.grid
     stream = torch.cuda.current_stream()
     pg.load_tiles(host, first)
     pg.synchronize()
@@ -227,7 +235,7 @@ def main():
 
     # ---- warm-up, then K timed steps with tiles resident in HBM ----------------------------
     for _ in range(args.warmup):
-        pg.compute_translations_async()
+        bp.step_async()
     barrier()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     launches = 0
@@ -235,7 +243,7 @@ def main():
         barrier()
         ev0.record(stream)
         for _ in range(args.steps):
-            pg.compute_translations_async()
+            bp.step_async()
             launches += pg.last_counts()["launches"]
         ev1.record(stream)
         barrier()
@@ -249,7 +257,7 @@ def main():
     pg.set_timing(2)
     kt_sum = {}
     for _ in range(max(1, min(args.steps, 5))):
-        pg.compute_translations_async()
+        bp.step_async()
         pg.synchronize()
         for k, v in pg.kernel_timings().items():
             s = kt_sum.setdefault(k, {"ms": 0.0, "launches": 0})
@@ -272,7 +280,8 @@ def main():
         "k6_finalize": 8 + 160 + 64}
     kd = kt_sum[dom]
     nsteps_k = max(1, min(args.steps, 5))
-    units_total = {"k1_fwd_rows": (e - halo), "k2_fwd_cols": (e - halo),
+    fwd_tiles = (e - b) if bp.use_exchange else (e - halo)   # halo received or recomputed
+    units_total = {"k1_fwd_rows": fwd_tiles, "k2_fwd_cols": fwd_tiles,
                    "k3_pair_cols": pairs_local, "k4_pair_rows": pairs_local,
                    "k5_ccf_moments": pairs_local, "k6_finalize": pairs_local}
     bytes_per_launch = alg_bytes_per_unit[dom] * units_total[dom] / (kd["launches"] / nsteps_k)
@@ -289,7 +298,7 @@ def main():
                                                                               / 1e3) / 1e9)
                                  / pk["hbm_gbs"] for k, v in kt_sum.items() if v["ms"] > 0}}
     design_bytes = sum(alg_bytes_per_unit[k] * units_total[k] for k in alg_bytes_per_unit)
-    survey_2pass = (e - halo) * (T + 3 * S) + pairs_local * (4 * S + 2 * T)
+    survey_2pass = fwd_tiles * (T + 3 * S) + pairs_local * (4 * S + 2 * T)
     roofline["step_alg_GBps"] = design_bytes / (dev_ms / 1e3) / 1e9
     roofline["step_frac"] = roofline["step_alg_GBps"] / pk["hbm_gbs"]
     roofline["survey_2pass_GBps"] = survey_2pass / (dev_ms / 1e3) / 1e9
@@ -305,8 +314,9 @@ def main():
     barrier()
     t0 = time.perf_counter()
     for _ in range(e2e_steps):
-        pg.load_tiles(host, first)
-        west, north = pg.compute_translations()     # D2H of the results, synchronous
+        pg.load_tiles(host, first)                  # H2D of this rank's tile rows
+        bp.step_async()
+        west, north = pg.get_translations()         # D2H of the results, synchronous
     torch.cuda.synchronize()
     e2e_s = max_over_ranks((time.perf_counter() - t0) / e2e_steps)
     h2d = (e - halo) * T
@@ -329,6 +339,8 @@ def main():
             "config": {"workload": f"{cfg['name']} (BASELINE.json configs[{args.config - 1}])",
                        "grid": f"{n}x{m}", "tile": f"{W}x{H} uint16", "pairs": int(total_pairs),
                        "tiles": n * m, "grid_wall_ms": ms, "parallelism": f"row-bands x{world}",
+                       "halo": ("nccl-exchange" if bp.use_exchange else
+                                ("recompute" if world > 1 else "none")),
                        "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)",
                        "overlap": cfg["overlap"], "seed": synthgrid.SEED},
             "roofline": roofline,
@@ -339,7 +351,7 @@ def main():
             "clocks": clocks,
         }
         print(json.dumps(line), flush=True)
-    pg.close()
+    bp.close()
     if world > 1:
         dist.destroy_process_group()
 

@@ -145,6 +145,22 @@ stitch_status stitch_get_translations(stitch_ctx* ctx, stitch_pair* west, stitch
 stitch_status stitch_forward_async(stitch_ctx* ctx);
 
 /*
+ * Split form of a step, for multi-GPU row bands:
+ *   stitch_forward_range_async — step 2 for the resident tiles [first_tile, first_tile+count)
+ *     (global row-major indices; INVALID_ARG if not resident);
+ *   stitch_spectra_range — device address and size of the resident spectra of a tile range
+ *     (phase codes, u32 [count][H][pitch]; contiguous), so the caller can send the last tile
+ *     row of its band to the next rank and receive its halo row (e.g. NCCL send/recv through
+ *     torch.distributed on the workspace tensor) instead of recomputing it;
+ *   stitch_pairs_async — steps 3-7 for every pair of the range, spectra already resident.
+ * compute_translations_async == forward_range_async(all resident) + pairs_async.
+ */
+stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, int32_t count);
+stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t count,
+                                   void** dev_ptr, size_t* bytes);
+stitch_status stitch_pairs_async(stitch_ctx* ctx);
+
+/*
  * Test hook: copy tile t's resident half spectrum F(ky, kx), ky in [0,H),
  * kx in [0, W/2] (complex64, [H][W/2+1][2] floats) to the host.  Valid after
  * stitch_forward_async / compute.  Synchronous.

@@ -57,7 +57,8 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_compute_translations", "stitch_get_translations", "stitch_forward_async",
            "stitch_debug_spectrum", "stitch_synchronize", "stitch_last_counts",
            "stitch_last_timings", "stitch_set_timing", "stitch_last_error", "stitch_destroy",
-           "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings"]
+           "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings",
+           "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async"]
 
 _lib = None
 
@@ -94,6 +95,9 @@ def load_library():
         "stitch_load_tiles": (ctypes.c_int, [vp, vp, i32, i32, i32]),
         "stitch_resident_range": (ctypes.c_int, [vp, P(i32), P(i32), P(i32)]),
         "stitch_kernel_timings": (ctypes.c_int, [vp, P(ctypes.c_float), P(i64)]),
+        "stitch_forward_range_async": (ctypes.c_int, [vp, i32, i32]),
+        "stitch_spectra_range": (ctypes.c_int, [vp, i32, i32, P(vp), P(ctypes.c_size_t)]),
+        "stitch_pairs_async": (ctypes.c_int, [vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -209,6 +213,30 @@ class PciamGrid:
 
     def forward_async(self) -> None:
         self._check(self.lib.stitch_forward_async(self._ctx), "forward")
+
+    def forward_range_async(self, first_tile: int, count: int) -> None:
+        """Step 2 for resident tiles [first_tile, first_tile + count) (global indices)."""
+        self._check(self.lib.stitch_forward_range_async(self._ctx, first_tile, count), "forward")
+
+    def pairs_async(self) -> None:
+        """Steps 3-7 for every pair of the context (spectra already resident)."""
+        self._check(self.lib.stitch_pairs_async(self._ctx), "pairs")
+
+    def spectra_range(self, first_tile: int, count: int) -> tuple[int, int]:
+        """(device address, bytes) of the resident spectra of tiles [first_tile, +count)."""
+        ptr, nbytes = ctypes.c_void_p(), ctypes.c_size_t()
+        self._check(self.lib.stitch_spectra_range(self._ctx, first_tile, count, ctypes.byref(ptr),
+                                                  ctypes.byref(nbytes)), "spectra range")
+        return ptr.value or 0, nbytes.value
+
+    def spectra_view(self, first_tile: int, count: int):
+        """The resident spectra of a tile range as a uint8 view of the torch workspace
+        (for torch.distributed send/recv); requires the torch workspace."""
+        if self._ws is None:
+            raise RuntimeError("spectra_view needs the torch workspace (use_torch=True)")
+        ptr, nbytes = self.spectra_range(first_tile, count)
+        off = ptr - self._ws.data_ptr()
+        return self._ws[off: off + nbytes]
 
     def get_translations(self, west: np.ndarray | None = None, north: np.ndarray | None = None):
         if west is None:

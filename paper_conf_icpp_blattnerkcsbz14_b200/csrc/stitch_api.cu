@@ -517,11 +517,12 @@ stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid,
     return load_common(ctx, dev_grid, n_bytes, cudaMemcpyDeviceToDevice);
 }
 
-static stitch_status forward_impl(stitch_ctx* ctx) {
+// Forward transforms (K1 + K2) of the resident tiles with local indices [lt0, lt0 + count).
+static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
     const PlanOps* o = ctx->ops;
-    const int nl = ctx->L.nlocal, ct = ctx->L.chunk_tiles;
-    for (int t0 = 0; t0 < nl; t0 += ct) {
-        const int nt = nl - t0 < ct ? nl - t0 : ct;
+    const int ct = ctx->L.chunk_tiles;
+    for (int t0 = lt0; t0 < lt0 + count; t0 += ct) {
+        const int nt = lt0 + count - t0 < ct ? lt0 + count - t0 : ct;
         if (ctx->grid_k1p > 0)
             o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, ctx->stream);
         else
@@ -535,32 +536,11 @@ static stitch_status forward_impl(stitch_ctx* ctx) {
     return STITCH_OK;
 }
 
-stitch_status stitch_forward_async(stitch_ctx* ctx) {
-    if (!ctx) return STITCH_ERR_INVALID_ARG;
-    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
-    ctx->launches = 0;
-    return forward_impl(ctx);
-}
-
-stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
-    if (!ctx) return STITCH_ERR_INVALID_ARG;
-    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "compute before load");
+// Steps 3-7 (K3..K6) for every pair of the range; spectra must be resident.
+static stitch_status pairs_impl(stitch_ctx* ctx) {
     const PlanOps* o = ctx->ops;
     cudaStream_t s = ctx->stream;
     const int64_t np = ctx->L.npairs;
-    ctx->launches = 0;
-    ctx->kkind.clear();
-    if (ctx->timing >= 2) {
-        if (ctx->kev.empty()) {
-            ctx->kev.resize(1024, nullptr);
-            for (auto& e : ctx->kev) CK(cudaEventCreate(&e), "event create");
-        }
-        CK(cudaEventRecord(ctx->kev[0], s), "event");
-    }
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[0], s), "event");
-    stitch_status st = forward_impl(ctx);
-    if (st != STITCH_OK) return st;
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], s), "event");
     if (np > 0) {
         CK(cudaMemsetAsync(ctx->keys, 0, (size_t)np * sizeof(unsigned long long), s), "memset");
         CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), s), "memset");
@@ -595,6 +575,72 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     }
     if (ctx->timing) CK(cudaEventRecord(ctx->ev[3], s), "event");
     ctx->computed = true;
+    return STITCH_OK;
+}
+
+// Start of a step: reset launch counters and (timing modes) record the start events.
+static stitch_status step_begin(stitch_ctx* ctx) {
+    cudaStream_t s = ctx->stream;
+    ctx->launches = 0;
+    ctx->kkind.clear();
+    ctx->computed = false;
+    if (ctx->timing >= 2) {
+        if (ctx->kev.empty()) {
+            ctx->kev.resize(1024, nullptr);
+            for (auto& e : ctx->kev) CK(cudaEventCreate(&e), "event create");
+        }
+        CK(cudaEventRecord(ctx->kev[0], s), "event");
+    }
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[0], s), "event");
+    return STITCH_OK;
+}
+
+stitch_status stitch_forward_async(stitch_ctx* ctx) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
+    stitch_status st = step_begin(ctx);
+    if (st != STITCH_OK) return st;
+    st = forward_impl(ctx, 0, ctx->L.nlocal);
+    if (st == STITCH_OK && ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
+    return st;
+}
+
+stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, int32_t count) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
+    if (count < 0 || first_tile < ctx->L.h_begin || first_tile + (int64_t)count > ctx->L.t_end)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
+    stitch_status st = step_begin(ctx);
+    if (st != STITCH_OK) return st;
+    st = forward_impl(ctx, first_tile - ctx->L.h_begin, count);
+    if (st == STITCH_OK && ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
+    return st;
+}
+
+stitch_status stitch_pairs_async(stitch_ctx* ctx) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "pairs before load");
+    return pairs_impl(ctx);
+}
+
+stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "compute before load");
+    stitch_status st = step_begin(ctx);
+    if (st != STITCH_OK) return st;
+    if ((st = forward_impl(ctx, 0, ctx->L.nlocal)) != STITCH_OK) return st;
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
+    return pairs_impl(ctx);
+}
+
+stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t count,
+                                   void** dev_ptr, size_t* bytes) {
+    if (!ctx || !dev_ptr || !bytes) return STITCH_ERR_INVALID_ARG;
+    if (count < 0 || first_tile < ctx->L.h_begin || first_tile + (int64_t)count > ctx->L.t_end)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
+    const size_t per = (size_t)ctx->H * ctx->ops->WP * sizeof(uint32_t);
+    *dev_ptr = reinterpret_cast<char*>(ctx->spec) + (size_t)(first_tile - ctx->L.h_begin) * per;
+    *bytes = (size_t)count * per;
     return STITCH_OK;
 }
 

@@ -1,0 +1,139 @@
+"""Row-band multi-GPU partition of a PCIAM grid.
+
+The paper runs one independent pipeline per GPU over a spatial decomposition of the
+grid and leaves the partition boundary unspecified (reading C16);
+P2P copies between cards are its future work (L1512-1517).  Here:
+
+* rank k of R owns the tiles [k*nt/R, (k+1)*nt/R) (row-major, nt = n*m) and the pairs
+  whose tile B it owns (Fig. 4 west/north pairs);
+* its pairs also need the m tiles before its first tile (one tile row, the "halo"):
+  their raw pixels are loaded with the band, their spectra are RECEIVED from rank k-1,
+  which owns them and has just transformed them -- one point-to-point send/recv per band
+  boundary (NCCL over NVLink through torch.distributed; gloo in the CPU tests);
+* results are merged with one all_gather of each rank's owned entries.
+
+If a band is shorter than a tile row the halo spans two ranks; the driver then falls
+back to recomputing the halo's forward transforms locally (no data-path collective).
+torch is plumbing here: process groups, the workspace tensor, the stream.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+
+import numpy as np
+
+
+@dataclass(frozen=True)
+class Band:
+    rank: int
+    world: int
+    t_begin: int      # first owned tile
+    t_end: int        # one past the last owned tile
+    halo_begin: int   # first resident tile = max(0, t_begin - m)
+    row_begin: int    # tile rows [row_begin, row_end) hold every resident tile
+    row_end: int
+
+    @property
+    def owned(self) -> int:
+        return self.t_end - self.t_begin
+
+
+def band(rank: int, world: int, n: int, m: int) -> Band:
+    nt = n * m
+    if not (0 <= rank < world) or world < 1:
+        raise ValueError("bad rank/world")
+    b, e = rank * nt // world, (rank + 1) * nt // world
+    halo = max(0, b - m)
+    return Band(rank, world, b, e, halo, halo // m, (e - 1) // m + 1 if e > 0 else 0)
+
+
+@dataclass(frozen=True)
+class HaloPlan:
+    """Tile ranges this rank sends to rank+1 / receives from rank-1 (None: nothing)."""
+    send: tuple[int, int] | None   # (first tile, count)
+    recv: tuple[int, int] | None
+
+
+def exchange_feasible(world: int, n: int, m: int) -> bool:
+    """Every halo lies inside the previous rank's band (all bands >= one tile row)."""
+    return world > 1 and all(band(k, world, n, m).owned >= m for k in range(world - 1))
+
+
+def halo_plan(rank: int, world: int, n: int, m: int) -> HaloPlan:
+    bd = band(rank, world, n, m)
+    recv = (bd.halo_begin, bd.t_begin - bd.halo_begin) if rank > 0 and bd.t_begin > 0 else None
+    send = None
+    if rank < world - 1:
+        nxt = band(rank + 1, world, n, m)
+        cnt = nxt.t_begin - nxt.halo_begin
+        if cnt > 0:
+            send = (nxt.halo_begin, cnt)
+    if recv and recv[1] == 0:
+        recv = None
+    return HaloPlan(send, recv)
+
+
+def exchange_halo(send_buf, recv_buf, rank: int, world: int, group=None) -> None:
+    """Send `send_buf` to rank+1 and receive `recv_buf` from rank-1 (batched P2P)."""
+    import torch.distributed as dist
+    ops = []
+    if send_buf is not None and rank + 1 < world:
+        ops.append(dist.P2POp(dist.isend, send_buf, rank + 1, group))
+    if recv_buf is not None and rank > 0:
+        ops.append(dist.P2POp(dist.irecv, recv_buf, rank - 1, group))
+    if ops:
+        for w in dist.batch_isend_irecv(ops):
+            w.wait()
+
+
+def gather_translations(west: np.ndarray, north: np.ndarray, bd: Band, group=None):
+    """Merge every rank's owned entries into full [n, m] arrays on all ranks."""
+    import torch.distributed as dist
+    mine = (bd.t_begin, bd.t_end, west.reshape(-1)[bd.t_begin:bd.t_end].copy(),
+            north.reshape(-1)[bd.t_begin:bd.t_end].copy())
+    parts = [None] * bd.world
+    dist.all_gather_object(parts, mine, group=group)
+    w, n = west.copy().reshape(-1), north.copy().reshape(-1)
+    for b, e, pw, pn in parts:
+        w[b:e] = pw
+        n[b:e] = pn
+    return w.reshape(west.shape), n.reshape(north.shape)
+
+
+class BandPciam:
+    """One rank's share of a grid: a PciamGrid over its band plus the halo exchange."""
+
+    def __init__(self, n: int, m: int, H: int, W: int, rank: int, world: int, device: int = 0,
+                 exchange: bool = True, group=None, **kw):
+        from . import PciamGrid
+        self.n, self.m, self.H, self.W = n, m, H, W
+        self.rank, self.world, self.group = rank, world, group
+        self.bd = band(rank, world, n, m)
+        self.plan = halo_plan(rank, world, n, m)
+        self.use_exchange = exchange and exchange_feasible(world, n, m)
+        self.grid = PciamGrid(n, m, H, W, device=device, tile_begin=self.bd.t_begin,
+                              tile_end=self.bd.t_end, **kw)
+        self.npairs = self.grid.npairs
+
+    def load_rows(self, rows, first_tile: int | None = None) -> None:
+        """Tiles of rows [row_begin, row_end) ([rows, m, H, W], host or device)."""
+        self.grid.load_tiles(rows, self.bd.row_begin * self.m if first_tile is None
+                             else first_tile)
+
+    def step_async(self) -> None:
+        """Steps 2-7 for the band: forward the owned tiles, exchange the halo row's
+        spectra with the neighbouring ranks, then every owned pair."""
+        if not self.use_exchange:
+            self.grid.compute_translations_async()     # halo recomputed locally
+            return
+        self.grid.forward_range_async(self.bd.t_begin, self.bd.owned)
+        send = self.grid.spectra_view(*self.plan.send) if self.plan.send else None
+        recv = self.grid.spectra_view(*self.plan.recv) if self.plan.recv else None
+        exchange_halo(send, recv, self.rank, self.world, self.group)
+        self.grid.pairs_async()
+
+    def translations(self):
+        return self.grid.get_translations()
+
+    def close(self) -> None:
+        self.grid.close()

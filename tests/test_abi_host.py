@@ -76,7 +76,7 @@ def test_row_band_pairs_partition_the_grid(lib, R):
 
 
 def test_workspace_size_matches_layout(lib):
-    cfg = pkg.make_config(42, 59, 1040, 1392, chunk_pairs=8)
+    cfg = pkg.make_config(42, 59, 1040, 1392, chunk_pairs=8, chunk_tiles=8)
     ws = pkg.workspace_size(cfg)
     H, W, WP = 1040, 1392, 704
     raw = 2478 * H * W * 2

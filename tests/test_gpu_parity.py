@@ -164,6 +164,36 @@ def test_world_size_invariance_row_bands():
         assert w.tobytes() == wf.tobytes() and nn.tobytes() == nf.tobytes(), R
 
 
+def test_halo_exchange_emulated_bit_identical():
+    """Row bands whose halo spectra are RECEIVED from the previous band's context (copied
+    device to device exactly as rank k-1 sends them over NCCL) instead of recomputed give
+    bit-identical results to the whole-grid context."""
+    from paper_conf_icpp_blattnerkcsbz14_b200.parallel import band, exchange_feasible, halo_plan
+    n, m = 6, 7
+    g = synthgrid.make_grid(n, m, 192, 256, seed=33)
+    wf, nf, _ = run_gpu(g.tiles)
+    for R in (2, 3, 4):
+        assert exchange_feasible(R, n, m)
+        bands = [band(k, R, n, m) for k in range(R)]
+        ctxs = [PciamGrid(n, m, 192, 256, tile_begin=b.t_begin, tile_end=b.t_end) for b in bands]
+        try:
+            for b, c in zip(bands, ctxs):
+                c.load_grid(g.tiles)
+                c.forward_range_async(b.t_begin, b.owned)        # owned tiles only
+            for k in range(1, R):
+                recv = ctxs[k].spectra_view(*halo_plan(k, R, n, m).recv)
+                send = ctxs[k - 1].spectra_view(*halo_plan(k - 1, R, n, m).send)
+                recv.copy_(send)
+            w = np.zeros_like(wf); nn = np.zeros_like(nf)
+            for c in ctxs:
+                c.pairs_async()
+                c.get_translations(w.reshape(-1), nn.reshape(-1))
+        finally:
+            for c in ctxs:
+                c.close()
+        assert w.tobytes() == wf.tobytes() and nn.tobytes() == nf.tobytes(), R
+
+
 def test_chunking_invariance():
     g = synthgrid.make_grid(4, 5, 192, 256, seed=32)
     ref = run_gpu(g.tiles)
