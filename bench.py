@@ -209,7 +209,7 @@ def main():
     bp = BandPciam(n, m, H, W, rank, world, device=local, exchange=not args.no_exchange,
                    chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles)
     pg = bp.grid
-    stream = torch.cuda.current_stream()
+    stream = pg.stream          # the stream the library enqueues on (events must be recorded here)
     pg.load_tiles(host, first)
     pg.synchronize()
     pairs_local = pg.npairs

@@ -141,15 +141,19 @@ class PciamGrid:
         self.device = device
         self._ctx = ctypes.c_void_p(None)
         self._ws = None
-        stream = None
         cfg = make_config(n, m, H, W, device, tile_begin, tile_end, chunk_pairs, chunk_tiles)
+        self.stream = None
         if use_torch:
             import torch
             dev = torch.device("cuda", device)
-            stream = torch.cuda.current_stream(dev).cuda_stream
+            cur = torch.cuda.current_stream(dev)
+            # The context enqueues on a real torch stream: the caller's current one, or --
+            # if that is the legacy default stream -- a dedicated one.  Record timing events
+            # and order other torch work against `self.stream`.
+            self.stream = cur if cur.cuda_stream != 0 else torch.cuda.Stream(dev)
             nbytes = workspace_size(cfg)
             self._ws = torch.empty(nbytes, dtype=torch.uint8, device=dev)
-            cfg.stream = stream
+            cfg.stream = self.stream.cuda_stream
             cfg.workspace = self._ws.data_ptr()
             cfg.workspace_bytes = nbytes
         self.cfg = cfg

@@ -94,9 +94,11 @@ template <int N, int R0, int SIGN, int L, int T, class Map, bool TW_SMEM>
 struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM> {
     static_assert(N == R0, "single-stage plan");
     static constexpr int R1 = 1;
-    template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid>
+    template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid,
+              class AfterLoads = NoMid>
     static __device__ __forceinline__ void run(const Src& src, const Xc&, Dst& dst,
-                                               const float2* __restrict__, const Mid& mid = Mid()) {
+                                               const float2* __restrict__, const Mid& mid = Mid(),
+                                               const AfterLoads& after_loads = AfterLoads()) {
         // one butterfly per line (the source is consumed inside the loop; `mid` runs after it)
         constexpr int TOTAL = L;
         constexpr int ITER = (TOTAL + T - 1) / T;
@@ -114,6 +116,7 @@ struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM> {
             }
         }
         __syncthreads();
+        after_loads();
         mid();
     }
 };
@@ -126,8 +129,9 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
     // Stage 1: radix R0 over R1 butterflies per line, source -> exchange.  IN_PLACE: the
     // source is the exchange buffer itself (a landing buffer reused as the exchange), so
     // every thread loads all of its butterflies before a barrier, then computes and stores.
-    template <bool IN_PLACE, class Src, class Xc>
-    static __device__ __forceinline__ void stage1(const Src& src, const Xc& xc) {
+    template <bool IN_PLACE, class Src, class Xc, class AfterLoads = NoMid>
+    static __device__ __forceinline__ void stage1(const Src& src, const Xc& xc,
+                                                  const AfterLoads& after_loads = AfterLoads()) {
         constexpr int TOTAL = L * R1;
         constexpr int ITER = (TOTAL + T - 1) / T;
         if constexpr (IN_PLACE) {
@@ -143,6 +147,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
                 }
             }
             __syncthreads();
+            after_loads();   // the source buffer is free from here on
 #pragma unroll
             for (int it = 0; it < ITER; ++it) {
                 const int g = threadIdx.x + it * T;
@@ -174,11 +179,13 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
 
     // `mid` runs (in every thread) after the barrier that ends stage 1, i.e. once the
     // source has been fully consumed: persistent kernels prefetch their next input there.
-    template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid>
+    template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid,
+              class AfterLoads = NoMid>
     static __device__ __forceinline__ void run(const Src& src, const Xc& xc, Dst& dst,
                                                const float2* __restrict__ tw2,
-                                               const Mid& mid = Mid()) {
-        stage1<IN_PLACE>(src, xc);
+                                               const Mid& mid = Mid(),
+                                               const AfterLoads& after_loads = AfterLoads()) {
+        stage1<IN_PLACE>(src, xc, after_loads);
         __syncthreads();
         mid();
         {   // stage 2: radix R1 over R0 butterflies per line, exchange -> destination

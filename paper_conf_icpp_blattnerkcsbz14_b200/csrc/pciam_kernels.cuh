@@ -73,13 +73,17 @@ struct Plan {
         CI::STAGES == 1 ? 0 : sizeof(float2) * COL_P * CI::R1 * (CI::R0 + COL_PAD);
     static constexpr size_t COL_BUF = ((COL_LAND > COL_XCH ? COL_LAND : COL_XCH) + 15) / 16 * 16;
     static constexpr int COL_TW2N = CI::R0 * (CI::R1 - 1);      // stage-2 twiddles in smem
+    // persistent column kernels: separate landing and exchange buffers (prefetch overlap)
+    static constexpr size_t COLP_XOFF = (COL_LAND + 127) / 128 * 128;
+    static constexpr size_t COLP_TOFF = COLP_XOFF + (COL_XCH + 15) / 16 * 16;
+    static constexpr size_t COLP_SMEM = COLP_TOFF + sizeof(float2) * (COL_TW2N > 0 ? COL_TW2N : 1);
     static constexpr size_t COL_SMEM = COL_BUF + sizeof(float2) * (COL_TW2N > 0 ? COL_TW2N : 1);
     static constexpr int BOXH = H / ((H + 255) / 256);   // TMA box rows (<= 256)
     static_assert(H % BOXH == 0, "H must split into equal TMA boxes of <= 256 rows");
     static_assert((BOXH * COL_P * 4) % 128 == 0 || H == BOXH, "TMA boxes must land 128-B aligned");
     // CTAs per SM the column kernels are register-budgeted for (shared memory allows this many)
     static constexpr int COL_MINB_RAW = (int)((220 * 1024) / (COL_SMEM + 1024));
-    static constexpr int COL_MINB = COL_MINB_RAW > 3 ? 3 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
+    static constexpr int COL_MINB = COL_MINB_RAW > 4 ? 4 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
     // register cap so COL_MINB CTAs of COL_T threads fit: the 64K-register file is split
     // over the 4 SM sub-partitions (16K each) and warps are dealt to them round robin
     static constexpr int COL_WARPS = (COL_T + 31) / 32;
@@ -286,6 +290,104 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
     FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, true>::template run<true>(src, xc,
                                                                                          dst, tws);
+}
+
+// ------------------------------------------ persistent column kernels ----
+// K2p / K3p: one CTA per SM walks (tile|pair, panel) items in static round robin.  Each
+// item's panel lands by TMA in its own buffer; stage 1 reads it into registers, and right
+// after that barrier the TMA for the next item is issued, so the fetch overlaps stage 1's
+// butterflies, the exchange and stage 2 of the current item.
+template <class PL, bool PHASE_OUT>
+__global__ void __launch_bounds__(PL::COL_T, 1)
+    k2p_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
+                 uint32_t* __restrict__ spec, int tile0, int ntiles,
+                 const float2* __restrict__ tw2) {
+    extern __shared__ __align__(128) unsigned char csmem[];
+    __shared__ uint64_t bar;
+    constexpr int NP = PL::WP / PL::COL_P;
+    const int nitems = ntiles * NP;
+    typename PL::ColX xc{reinterpret_cast<float2*>(csmem + PL::COLP_XOFF)};
+    float2* tws = reinterpret_cast<float2*>(csmem + PL::COLP_TOFF);
+    auto issue = [&](int item) {
+        const int tl = item / NP, panel = item - tl * NP;
+        mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C);
+        tma_panel<PL>(csmem, &tmG, 2 * panel * PL::COL_P, tl * PL::H, 8, &bar);
+    };
+    if (threadIdx.x == 0) {
+        prefetch_tensormap(&tmG);
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    __syncthreads();
+    if (threadIdx.x == 0 && (int)blockIdx.x < nitems) issue(blockIdx.x);
+    using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, true>;
+    int k = 0;
+    for (int item = blockIdx.x; item < nitems; item += gridDim.x, ++k) {
+        mbar_wait(&bar, k & 1);
+        const int tl = item / NP, c0 = (item - tl * NP) * PL::COL_P;
+        const int nxt = item + gridDim.x;
+        auto after_loads = [&]() {
+            if (threadIdx.x == 0 && nxt < nitems) {
+                fence_proxy_async();
+                issue(nxt);
+            }
+        };
+        LandSrc<PL> src{reinterpret_cast<const float2*>(csmem)};
+        if constexpr (PHASE_OUT) {
+            PhaseDst<PL> dst{spec + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
+            Run::template run<true>(src, xc, dst, tws, NoMid(), after_loads);
+        } else {
+            PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
+            Run::template run<true>(src, xc, dst, tws, NoMid(), after_loads);
+        }
+    }
+}
+
+template <class PL>
+__global__ void __launch_bounds__(PL::COL_T, 1)
+    k3p_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
+                  const PairIdx* __restrict__ pairs, int pair0, int npairs,
+                  const float2* __restrict__ tw2) {
+    extern __shared__ __align__(128) unsigned char csmem[];
+    __shared__ uint64_t bar;
+    constexpr int NP = PL::WP / PL::COL_P;
+    const int nitems = npairs * NP;
+    uint32_t* la = reinterpret_cast<uint32_t*>(csmem);
+    uint32_t* lb = reinterpret_cast<uint32_t*>(csmem + PL::COL_PHASE_B);
+    typename PL::ColX xc{reinterpret_cast<float2*>(csmem + PL::COLP_XOFF)};
+    float2* tws = reinterpret_cast<float2*>(csmem + PL::COLP_TOFF);
+    auto issue = [&](int item) {
+        const int pl = item / NP, panel = item - pl * NP;
+        const PairIdx pr = pairs[pair0 + pl];
+        mbar_arrive_expect_tx(&bar, (uint32_t)(2 * PL::H * PL::COL_P * 4));
+        tma_panel<PL>(la, &tmS, panel * PL::COL_P, pr.a * PL::H, 4, &bar);
+        tma_panel<PL>(lb, &tmS, panel * PL::COL_P, pr.b * PL::H, 4, &bar);
+    };
+    if (threadIdx.x == 0) {
+        prefetch_tensormap(&tmS);
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    __syncthreads();
+    if (threadIdx.x == 0 && (int)blockIdx.x < nitems) issue(blockIdx.x);
+    using Run = FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, true>;
+    int k = 0;
+    for (int item = blockIdx.x; item < nitems; item += gridDim.x, ++k) {
+        mbar_wait(&bar, k & 1);
+        const int pl = item / NP, c0 = (item - pl * NP) * PL::COL_P;
+        const int nxt = item + gridDim.x;
+        auto after_loads = [&]() {
+            if (threadIdx.x == 0 && nxt < nitems) {
+                fence_proxy_async();
+                issue(nxt);
+            }
+        };
+        NcpsPhaseSrc<PL> src{la, lb};
+        PanelIO<PL> dst{Q + (size_t)pl * PL::H * PL::WP + c0};
+        Run::template run<true>(src, xc, dst, tws, NoMid(), after_loads);
+    }
 }
 
 // ------------------------------------------------------------------ K4 ----

@@ -10,8 +10,10 @@
 
 #include <algorithm>
 #include <cmath>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <map>
 #include <new>
 #include <string>
 #include <vector>
@@ -40,6 +42,10 @@ struct PlanOps {
                 cudaStream_t);
     void (*k5)(const uint16_t*, const PairIdx*, const unsigned long long*, unsigned long long*, int,
                int, cudaStream_t);
+    void (*k2p)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, int,
+                cudaStream_t);
+    void (*k3p)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
+                cudaStream_t);
     void (*k1)(const uint16_t*, float2*, int, int, const float2*, const float2*, cudaStream_t);
     void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, cudaStream_t);
     void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
@@ -78,6 +84,9 @@ cudaError_t plan_setup(int* grid_k1p, int* grid_k4p) {
         return e;
     *grid_k4p = nb * sms;
     if ((e = max_smem(k5_ccf_moments<PL::W, PL::H>, k5_smem_bytes(PL::W))) != cudaSuccess) return e;
+    if ((e = max_smem(k2p_fwd_cols<PL, true>, PL::COLP_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(k2p_fwd_cols<PL, false>, PL::COLP_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(k3p_pair_cols<PL>, PL::COLP_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k1_fwd_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k4_pair_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM)) != cudaSuccess) return e;
@@ -129,6 +138,24 @@ void launch_k4p(const float2* Q, unsigned long long* keys, int p0, int np, const
 }
 
 template <class PL>
+void launch_k2p(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt,
+                const float2* tw2, bool phase_out, int grid, cudaStream_t s) {
+    const int items = nt * (PL::WP / PL::COL_P);
+    const int gx = grid < items ? grid : items;
+    if (phase_out)
+        k2p_fwd_cols<PL, true><<<gx, PL::COL_T, PL::COLP_SMEM, s>>>(tmG, G, spec, t0, nt, tw2);
+    else
+        k2p_fwd_cols<PL, false><<<gx, PL::COL_T, PL::COLP_SMEM, s>>>(tmG, G, spec, t0, nt, tw2);
+}
+template <class PL>
+void launch_k3p(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
+                const float2* tw2, int grid, cudaStream_t s) {
+    const int items = np * (PL::WP / PL::COL_P);
+    const int gx = grid < items ? grid : items;
+    k3p_pair_cols<PL><<<gx, PL::COL_T, PL::COLP_SMEM, s>>>(tmS, Q, pairs, p0, np, tw2);
+}
+
+template <class PL>
 void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long long* keys,
                unsigned long long* mom, int p0, int np, cudaStream_t s) {
     k5_ccf_moments<PL::W, PL::H><<<dim3(k5_grid_x(PL::H), np), CCF_T, k5_smem_bytes(PL::W), s>>>(
@@ -140,7 +167,8 @@ PlanOps make_ops() {
     return PlanOps{PL::W,       PL::H,         PL::M,          PL::WC,        PL::WP,
                    PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
                    PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
-                   launch_k1<PL>, launch_k2<PL>, launch_k3<PL>, launch_k4<PL>};
+                   launch_k2p<PL>, launch_k3p<PL>, launch_k1<PL>, launch_k2<PL>, launch_k3<PL>,
+                   launch_k4<PL>};
 }
 
 const PlanOps* find_plan(int W, int H) {
@@ -176,7 +204,7 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     int64_t np = 0;
     for (int t = L->t_begin; t < L->t_end; ++t) np += (t % m >= 1) + (t / m >= 1);
     L->npairs = np;
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 24;
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 32;
     L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 16;
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
@@ -229,6 +257,16 @@ struct stitch_ctx {
     bool loaded = false, computed = false;
     int64_t launches = 0;
     int grid_k1p = 0, grid_k4p = 0;   // persistent-kernel grids (0: use the non-persistent kernel)
+    int grid_colp = 0;                // persistent column kernels (K2p/K3p): one CTA per SM
+    // CUDA graphs of the launch sequences (captured on first use on an internal stream,
+    // replayed on the caller's stream): one graph launch per step instead of ~700 launches
+    bool use_graph = true;
+    cudaStream_t cap_stream = nullptr;
+    struct GraphRec {
+        cudaGraphExec_t exec;
+        int64_t launches;
+    };
+    std::map<uint64_t, GraphRec> graphs;
     int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     float ms[4] = {0, 0, 0, 0};
@@ -314,6 +352,8 @@ void stitch_destroy(stitch_ctx* ctx) {
         if (e) cudaEventDestroy(e);
     for (auto& e : ctx->kev)
         if (e) cudaEventDestroy(e);
+    for (auto& g : ctx->graphs) cudaGraphExecDestroy(g.second.exec);
+    if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
     if (ctx->own_mem && ctx->mem) cudaFree(ctx->mem);
     if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
     delete ctx;
@@ -347,6 +387,20 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     cudaError_t e = cudaSetDevice(cfg->device);
     if (e != cudaSuccess) return bail(STITCH_ERR_CUDA);
     if ((e = ops->setup(&ctx->grid_k1p, &ctx->grid_k4p)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    {
+        // column-kernel variant: one CTA per panel (default: several CTAs per SM overlap each
+        // other's TMA waits) or persistent with TMA prefetch (STITCH_COL_PERSIST=1; one CTA
+        // per SM, measured slower on B200: fewer resident warps)
+        const char* env = std::getenv("STITCH_COL_PERSIST");
+        int sms = 0;
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
+        ctx->grid_colp = (env && env[0] == '1') ? sms : 0;
+        const char* genv = std::getenv("STITCH_GRAPH");   // STITCH_GRAPH=0: direct launches
+        ctx->use_graph = !(genv && genv[0] == '0');
+        if (ctx->use_graph &&
+            cudaStreamCreateWithFlags(&ctx->cap_stream, cudaStreamNonBlocking) != cudaSuccess)
+            return bail(STITCH_ERR_CUDA);
+    }
 
     if (cfg->stream) {
         ctx->stream = (cudaStream_t)cfg->stream;
@@ -528,7 +582,10 @@ static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
         else
             o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->stream);
         CK(mark(ctx, 0), "event");
-        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->stream);
+        if (ctx->grid_colp > 0)
+            o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, ctx->stream);
+        else
+            o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->stream);
         CK(mark(ctx, 1), "event");
         ctx->launches += 2;
     }
@@ -548,7 +605,10 @@ static stitch_status pairs_impl(stitch_ctx* ctx) {
         const int cp = ctx->L.chunk_pairs;
         for (int64_t p0 = 0; p0 < np; p0 += cp) {
             const int npc = (int)(np - p0 < cp ? np - p0 : cp);
-            o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
+            if (ctx->grid_colp > 0)
+                o->k3p(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, ctx->grid_colp, s);
+            else
+                o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
             CK(mark(ctx, 2), "event");
             if (ctx->grid_k4p > 0)
                 o->k4p(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, ctx->grid_k4p, s);
@@ -595,14 +655,50 @@ static stitch_status step_begin(stitch_ctx* ctx) {
     return STITCH_OK;
 }
 
+// Enqueue `body` (which launches on ctx->stream) directly, or -- graph mode, no event
+// timing -- as a CUDA graph captured once per key on the internal capture stream and
+// replayed on the caller's stream.  Every launch parameter (pointers, tensor maps, chunk
+// schedule) is fixed per context, so a replay is exactly the captured sequence.
+extern "C++" {
+template <class F>
+static stitch_status run_graphed(stitch_ctx* ctx, uint64_t key, F body) {
+    if (ctx->timing || !ctx->use_graph) return body();
+    auto it = ctx->graphs.find(key);
+    if (it == ctx->graphs.end()) {
+        cudaStream_t user = ctx->stream;
+        const int64_t l0 = ctx->launches;
+        ctx->stream = ctx->cap_stream;
+        cudaError_t e = cudaStreamBeginCapture(ctx->cap_stream, cudaStreamCaptureModeThreadLocal);
+        if (e != cudaSuccess) {
+            ctx->stream = user;
+            return cuda_fail(ctx, e, "begin capture");
+        }
+        stitch_status st = body();
+        cudaGraph_t g = nullptr;
+        e = cudaStreamEndCapture(ctx->cap_stream, &g);
+        ctx->stream = user;
+        if (st != STITCH_OK) {
+            if (g) cudaGraphDestroy(g);
+            return st;
+        }
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "end capture");
+        cudaGraphExec_t ex = nullptr;
+        e = cudaGraphInstantiate(&ex, g, 0);
+        cudaGraphDestroy(g);
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "graph instantiate");
+        it = ctx->graphs.emplace(key, stitch_ctx::GraphRec{ex, ctx->launches - l0}).first;
+        ctx->launches = l0;
+    }
+    CK(cudaGraphLaunch(it->second.exec, ctx->stream), "graph launch");
+    ctx->launches += it->second.launches;
+    return STITCH_OK;
+}
+}  // extern "C++" 
+
 stitch_status stitch_forward_async(stitch_ctx* ctx) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
-    stitch_status st = step_begin(ctx);
-    if (st != STITCH_OK) return st;
-    st = forward_impl(ctx, 0, ctx->L.nlocal);
-    if (st == STITCH_OK && ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
-    return st;
+    return stitch_forward_range_async(ctx, ctx->L.h_begin, ctx->L.nlocal);
 }
 
 stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, int32_t count) {
@@ -612,7 +708,8 @@ stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, in
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
-    st = forward_impl(ctx, first_tile - ctx->L.h_begin, count);
+    const uint64_t key = (2ull << 60) | ((uint64_t)(uint32_t)first_tile << 30) | (uint32_t)count;
+    st = run_graphed(ctx, key, [&]() { return forward_impl(ctx, first_tile - ctx->L.h_begin, count); });
     if (st == STITCH_OK && ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
     return st;
 }
@@ -620,7 +717,9 @@ stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, in
 stitch_status stitch_pairs_async(stitch_ctx* ctx) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "pairs before load");
-    return pairs_impl(ctx);
+    stitch_status st = run_graphed(ctx, 3ull << 60, [&]() { return pairs_impl(ctx); });
+    if (st == STITCH_OK) ctx->computed = true;
+    return st;
 }
 
 stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
@@ -628,9 +727,14 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "compute before load");
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
-    if ((st = forward_impl(ctx, 0, ctx->L.nlocal)) != STITCH_OK) return st;
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
-    return pairs_impl(ctx);
+    st = run_graphed(ctx, 1ull << 60, [&]() {
+        stitch_status s2 = forward_impl(ctx, 0, ctx->L.nlocal);
+        if (s2 != STITCH_OK) return s2;
+        if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
+        return pairs_impl(ctx);
+    });
+    if (st == STITCH_OK) ctx->computed = true;
+    return st;
 }
 
 stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t count,

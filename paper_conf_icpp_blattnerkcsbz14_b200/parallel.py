@@ -126,10 +126,12 @@ class BandPciam:
         if not self.use_exchange:
             self.grid.compute_translations_async()     # halo recomputed locally
             return
+        import torch
         self.grid.forward_range_async(self.bd.t_begin, self.bd.owned)
         send = self.grid.spectra_view(*self.plan.send) if self.plan.send else None
         recv = self.grid.spectra_view(*self.plan.recv) if self.plan.recv else None
-        exchange_halo(send, recv, self.rank, self.world, self.group)
+        with torch.cuda.stream(self.grid.stream):   # NCCL ordered after the forward, before pairs
+            exchange_halo(send, recv, self.rank, self.world, self.group)
         self.grid.pairs_async()
 
     def translations(self):

@@ -180,10 +180,13 @@ def test_halo_exchange_emulated_bit_identical():
             for b, c in zip(bands, ctxs):
                 c.load_grid(g.tiles)
                 c.forward_range_async(b.t_begin, b.owned)        # owned tiles only
+            for c in ctxs:
+                c.synchronize()
             for k in range(1, R):
                 recv = ctxs[k].spectra_view(*halo_plan(k, R, n, m).recv)
                 send = ctxs[k - 1].spectra_view(*halo_plan(k - 1, R, n, m).send)
                 recv.copy_(send)
+            torch.cuda.synchronize()
             w = np.zeros_like(wf); nn = np.zeros_like(nf)
             for c in ctxs:
                 c.pairs_async()
