@@ -57,7 +57,12 @@ struct RowXchg {
     }
     // element n of the transform in natural order: the slot stage 2 read it from
     // (u = n mod R0, v = n / R0), so stage 2 may write its outputs back in place
-    __device__ __forceinline__ float2& nat(int line, int n) const { return at(line, n % R0, n / R0); }
+    __device__ __forceinline__ float2& nat(int line, int n) const {
+        if constexpr (PAD == 0)
+            return s[line * LSTRIDE + n];       // v * R0 + u == n
+        else
+            return at(line, n % R0, n / R0);
+    }
     __device__ __forceinline__ void store(int line, int n, float2 v) const { nat(line, n) = v; }
 };
 // Exchange buffer for a panel of P columns: element (u, v) of column c at

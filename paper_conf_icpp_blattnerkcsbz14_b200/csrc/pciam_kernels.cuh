@@ -113,6 +113,28 @@ struct U16RowSrc {  // z[n] = x[2n] + i x[2n+1], straight from the uint16 row
     }
 };
 
+// Real-to-complex post-processing of one line (Z = the length-M complex FFT of the packed
+// row, in the exchange buffer, natural order; Z[M] == Z[0]).  For q in [0, M/2]:
+//   E = (Z[q] + conj Z[M-q]) / 2,  O = (Z[q] - conj Z[M-q]) / (2i)
+//   X[q] = E + w_W^q O,   X[M-q] = conj(E - w_W^q O)
+// (E and O of M-q are conj(E), conj(O), and w_W^{M-q} = -conj(w_W^q)), so one iteration
+// writes the mirror pair; bins [M+1, WP) of the padded row are zeroed.
+template <class PL, class Xc, class TwLoad>
+__device__ __forceinline__ void r2c_post_line(const Xc& xc, int line, float2* __restrict__ out,
+                                              const TwLoad& twq) {
+    constexpr int M = PL::M;
+    for (int q = threadIdx.x; q <= M / 2; q += PL::ROW_T) {
+        const float2 zq = xc.nat(line, q);
+        const float2 zm = xc.nat(line, q == 0 ? 0 : M - q);
+        const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
+        const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
+        const float2 wo = cmul(twq(q), O);
+        out[q] = make_float2(E.x + wo.x, E.y + wo.y);
+        if (2 * q != M) out[M - q] = make_float2(E.x - wo.x, wo.y - E.y);
+    }
+    for (int q = M + 1 + threadIdx.x; q < PL::WP; q += PL::ROW_T) out[q] = make_float2(0.f, 0.f);
+}
+
 template <class PL>
 __global__ void __launch_bounds__(PL::ROW_T) k1_fwd_rows(const uint16_t* __restrict__ raw,
                                                          float2* __restrict__ G, int tile0,
@@ -127,25 +149,12 @@ __global__ void __launch_bounds__(PL::ROW_T) k1_fwd_rows(const uint16_t* __restr
     // stage 2 writes Z[n] back into the slot it read it from (in place, per thread)
     FftRun<typename PL::Row, -1, L, T, RowMap>::run(src, xc, xc, tw2);
     __syncthreads();
-    // Real-to-complex post-processing, q in [0, M] (Z[M] == Z[0]):
-    //   E = (Z[q] + conj Z[M-q]) / 2,  O = (Z[q] - conj Z[M-q]) / (2i),  X[q] = E + w_W^q O
 #pragma unroll 1
-    for (int line = 0; line < L; ++line) {
-        float2* out = G + ((size_t)blockIdx.y * PL::H + y0 + line) * PL::WP;
-        for (int q = threadIdx.x; q < PL::WP; q += T) {
-            float2 X = make_float2(0.f, 0.f);
-            if (q <= M) {
-                const float2 zq = xc.nat(line, q == M ? 0 : q);
-                const float2 zm = xc.nat(line, q == 0 ? 0 : M - q);
-                const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
-                const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
-                const float2 wo = cmul(__ldg(&twW[q]), O);
-                X = make_float2(E.x + wo.x, E.y + wo.y);
-            }
-            out[q] = X;
-        }
-    }
+    for (int line = 0; line < L; ++line)
+        r2c_post_line<PL>(xc, line, G + ((size_t)blockIdx.y * PL::H + y0 + line) * PL::WP,
+                          [&](int q) { return __ldg(&twW[q]); });
 }
+
 
 // ------------------------------------------------------------------ K2 ----
 template <class PL>
@@ -560,21 +569,9 @@ __global__ void __launch_bounds__(PL::ROW_T) k1p_fwd_rows(const uint16_t* __rest
         __syncthreads();
         float2* out0 = G + ((size_t)tl * PL::H + y0) * PL::WP;
 #pragma unroll 1
-        for (int line = 0; line < L; ++line) {
-            float2* out = out0 + (size_t)line * PL::WP;
-            for (int q = threadIdx.x; q < PL::WP; q += T) {
-                float2 X = make_float2(0.f, 0.f);
-                if (q <= M) {
-                    const float2 zq = xc.nat(line, q == M ? 0 : q);
-                    const float2 zm = xc.nat(line, q == 0 ? 0 : M - q);
-                    const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
-                    const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
-                    const float2 wo = cmul(twWs[q], O);
-                    X = make_float2(E.x + wo.x, E.y + wo.y);
-                }
-                out[q] = X;
-            }
-        }
+        for (int line = 0; line < L; ++line)
+            r2c_post_line<PL>(xc, line, out0 + (size_t)line * PL::WP,
+                              [&](int q) { return twWs[q]; });
         __syncthreads();   // exchange free
     }
 }

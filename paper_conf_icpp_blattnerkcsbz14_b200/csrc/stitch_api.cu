@@ -267,6 +267,13 @@ struct stitch_ctx {
         int64_t launches;
     };
     std::map<uint64_t, GraphRec> graphs;
+    // concurrent schedule (timing off): forward chunks, pair chunks and CCF chunks on three
+    // internal streams joined by events, so compute-bound and memory-bound kernels overlap
+    bool concurrent = true;
+    cudaStream_t s_fwd = nullptr, s_pair = nullptr, s_ccf = nullptr;
+    std::vector<cudaEvent_t> ev_fwd, ev_k4;   // per forward chunk / per pair chunk
+    cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
+    std::vector<int> pair_need;               // forward chunk completing each pair chunk's tiles
     int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     float ms[4] = {0, 0, 0, 0};
@@ -354,6 +361,15 @@ void stitch_destroy(stitch_ctx* ctx) {
         if (e) cudaEventDestroy(e);
     for (auto& g : ctx->graphs) cudaGraphExecDestroy(g.second.exec);
     if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
+    for (auto& e : ctx->ev_fwd)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : ctx->ev_k4)
+        if (e) cudaEventDestroy(e);
+    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
+    for (auto& e : ctx->ev_join)
+        if (e) cudaEventDestroy(e);
+    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf})
+        if (st) cudaStreamDestroy(st);
     if (ctx->own_mem && ctx->mem) cudaFree(ctx->mem);
     if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
     delete ctx;
@@ -397,6 +413,28 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         ctx->grid_colp = (env && env[0] == '1') ? sms : 0;
         const char* genv = std::getenv("STITCH_GRAPH");   // STITCH_GRAPH=0: direct launches
         ctx->use_graph = !(genv && genv[0] == '0');
+        const char* cenv = std::getenv("STITCH_CONCURRENT");  // STITCH_CONCURRENT=0: one stream
+        ctx->concurrent = !(cenv && cenv[0] == '0');
+        if (ctx->concurrent) {
+            for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf})
+                if (cudaStreamCreateWithFlags(st, cudaStreamNonBlocking) != cudaSuccess)
+                    return bail(STITCH_ERR_CUDA);
+            const int nf = (L.nlocal + L.chunk_tiles - 1) / L.chunk_tiles;
+            const int nc = (int)((L.npairs + L.chunk_pairs - 1) / L.chunk_pairs);
+            ctx->ev_fwd.assign(nf, nullptr);
+            ctx->ev_k4.assign(nc, nullptr);
+            for (auto& e : ctx->ev_fwd)
+                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                    return bail(STITCH_ERR_CUDA);
+            for (auto& e : ctx->ev_k4)
+                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                    return bail(STITCH_ERR_CUDA);
+            if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess)
+                return bail(STITCH_ERR_CUDA);
+            for (auto& e : ctx->ev_join)
+                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                    return bail(STITCH_ERR_CUDA);
+        }
         if (ctx->use_graph &&
             cudaStreamCreateWithFlags(&ctx->cap_stream, cudaStreamNonBlocking) != cudaSuccess)
             return bail(STITCH_ERR_CUDA);
@@ -509,6 +547,13 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         }
     }
     ctx->res_h.resize((size_t)L.npairs);
+    // forward chunk that completes every tile a pair chunk reads (concurrent schedule)
+    for (int64_t p0 = 0; p0 < L.npairs; p0 += L.chunk_pairs) {
+        int mx = 0;
+        for (int64_t p = p0; p < L.npairs && p < p0 + L.chunk_pairs; ++p)
+            mx = std::max(mx, std::max(pl[(size_t)p].a, pl[(size_t)p].b));
+        ctx->pair_need.push_back(mx / L.chunk_tiles);
+    }
     if ((e = cudaMemcpyAsync(ctx->twM, tw.data(), tw.size() * sizeof(float2),
                              cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
         return bail(STITCH_ERR_CUDA);
@@ -659,6 +704,73 @@ static stitch_status step_begin(stitch_ctx* ctx) {
 // timing -- as a CUDA graph captured once per key on the internal capture stream and
 // replayed on the caller's stream.  Every launch parameter (pointers, tensor maps, chunk
 // schedule) is fixed per context, so a replay is exactly the captured sequence.
+// Whole step on three streams (timing off): s_fwd runs the forward chunks (K1, K2) and
+// records an event per chunk; s_pair runs the pair chunks (K3, K4), each waiting for the
+// forward chunk that completes the tiles it reads; s_ccf runs K5 per pair chunk behind
+// its K4, then K6.  Buffers G (s_fwd) and Q (s_pair) are only touched by one stream.
+static stitch_status compute_concurrent(stitch_ctx* ctx) {
+    const PlanOps* o = ctx->ops;
+    cudaStream_t m = ctx->stream;
+    const int64_t np = ctx->L.npairs;
+    const int nl = ctx->L.nlocal, ct = ctx->L.chunk_tiles, cp = ctx->L.chunk_pairs;
+    if (np > 0) {
+        CK(cudaMemsetAsync(ctx->keys, 0, (size_t)np * sizeof(unsigned long long), m), "memset");
+        CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), m), "memset");
+    }
+    CK(cudaEventRecord(ctx->ev_fork, m), "fork");
+    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf})
+        CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
+    cudaStream_t sf = ctx->s_fwd, sp = ctx->s_pair, sk = ctx->s_ccf;
+    for (int f = 0, t0 = 0; t0 < nl; ++f, t0 += ct) {
+        const int nt = nl - t0 < ct ? nl - t0 : ct;
+        if (ctx->grid_k1p > 0)
+            o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, sf);
+        else
+            o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, sf);
+        if (ctx->grid_colp > 0)
+            o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, sf);
+        else
+            o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, sf);
+        CK(cudaEventRecord(ctx->ev_fwd[f], sf), "event");
+        ctx->launches += 2;
+    }
+    int waited = -1;
+    for (int c = 0; (int64_t)c * cp < np; ++c) {
+        const int64_t p0 = (int64_t)c * cp;
+        const int npc = (int)(np - p0 < cp ? np - p0 : cp);
+        const int need = ctx->pair_need[c];
+        if (need > waited) {
+            CK(cudaStreamWaitEvent(sp, ctx->ev_fwd[need], 0), "wait forward");
+            waited = need;
+        }
+        if (ctx->grid_colp > 0)
+            o->k3p(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, ctx->grid_colp, sp);
+        else
+            o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, sp);
+        if (ctx->grid_k4p > 0)
+            o->k4p(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, ctx->grid_k4p, sp);
+        else
+            o->k4(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, sp);
+        CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
+        CK(cudaStreamWaitEvent(sk, ctx->ev_k4[c], 0), "wait k4");
+        o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, sk);
+        ctx->launches += 3;
+    }
+    if (np > 0) {
+        k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(ctx->keys, ctx->mom, ctx->res,
+                                                                  ctx->H, ctx->W, (int)np);
+        ctx->launches += 1;
+    }
+    CK(cudaGetLastError(), "concurrent launch");
+    cudaStream_t ss[3] = {sf, sp, sk};
+    for (int i = 0; i < 3; ++i) {
+        CK(cudaEventRecord(ctx->ev_join[i], ss[i]), "join");
+        CK(cudaStreamWaitEvent(m, ctx->ev_join[i], 0), "join wait");
+    }
+    ctx->computed = true;
+    return STITCH_OK;
+}
+
 extern "C++" {
 template <class F>
 static stitch_status run_graphed(stitch_ctx* ctx, uint64_t key, F body) {
@@ -728,6 +840,7 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
     st = run_graphed(ctx, 1ull << 60, [&]() {
+        if (ctx->concurrent && !ctx->timing) return compute_concurrent(ctx);
         stitch_status s2 = forward_impl(ctx, 0, ctx->L.nlocal);
         if (s2 != STITCH_OK) return s2;
         if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
