@@ -76,13 +76,36 @@ def twiddle(e, a, num, den, sign):
     return (re, im)
 
 
+_BEST = {}
+
+
+def _cost(n, sp):
+    """Instruction count of the codelet for n when its top-level split is sp."""
+    e = Em()
+    xs = [(f"x{j}r", f"x{j}i") for j in range(n)]
+    _FORCE[n] = sp
+    try:
+        gen(e, xs, -1)
+    finally:
+        del _FORCE[n]
+    return sum(1 + l.count(" * ") * ("fmaf(" in l) for l in e.lines
+               if not (l.count("= -t") and l.count("t") == 2))
+
+
+_FORCE = {}
+
+
 def split(n):
-    if n % 4 == 0 and n != 4:
-        return 4, n // 4
-    for p in range(2, n):
-        if n % p == 0:
-            return p, n // p
-    return None
+    """Cooley-Tukey split n = n1 * n2 of a composite radix, chosen (recursively, memoised)
+    to minimise the straight-line instruction count; None for a prime."""
+    if n in _FORCE:
+        return _FORCE[n]
+    divs = [d for d in range(2, n) if n % d == 0]
+    if not divs:
+        return None
+    if n not in _BEST:
+        _BEST[n] = min(((d, n // d) for d in divs), key=lambda sp: (_cost(n, sp), sp))
+    return _BEST[n]
 
 
 def gen(e, xs, sign):
