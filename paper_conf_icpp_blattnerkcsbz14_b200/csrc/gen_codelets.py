@@ -108,6 +108,76 @@ def split(n):
     return _BEST[n]
 
 
+def primitive_root(p):
+    for g in range(2, p):
+        if all(pow(g, (p - 1) // q, p) != 1 for q in range(2, p) if (p - 1) % q == 0
+               and all(q % r for r in range(2, q))):
+            return g
+    raise ValueError(p)
+
+
+def prime_rader(e, xs, sign):
+    """Prime p with h = (p-1)/2 even: symmetric form with the cosine half evaluated as a
+    cyclic correlation of length h (Rader ordering j = g^a, k = g^-b; C_m = cos(2 pi g^m/p)
+    is h-periodic) split by CRT into a cyclic and a negacyclic correlation of length h/2:
+    126 instead of 196 FMAs per component at p = 29.  The sine half (anti-periodic, a
+    negacyclic correlation) stays direct."""
+    n = len(xs)
+    h = (n - 1) // 2
+    g = primitive_root(n)
+    ja = [pow(g, a, n) for a in range(h)]                    # representatives of +-j
+    kb = [pow(g, (n - 1 - b) % (n - 1), n) for b in range(h)]  # g^-b
+    s = [cadd(e, xs[j], xs[n - j]) for j in ja]
+    d = [csub(e, xs[j], xs[n - j]) for j in ja]
+    acc = xs[0]
+    for a in range(h):
+        acc = cadd(e, acc, s[a])
+    out = [None] * n
+    out[0] = acc
+    q = h // 2
+    C = [math.cos(2.0 * math.pi * pow(g, m, n) / n) for m in range(h)]
+    P = [0.5 * (C[m] + C[(m + q) % h]) for m in range(q)]    # period q
+    Nm = [0.5 * (C[m] - C[(m + q) % h]) for m in range(h)]   # anti-periodic (q), index mod h
+    A = [[None, None] for _ in range(h)]
+    for comp in (0, 1):
+        up = [e.let(f"{s[a][comp]} + {s[a + q][comp]}") for a in range(q)]
+        um = [e.let(f"{s[a][comp]} - {s[a + q][comp]}") for a in range(q)]
+        for b in range(q):
+            pp = xs[0][comp]
+            for a in range(q):
+                pp = e.let(f"fmaf({up[a]}, {flit(P[(a - b) % q])}, {pp})")
+            nn = None
+            for a in range(q):
+                m = a - b                      # N_{a-b}: N_{m+q} = -N_m
+                c = Nm[m] if m >= 0 else -Nm[m + q]
+                nn = e.let(f"{um[a]} * {flit(c)}") if nn is None else \
+                    e.let(f"fmaf({um[a]}, {flit(c)}, {nn})")
+            A[b][comp] = e.let(f"{pp} + {nn}")
+            A[b + q][comp] = e.let(f"{pp} - {nn}")
+    for b in range(h):
+        k = kb[b]
+        br = bi = None
+        for a in range(h):
+            sn = math.sin(2.0 * math.pi * ((ja[a] * k) % n) / n)
+            if br is None:
+                br = e.let(f"{d[a][0]} * {flit(sn)}")
+                bi = e.let(f"{d[a][1]} * {flit(sn)}")
+            else:
+                br = e.let(f"fmaf({d[a][0]}, {flit(sn)}, {br})")
+                bi = e.let(f"fmaf({d[a][1]}, {flit(sn)}, {bi})")
+        ar, ai = A[b]
+        if sign < 0:
+            out[k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
+            out[n - k] = (e.let(f"{ar} - {bi}"), e.let(f"{ai} + {br}"))
+        else:
+            out[k] = (e.let(f"{ar} - {bi}"), e.let(f"{ai} + {br}"))
+            out[n - k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
+    return out
+
+
+RADER_MIN = 13   # primes from here use prime_rader (h even); smaller ones the plain form
+
+
 def gen(e, xs, sign):
     n = len(xs)
     if n == 1:
@@ -115,6 +185,8 @@ def gen(e, xs, sign):
     if n == 2:
         return [cadd(e, xs[0], xs[1]), csub(e, xs[0], xs[1])]
     sp = split(n)
+    if sp is None and n >= RADER_MIN and ((n - 1) // 2) % 2 == 0:
+        return prime_rader(e, xs, sign)
     if sp is None:                     # prime: symmetric form
         h = (n - 1) // 2
         s = [None] + [cadd(e, xs[j], xs[n - j]) for j in range(1, h + 1)]

@@ -653,7 +653,7 @@ __global__ void __launch_bounds__(PL::ROW_T) k4p_pair_rows(const float2* __restr
 //   candidate dx = W-x : a = A[dy+i][W - x + j],  j <  x
 // accumulating the exact integer moments Sa, Sb, Saa, Sbb, Sab (u32 / u64 wide MADs).
 constexpr int CCF_ROWS = 64;   // rows of one group per CTA
-constexpr int CCF_BATCH = 8;   // rows staged in shared memory at a time (one warp per row)
+constexpr int CCF_BATCH = 4;   // rows staged in shared memory at a time (two warps per row)
 constexpr int CCF_T = 256;
 
 __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v) {
@@ -663,7 +663,7 @@ __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
 }
 
 struct Moments {
-    uint32_t sa = 0, sb = 0;  // <= CCF_ROWS/CCF_BATCH * ceil(W/32) * 65535 < 2^32 per lane
+    uint32_t sa = 0, sb = 0;  // <= CCF_ROWS/CCF_BATCH * ceil(W/64) * 65535 < 2^32 per lane
     unsigned long long saa = 0, sbb = 0, sab = 0;
     __device__ __forceinline__ void add(uint32_t a, uint32_t b) {
         sa += a;
@@ -675,20 +675,23 @@ struct Moments {
 };
 
 // Moments of one candidate over one staged row: a = ar[off + j], b = br[j], j < w.
-// Lane l takes j = l + 32k (conflict-free 2-byte shared loads), unrolled by 4.
-__device__ __forceinline__ void row_moments(Moments& m, const uint16_t* ar, const uint16_t* br,
-                                            int off, int w, int lane) {
-    const uint16_t* a = ar + off + lane;
-    const uint16_t* b = br + lane;
-    const int n = w - lane;                  // elements this lane may touch: j' = 32k < n
+// The two warps of a row interleave: lane l of half h takes j = 32h + l + 64k
+// (conflict-free 2-byte shared loads), alternating two accumulator sets so the wide
+// multiply-add chains overlap.  (A single pass pairing each B pixel with both candidates
+// was measured 2x slower: the compiler predicates both candidates' bodies everywhere.)
+__device__ __forceinline__ void row_moments(Moments& m, Moments& m2, const uint16_t* ar,
+                                            const uint16_t* br, int off, int w, int j0) {
+    const uint16_t* a = ar + off + j0;
+    const uint16_t* b = br + j0;
+    const int n = w - j0;                    // this lane touches j' = 64k < n
     int k = 0;
-    for (; k + 96 < n; k += 128) {
+    for (; k + 192 < n; k += 256) {
         m.add(a[k], b[k]);
-        m.add(a[k + 32], b[k + 32]);
-        m.add(a[k + 64], b[k + 64]);
-        m.add(a[k + 96], b[k + 96]);
+        m2.add(a[k + 64], b[k + 64]);
+        m.add(a[k + 128], b[k + 128]);
+        m2.add(a[k + 192], b[k + 192]);
     }
-    for (; k < n; k += 32) m.add(a[k], b[k]);
+    for (; k < n; k += 64) m.add(a[k], b[k]);
 }
 
 template <int W, int H>
@@ -736,7 +739,8 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
         __syncthreads();
     }
     const int w0 = W - x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    Moments m0, m1;
+    const int rrow = warp >> 1, j0 = 32 * (warp & 1) + lane;   // two warps per staged row
+    Moments m0, m1, m0b, m1b;
     for (int bi = 0; bi < nbatch; ++bi) {
         const int rows = min(CCF_BATCH, rows_total - bi * CCF_BATCH);
         const int buf = bi % BUFS;
@@ -756,16 +760,19 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
             }
             __syncthreads();
         }
-        if (warp < rows) {                     // one warp per staged row
-            const uint16_t* ar = bufA(buf) + warp * W;
-            const uint16_t* br = bufB(buf) + warp * W;
-            row_moments(m0, ar, br, x, w0, lane);   // candidate dx = x
-            row_moments(m1, ar, br, w0, x, lane);   // candidate dx = W - x
+        if (rrow < rows) {
+            const uint16_t* ar = bufA(buf) + rrow * W;
+            const uint16_t* br = bufB(buf) + rrow * W;
+            row_moments(m0, m0b, ar, br, x, w0, j0);   // candidate dx = x
+            row_moments(m1, m1b, ar, br, w0, x, j0);   // candidate dx = W - x
         }
         __syncthreads();                       // buffer free for batch bi+2
     }
-    unsigned long long v[10] = {m0.sa, m0.sb, m0.saa, m0.sbb, m0.sab,
-                                m1.sa, m1.sb, m1.saa, m1.sbb, m1.sab};
+    unsigned long long v[10] = {
+        (unsigned long long)m0.sa + m0b.sa, (unsigned long long)m0.sb + m0b.sb, m0.saa + m0b.saa,
+        m0.sbb + m0b.sbb, m0.sab + m0b.sab,
+        (unsigned long long)m1.sa + m1b.sa, (unsigned long long)m1.sb + m1b.sb, m1.saa + m1b.saa,
+        m1.sbb + m1b.sbb, m1.sab + m1b.sab};
 #pragma unroll
     for (int q = 0; q < 10; ++q) {
         v[q] = warp_sum_u64(v[q]);
