@@ -173,13 +173,15 @@ struct LandSrc {  // a landed complex panel [H][COL_P] in shared memory
 // Resident spectrum code: the phase of F in 31-bit fixed point (top bits, 2^32 per turn)
 // plus a nonzero flag (bit 0).  Step 3 needs only phases: F_A conj(F_B) / |F_A conj(F_B)|
 // = exp(i (phi_A - phi_B)), and 0 where F_A or F_B vanishes (reading C4).
-// atan2(y, x) / pi in (-1, 1]: octant reduction + a degree-8 polynomial in t^2 for
-// atan(t)/pi on [0, 1] (coefficients fitted in double, max error 1.6e-7 rad in fp32;
-// the fp32 spectrum's own phase error is ~1e-6 rad).
-__device__ __forceinline__ float atan2_halfturns(float y, float x) {
-    const float ax = fabsf(x), ay = fabsf(y);
+// Phase code of v: atan2(v.y, v.x) / pi in [-1, 1] by octant reduction + a degree-8
+// polynomial in t^2 for atan(t)/pi on [0, 1] (coefficients fitted in double, max error
+// 1.6e-7 rad in fp32; the fp32 spectrum's own phase error is ~1e-6 rad), scaled to 2^31
+// per half turn; bit 0 = nonzero flag.  A zero v gives t = 0*inf = NaN -> an arbitrary
+// code with flag 0, which makes every NCPS product with it 0 (reading C4).
+__device__ __forceinline__ uint32_t phase_code(float2 v) {
+    const float ax = fabsf(v.x), ay = fabsf(v.y);
     const float mx = fmaxf(ax, ay), mn = fminf(ax, ay);
-    const float t = mx > 0.f ? __fdividef(mn, mx) : 0.f;
+    const float t = __fdividef(mn, mx);
     const float s = t * t;
     float p = 0.0009368208120577037f;
     p = fmaf(p, s, -0.00521085737273097f);
@@ -190,16 +192,12 @@ __device__ __forceinline__ float atan2_halfturns(float y, float x) {
     p = fmaf(p, s, 0.06363658607006073f);
     p = fmaf(p, s, -0.10610226541757584f);
     p = fmaf(p, s, 0.31830987334251404f);
-    float r = p * t;                       // atan(mn/mx) / pi in [0, 1/4]
-    if (ay > ax) r = 0.5f - r;
-    if (x < 0.f) r = 1.0f - r;
-    return y < 0.f ? -r : r;
-}
-
-__device__ __forceinline__ uint32_t phase_code(float2 v) {
-    const float t = atan2_halfturns(v.y, v.x);                       // [-1, 1]
-    const int32_t q = __float2int_rn(t * 2147483648.0f);            // saturates at t = 1
-    return ((uint32_t)q & ~1u) | ((v.x != 0.f || v.y != 0.f) ? 1u : 0u);
+    float r = p * t;                                 // atan(mn/mx) / pi in [0, 1/4]
+    r = ay > ax ? 0.5f - r : r;
+    r = v.x < 0.f ? 1.0f - r : r;
+    r = copysignf(r, v.y);                           // [-1, 1]
+    const int32_t q = __float2int_rn(r * 2147483648.0f);   // saturates at r = 1
+    return ((uint32_t)q & ~1u) | (mx > 0.f ? 1u : 0u);
 }
 
 template <class PL>

@@ -125,3 +125,37 @@ def test_generated_codelets_are_dfts():
         j = np.arange(n)
         ref = np.exp(sign * 2j * math.pi * np.outer(j, j) / n) @ x
         assert np.abs(got - ref).max() <= 1e-6 * np.abs(ref).max(), (n, tag)
+
+
+def test_phase_code_polynomial_matches_atan2():
+    """The K2 phase encoder's atan2 (octant reduction + fitted polynomial, pciam_kernels.cuh)
+    re-evaluated in float32 on the host: within 3e-7 rad of the exact angle, and the
+    NCPS decoder's wrap-around difference of two codes recovers phase differences."""
+    src = open(os.path.join(ROOT, "paper_conf_icpp_blattnerkcsbz14_b200", "csrc",
+                            "pciam_kernels.cuh")).read()
+    body = src[src.index("__device__ __forceinline__ uint32_t phase_code"):]
+    body = body[:body.index("\n}\n")]
+    coef = [float(c) for c in re.findall(r"fmaf\(p, s, (-?\d\.\d+)f\)", body)]
+    coef = [float(re.search(r"float p = (-?\d\.\d+)f;", body).group(1))] + coef
+    assert len(coef) == 9
+    rng = np.random.default_rng(5)
+    z = (rng.standard_normal(200000) + 1j * rng.standard_normal(200000)).astype(np.complex64)
+    x, y = z.real.astype(np.float32), z.imag.astype(np.float32)
+    ax, ay = np.abs(x), np.abs(y)
+    mx, mn = np.maximum(ax, ay), np.minimum(ax, ay)
+    t = (mn / mx).astype(np.float32)
+    s = (t * t).astype(np.float32)
+    p = np.float32(coef[0])
+    for c in coef[1:]:
+        p = (p * s + np.float32(c)).astype(np.float32)
+    r = (p * t).astype(np.float32)
+    r = np.where(ay > ax, np.float32(0.5) - r, r)
+    r = np.where(x < 0, np.float32(1.0) - r, r)
+    r = np.copysign(r, y)
+    err = np.abs(np.angle(np.exp(1j * (np.pi * r.astype(np.float64) - np.angle(z.astype(np.complex128))))))
+    assert err.max() <= 3e-7
+    q = np.clip(np.rint(r.astype(np.float64) * 2**31), -2**31, 2**31 - 1).astype(np.int64)
+    code = (q.astype(np.uint32) & np.uint32(0xFFFFFFFE)) | np.uint32(1)
+    d = (code[:-1] - code[1:]).astype(np.uint32).view(np.int32).astype(np.float64) * (2 * np.pi / 2**32)
+    ref = np.angle(z[:-1].astype(np.complex128) * np.conj(z[1:].astype(np.complex128)))
+    assert np.abs(np.angle(np.exp(1j * (d - ref)))).max() <= 1e-6
