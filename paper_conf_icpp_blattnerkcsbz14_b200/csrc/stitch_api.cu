@@ -204,8 +204,8 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     int64_t np = 0;
     for (int t = L->t_begin; t < L->t_end; ++t) np += (t % m >= 1) + (t / m >= 1);
     L->npairs = np;
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 32;
-    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 16;
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 64;
+    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 32;
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     size_t o = 0;
