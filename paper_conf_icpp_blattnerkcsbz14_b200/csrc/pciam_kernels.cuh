@@ -550,6 +550,8 @@ __global__ void __launch_bounds__(PL::ROW_T) k1p_fwd_rows(const uint16_t* __rest
     __syncthreads();
     // One landing buffer: block k+1's rows are fetched (TMA bulk copy) as soon as stage 1
     // of block k has consumed them, overlapping stage 2 + post-processing of block k.
+    // Round robin over row blocks: neighbouring CTAs read neighbouring raw rows
+    // (measured faster than contiguous per-CTA ranges here).
     if (threadIdx.x == 0 && (int)blockIdx.x < nblk) issue(blockIdx.x, 0);
     int k = 0;
     for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++k) {
@@ -589,7 +591,7 @@ struct C2RSmemSrc {  // C2R pre-processing from a landed Q row block (pitch LP)
 };
 
 template <class PL>
-__global__ void __launch_bounds__(PL::ROW_T) k4p_pair_rows(const float2* __restrict__ Q,
+__global__ void __launch_bounds__(PL::ROW_T, 4) k4p_pair_rows(const float2* __restrict__ Q,
                                                            unsigned long long* __restrict__ keys,
                                                            int pair0, int npairs,
                                                            const float2* __restrict__ tw2,
@@ -617,25 +619,43 @@ __global__ void __launch_bounds__(PL::ROW_T) k4p_pair_rows(const float2* __restr
     }
     for (int i = threadIdx.x; i < PL::ROW_TW2; i += T) tw2s[i] = __ldg(tw2 + i);
     __syncthreads();
-    // One landing buffer, refilled (TMA bulk copies) as soon as stage 1 consumed it.
-    if (threadIdx.x == 0 && (int)blockIdx.x < nblk) issue(blockIdx.x, 0);
+    // Each CTA walks a contiguous range of row blocks (consecutive rows of mostly one pair):
+    // one landing buffer, refilled (TMA bulk copies) as soon as stage 1 consumed it; the
+    // running (max, index) of every thread carries across the blocks of a pair and is
+    // reduced (block reduction + one atomicMax) only when the pair changes.
+    const int b0 = (int)((long long)nblk * blockIdx.x / gridDim.x);
+    const int b1 = (int)((long long)nblk * (blockIdx.x + 1) / gridDim.x);
+    if (threadIdx.x == 0 && b0 < b1) issue(b0, 0);
+    ArgmaxDst acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
+    int cur = -1;
     int k = 0;
-    for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++k) {
-        mbar_wait(&bar[0], k & 1);
+    for (int blk = b0; blk < b1; ++blk, ++k) {
         const int pl = blk / BPP, y0 = (blk - pl * BPP) * L;
-        const int nxt = blk + gridDim.x;
+        if (pl != cur) {                                   // block-uniform
+            if (cur >= 0) {
+                const unsigned long long best = block_max_u64<T>(acc.key());
+                if (threadIdx.x == 0) atomicMax(&keys[pair0 + cur], best);
+            }
+            cur = pl;
+            acc.best_v = -1.f;
+            acc.best_i = 0xFFFFFFFFu;
+        }
+        acc.row_base = y0;
+        mbar_wait(&bar[0], k & 1);
+        const int nxt = blk + 1;
         C2RSmemSrc<PL> src{land, twW};
-        ArgmaxDst dst{-1.f, 0xFFFFFFFFu, y0, PL::W};
         auto prefetch = [&]() {
-            if (threadIdx.x == 0 && nxt < nblk) {
+            if (threadIdx.x == 0 && nxt < b1) {
                 fence_proxy_async();
                 issue(nxt, 0);
             }
         };
-        FftRun<typename PL::Row, +1, L, T, RowMap, true>::run(src, xc, dst, tw2s, prefetch);
-        const unsigned long long best = block_max_u64<T>(dst.key());
-        if (threadIdx.x == 0) atomicMax(&keys[pair0 + pl], best);
-        __syncthreads();   // exchange and reduction scratch free
+        FftRun<typename PL::Row, +1, L, T, RowMap, true>::run(src, xc, acc, tw2s, prefetch);
+        __syncthreads();   // exchange free for the next block
+    }
+    if (cur >= 0) {
+        const unsigned long long best = block_max_u64<T>(acc.key());
+        if (threadIdx.x == 0) atomicMax(&keys[pair0 + cur], best);
     }
 }
 
@@ -732,9 +752,9 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
             mbar_init(&bar[0], 1);
             mbar_init(&bar[1], 1);
             fence_mbar_init();
-            issue(0);
         }
         __syncthreads();
+        if (threadIdx.x == 0) issue(0);
     }
     const int w0 = W - x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int rrow = warp >> 1, j0 = 32 * (warp & 1) + lane;   // two warps per staged row

@@ -1,0 +1,17 @@
+#!/bin/bash
+# compute-sanitizer passes over config 1 (3x3 grid of 256x192) and a 2x2 grid of 1392x1040
+# (run on the GPU box).  Graphs/concurrency off so every launch is checked directly.
+export STITCH_GRAPH=0
+SMOKE='import __graft_entry__ as g; g.smoke()'
+BIG='import numpy as np, synthgrid; from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid
+g = synthgrid.make_grid(2, 2, 1040, 1392)
+p = PciamGrid(2, 2, 1040, 1392, chunk_pairs=2, chunk_tiles=2); p.load_grid(g.tiles); w, n = p.compute_translations()
+print("big ok", w["dx"].tolist(), n["dy"].tolist())'
+for tool in memcheck racecheck synccheck initcheck; do
+  echo "== $tool (config 1)"
+  timeout 900 compute-sanitizer --tool $tool --print-limit 20 python -c "$SMOKE" 2>&1 | tail -6
+done
+for tool in memcheck racecheck; do
+  echo "== $tool (2x2 @ 1392x1040)"
+  timeout 1200 compute-sanitizer --tool $tool --print-limit 20 python -c "$BIG" 2>&1 | tail -6
+done
