@@ -196,7 +196,9 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
         {   // stage 2: radix R1 over R0 butterflies per line, exchange -> destination
             constexpr int TOTAL = L * R0;
             constexpr int ITER = (TOTAL + T - 1) / T;
-#pragma unroll
+            // not unrolled: one copy of the (large) butterfly + epilogue keeps the kernel
+            // inside the instruction cache
+#pragma unroll 1
             for (int it = 0; it < ITER; ++it) {
                 const int g = threadIdx.x + it * T;
                 if (TOTAL % T == 0 || g < TOTAL) {
