@@ -659,6 +659,10 @@ __global__ void __launch_bounds__(PL::ROW_T, 4) k4p_pair_rows(const float2* __re
     }
 }
 
+}  // namespace stitch
+#include "warp_rows.cuh"
+namespace stitch {
+
 // ------------------------------------------------------------------ K5 ----
 // Candidate overlaps of pair p (Fig. 2 l.8-11 unified, Fig. 3): candidate (dx, dy) has
 // region a = A[dy:H, dx:W], b = B[0:H-dy, 0:W-dx].  c1 = (x, y) and c2 = (W-x, y) share

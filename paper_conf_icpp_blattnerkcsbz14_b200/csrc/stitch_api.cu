@@ -36,7 +36,7 @@ using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 32, 8, 32, 0, 0>;
 struct PlanOps {
     int W, H, M, WC, WP, row_l, col_p;
     int row_r0, row_r1, col_r0, col_r1;  // stage radices (r1 = 1: single stage)
-    cudaError_t (*setup)(int* grid_k1p, int* grid_k4p);  // persistent grids (0 = not used)
+    cudaError_t (*setup)(int* grid_k1p, int* grid_k4p, int* grid_k1w, int* grid_k4w);
     void (*k1p)(const uint16_t*, float2*, int, int, const float2*, const float2*, int, cudaStream_t);
     void (*k4p)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
                 cudaStream_t);
@@ -45,6 +45,9 @@ struct PlanOps {
     void (*k2p)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, int,
                 cudaStream_t);
     void (*k3p)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
+                cudaStream_t);
+    void (*k1w)(const uint16_t*, float2*, int, int, const float2*, const float2*, int, cudaStream_t);
+    void (*k4w)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
                 cudaStream_t);
     void (*k1)(const uint16_t*, float2*, int, int, const float2*, const float2*, cudaStream_t);
     void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, cudaStream_t);
@@ -63,8 +66,9 @@ cudaError_t max_smem(K* kernel, size_t bytes) {
 }
 
 template <class PL>
-cudaError_t plan_setup(int* grid_k1p, int* grid_k4p) {
+cudaError_t plan_setup(int* grid_k1p, int* grid_k4p, int* grid_k1w, int* grid_k4w) {
     cudaError_t e;
+    *grid_k1w = *grid_k4w = 0;
     using RP = RowPersist<PL>;
     int dev = 0, sms = 0, nb = 0;
     if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
@@ -87,6 +91,21 @@ cudaError_t plan_setup(int* grid_k1p, int* grid_k4p) {
     if ((e = max_smem(k2p_fwd_cols<PL, true>, PL::COLP_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k2p_fwd_cols<PL, false>, PL::COLP_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k3p_pair_cols<PL>, PL::COLP_SMEM)) != cudaSuccess) return e;
+    if constexpr (RowWarp<PL>::OK) {
+        using RW = RowWarp<PL>;
+        if ((e = max_smem(k1w_fwd_rows<PL>, RW::SMEM_K1)) != cudaSuccess) return e;
+        if ((e = max_smem(k4w_pair_rows<PL>, RW::SMEM_K4)) != cudaSuccess) return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1w_fwd_rows<PL>,
+                                                                32 * ROWW_WARPS, RW::SMEM_K1)) !=
+            cudaSuccess)
+            return e;
+        *grid_k1w = nb * sms;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k4w_pair_rows<PL>,
+                                                                32 * ROWW_WARPS, RW::SMEM_K4)) !=
+            cudaSuccess)
+            return e;
+        *grid_k4w = nb * sms;
+    }
     if ((e = max_smem(k1_fwd_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k4_pair_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
     if ((e = max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM)) != cudaSuccess) return e;
@@ -156,6 +175,26 @@ void launch_k3p(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0,
 }
 
 template <class PL>
+void launch_k1w(const uint16_t* raw, float2* G, int t0, int nt, const float2* tw2,
+                const float2* twW, int grid, cudaStream_t s) {
+    if constexpr (RowWarp<PL>::OK) {
+        const int warps = (nt * PL::H + 0) / 1;
+        const int need = (warps + ROWW_WARPS - 1) / ROWW_WARPS;
+        k1w_fwd_rows<PL><<<grid < need ? grid : need, 32 * ROWW_WARPS, RowWarp<PL>::SMEM_K1, s>>>(
+            raw, G, t0, nt, tw2, twW);
+    }
+}
+template <class PL>
+void launch_k4w(const float2* Q, unsigned long long* keys, int p0, int np, const float2* tw2,
+                const float2* twW, int grid, cudaStream_t s) {
+    if constexpr (RowWarp<PL>::OK) {
+        const int need = (np * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
+        k4w_pair_rows<PL><<<grid < need ? grid : need, 32 * ROWW_WARPS, RowWarp<PL>::SMEM_K4, s>>>(
+            Q, keys, p0, np, tw2, twW);
+    }
+}
+
+template <class PL>
 void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long long* keys,
                unsigned long long* mom, int p0, int np, cudaStream_t s) {
     k5_ccf_moments<PL::W, PL::H><<<dim3(k5_grid_x(PL::H), np), CCF_T, k5_smem_bytes(PL::W), s>>>(
@@ -167,8 +206,8 @@ PlanOps make_ops() {
     return PlanOps{PL::W,       PL::H,         PL::M,          PL::WC,        PL::WP,
                    PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
                    PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
-                   launch_k2p<PL>, launch_k3p<PL>, launch_k1<PL>, launch_k2<PL>, launch_k3<PL>,
-                   launch_k4<PL>};
+                   launch_k2p<PL>, launch_k3p<PL>, launch_k1w<PL>, launch_k4w<PL>, launch_k1<PL>,
+                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>};
 }
 
 const PlanOps* find_plan(int W, int H) {
@@ -258,6 +297,7 @@ struct stitch_ctx {
     int64_t launches = 0;
     int grid_k1p = 0, grid_k4p = 0;   // persistent-kernel grids (0: use the non-persistent kernel)
     int grid_colp = 0;                // persistent column kernels (K2p/K3p): one CTA per SM
+    int grid_k1w = 0, grid_k4w = 0;   // warp-per-line row kernels (0: not used)
     // CUDA graphs of the launch sequences (captured on first use on an internal stream,
     // replayed on the caller's stream): one graph launch per step instead of ~700 launches
     bool use_graph = true;
@@ -402,7 +442,13 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     };
     cudaError_t e = cudaSetDevice(cfg->device);
     if (e != cudaSuccess) return bail(STITCH_ERR_CUDA);
-    if ((e = ops->setup(&ctx->grid_k1p, &ctx->grid_k4p)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if ((e = ops->setup(&ctx->grid_k1p, &ctx->grid_k4p, &ctx->grid_k1w, &ctx->grid_k4w)) !=
+        cudaSuccess)
+        return bail(STITCH_ERR_CUDA);
+    {
+        const char* wenv = std::getenv("STITCH_ROWWARP");   // STITCH_ROWWARP=0: CTA row kernels
+        if (wenv && wenv[0] == '0') ctx->grid_k1w = ctx->grid_k4w = 0;
+    }
     {
         // column-kernel variant: one CTA per panel (default: several CTAs per SM overlap each
         // other's TMA waits) or persistent with TMA prefetch (STITCH_COL_PERSIST=1; one CTA
@@ -616,16 +662,34 @@ stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid,
     return load_common(ctx, dev_grid, n_bytes, cudaMemcpyDeviceToDevice);
 }
 
+// Row kernels: warp-per-line (K1w/K4w) where the plan allows, else persistent CTA rows
+// (K1p/K4p), else one CTA per row block (K1/K4).
+static void launch_k1_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
+    const PlanOps* o = ctx->ops;
+    if (ctx->grid_k1w > 0)
+        o->k1w(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1w, s);
+    else if (ctx->grid_k1p > 0)
+        o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, s);
+    else
+        o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, s);
+}
+static void launch_k4_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s) {
+    const PlanOps* o = ctx->ops;
+    if (ctx->grid_k4w > 0)
+        o->k4w(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, ctx->grid_k4w, s);
+    else if (ctx->grid_k4p > 0)
+        o->k4p(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, ctx->grid_k4p, s);
+    else
+        o->k4(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, s);
+}
+
 // Forward transforms (K1 + K2) of the resident tiles with local indices [lt0, lt0 + count).
 static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
     const PlanOps* o = ctx->ops;
     const int ct = ctx->L.chunk_tiles;
     for (int t0 = lt0; t0 < lt0 + count; t0 += ct) {
         const int nt = lt0 + count - t0 < ct ? lt0 + count - t0 : ct;
-        if (ctx->grid_k1p > 0)
-            o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, ctx->stream);
-        else
-            o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->stream);
+        launch_k1_any(ctx, t0, nt, ctx->stream);
         CK(mark(ctx, 0), "event");
         if (ctx->grid_colp > 0)
             o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, ctx->stream);
@@ -655,10 +719,7 @@ static stitch_status pairs_impl(stitch_ctx* ctx) {
             else
                 o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
             CK(mark(ctx, 2), "event");
-            if (ctx->grid_k4p > 0)
-                o->k4p(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, ctx->grid_k4p, s);
-            else
-                o->k4(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, s);
+            launch_k4_any(ctx, (int)p0, npc, s);
             CK(mark(ctx, 3), "event");
             ctx->launches += 2;
         }
@@ -723,10 +784,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx) {
     cudaStream_t sf = ctx->s_fwd, sp = ctx->s_pair, sk = ctx->s_ccf;
     for (int f = 0, t0 = 0; t0 < nl; ++f, t0 += ct) {
         const int nt = nl - t0 < ct ? nl - t0 : ct;
-        if (ctx->grid_k1p > 0)
-            o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, sf);
-        else
-            o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, sf);
+        launch_k1_any(ctx, t0, nt, sf);
         if (ctx->grid_colp > 0)
             o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, sf);
         else
@@ -747,10 +805,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx) {
             o->k3p(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, ctx->grid_colp, sp);
         else
             o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, sp);
-        if (ctx->grid_k4p > 0)
-            o->k4p(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, ctx->grid_k4p, sp);
-        else
-            o->k4(ctx->Q, ctx->keys, (int)p0, npc, ctx->twM, ctx->twW, sp);
+        launch_k4_any(ctx, (int)p0, npc, sp);
         CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
         CK(cudaStreamWaitEvent(sk, ctx->ev_k4[c], 0), "wait k4");
         o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, sk);
@@ -925,10 +980,7 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
     // with the same K1 + K2 kernels into the chunk buffer G (slot 0) and copy it out.
     const int lt = tile - ctx->L.h_begin;
     const PlanOps* o = ctx->ops;
-    if (ctx->grid_k1p > 0)
-        o->k1p(ctx->raw, ctx->G, lt, 1, ctx->twM, ctx->twW, ctx->grid_k1p, ctx->stream);
-    else
-        o->k1(ctx->raw, ctx->G, lt, 1, ctx->twM, ctx->twW, ctx->stream);
+    launch_k1_any(ctx, lt, 1, ctx->stream);
     o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->twH, false, ctx->stream);
     CK(cudaGetLastError(), "spectrum launch");
     CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->G,

@@ -1,0 +1,233 @@
+// warp_rows.cuh — warp-per-line row kernels (K1w, K4w): no CTA-wide barriers.
+//
+// The row transforms (length M = W/2 = R0*R1 with R0, R1 <= 32) are small enough for one
+// warp: stage 1 gives each of R1 lanes a radix-R0 butterfly, stage 2 each of R0 lanes a
+// radix-R1 butterfly, with the exchange in the warp's own shared-memory slice and
+// __syncwarp between the stages.  Each warp streams a contiguous range of rows: the next
+// row lands by TMA bulk copy (per-warp mbarrier) as soon as stage 1 has read the current
+// one.  Warps never wait for each other, so the scheduler always has independent work
+// (the CTA-level versions K1p/K4p lose ~1/3 of their stall cycles at barriers).
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include "async_copy.cuh"
+#include "fft_engine.cuh"
+
+namespace stitch {
+
+// Exchange slot of element (u < R0, v < R1): v*(R0+PAD) + u; natural index n = v*R0 + u.
+template <int R0, int R1, int PAD>
+struct WarpXchg {
+    float2* s;
+    static constexpr int SIZE = R1 * (R0 + PAD);
+    __device__ __forceinline__ float2& at(int u, int v) const { return s[v * (R0 + PAD) + u]; }
+    __device__ __forceinline__ float2& nat(int n) const {
+        if constexpr (PAD == 0)
+            return s[n];
+        else
+            return at(n % R0, n / R0);
+    }
+    __device__ __forceinline__ void store(int, int n, float2 v) const { nat(n) = v; }
+};
+
+template <class RX, int SIGN, int PAD>
+struct WarpFft2;
+
+template <int N, int R0, int R1, int SIGN, int PAD>
+struct WarpFft2<Radix<N, R0, R1>, SIGN, PAD> {
+    static_assert(R0 <= 32 && R1 <= 32, "warp FFT: radices must fit a warp");
+    using Xc = WarpXchg<R0, R1, PAD>;
+    // src.load(0, n), dst.store(0, n, v); tw2s: stage-2 twiddles [b*(R1-1) + j-1] (shared)
+    template <class Src, class Dst, class Mid>
+    static __device__ __forceinline__ void run(const Src& src, const Xc& xc, Dst& dst,
+                                               const float2* tw2s, int lane, const Mid& mid) {
+        if (lane < R1) {                       // stage 1: radix R0, butterfly b = lane
+            float2 v[R0];
+#pragma unroll
+            for (int j = 0; j < R0; ++j) v[j] = src.load(0, lane + j * R1);
+            Dft<R0, SIGN>::run(v);
+#pragma unroll
+            for (int j = 0; j < R0; ++j) xc.at(j, lane) = v[j];
+        }
+        __syncwarp();
+        mid();                                 // source fully read: prefetch the next line
+        if (lane < R0) {                       // stage 2: radix R1, butterfly b = lane
+            float2 v[R1];
+#pragma unroll
+            for (int j = 0; j < R1; ++j) v[j] = xc.at(lane, j);
+            const float2* tw = tw2s + lane * (R1 - 1);
+#pragma unroll
+            for (int j = 1; j < R1; ++j) v[j] = SIGN < 0 ? cmul(v[j], tw[j - 1]) : cmulc(v[j], tw[j - 1]);
+            Dft<R1, SIGN>::run(v);
+#pragma unroll
+            for (int j = 0; j < R1; ++j) dst.store(0, lane + j * R0, v[j]);
+        }
+    }
+};
+
+constexpr int ROWW_WARPS = 8;   // warps per CTA of the warp-per-line kernels
+
+template <class PL>
+struct RowWarp {
+    using RI = typename PL::RI;
+    static constexpr int PAD = (RI::R0 % 2 == 0) ? 1 : 0;        // odd stride across lanes
+    using Fft = WarpFft2<typename PL::Row, -1, PAD>;
+    using IFft = WarpFft2<typename PL::Row, +1, PAD>;
+    static constexpr int XCH = RI::R1 * (RI::R0 + PAD);          // float2 per warp
+    static constexpr int RAWB = PL::W * 2;                       // raw row bytes (K1)
+    static constexpr int QROW = PL::WP * 8;                      // Q row bytes (K4)
+    static constexpr size_t OFF_TW2 = 64;                        // after 8 mbarriers
+    static constexpr size_t OFF_TWW = OFF_TW2 + (size_t)(PL::ROW_TW2 > 0 ? PL::ROW_TW2 : 1) * 8;
+    static constexpr size_t OFF_WARP = (OFF_TWW + (size_t)(PL::M + 1) * 8 + 127) / 128 * 128;
+    static constexpr size_t WARP_K1 = ((size_t)RAWB + 15) / 16 * 16 + (size_t)XCH * 8;
+    static constexpr size_t WARP_K4 = (size_t)QROW + (size_t)XCH * 8;
+    static constexpr size_t SMEM_K1 = OFF_WARP + ROWW_WARPS * WARP_K1;
+    static constexpr size_t SMEM_K4 = OFF_WARP + ROWW_WARPS * WARP_K4;
+    static constexpr bool OK = RI::STAGES == 2 && RAWB % 16 == 0;
+};
+
+template <class PL>
+__device__ __forceinline__ void rowwarp_tables(float2* tw2s, float2* twWs, const float2* tw2,
+                                               const float2* twW) {
+    for (int i = threadIdx.x; i < PL::ROW_TW2; i += 32 * ROWW_WARPS) tw2s[i] = __ldg(tw2 + i);
+    for (int i = threadIdx.x; i <= PL::M; i += 32 * ROWW_WARPS) twWs[i] = __ldg(twW + i);
+}
+
+// ------------------------------------------------------------------ K1w ----
+template <class PL>
+__global__ void __launch_bounds__(32 * ROWW_WARPS, 2)
+    k1w_fwd_rows(const uint16_t* __restrict__ raw, float2* __restrict__ G, int tile0, int ntiles,
+                 const float2* __restrict__ tw2, const float2* __restrict__ twW) {
+    using RW = RowWarp<PL>;
+    constexpr int M = PL::M, H = PL::H;
+    extern __shared__ __align__(128) unsigned char smem_w[];
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem_w);
+    float2* tw2s = reinterpret_cast<float2*>(smem_w + RW::OFF_TW2);
+    float2* twWs = reinterpret_cast<float2*>(smem_w + RW::OFF_TWW);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned char* mine = smem_w + RW::OFF_WARP + warp * RW::WARP_K1;
+    const uint32_t* land = reinterpret_cast<const uint32_t*>(mine);
+    typename RW::Fft::Xc xc{reinterpret_cast<float2*>(mine + (RW::WARP_K1 - RW::XCH * 8))};
+    uint64_t* bar = &bars[warp];
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+    }
+    rowwarp_tables<PL>(tw2s, twWs, tw2, twW);
+    __syncthreads();                           // the only CTA-wide barrier
+    const long long nrows = (long long)ntiles * H;
+    const long long gw = (long long)blockIdx.x * ROWW_WARPS + warp, nw = (long long)gridDim.x * ROWW_WARPS;
+    const int r0 = (int)(nrows * gw / nw), r1 = (int)(nrows * (gw + 1) / nw);
+    auto issue = [&](int r) {                  // global row r = tile*H + y of this chunk
+        mbar_arrive_expect_tx(bar, RW::RAWB);
+        bulk_g2s(mine, raw + ((size_t)tile0 * H + r) * PL::W, RW::RAWB, bar);
+    };
+    if (lane == 0 && r0 < r1) issue(r0);
+    int k = 0;
+    for (int r = r0; r < r1; ++r, ++k) {
+        mbar_wait(bar, k & 1);
+        struct Src {
+            const uint32_t* p;
+            __device__ __forceinline__ float2 load(int, int n) const {
+                const uint32_t u = p[n];
+                return make_float2((float)(u & 0xFFFFu), (float)(u >> 16));
+            }
+        } src{land};
+        auto prefetch = [&]() {
+            if (lane == 0 && r + 1 < r1) {
+                fence_proxy_async();
+                issue(r + 1);
+            }
+        };
+        RW::Fft::run(src, xc, xc, tw2s, lane, prefetch);   // natural-order Z back in place
+        __syncwarp();
+        float2* out = G + (size_t)r * PL::WP;
+        for (int q = lane; q <= M / 2; q += 32) {
+            const float2 zq = xc.nat(q);
+            const float2 zm = xc.nat(q == 0 ? 0 : M - q);
+            const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
+            const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
+            const float2 wo = cmul(twWs[q], O);
+            out[q] = make_float2(E.x + wo.x, E.y + wo.y);
+            if (2 * q != M) out[M - q] = make_float2(E.x - wo.x, wo.y - E.y);
+        }
+        for (int q = M + 1 + lane; q < PL::WP; q += 32) out[q] = make_float2(0.f, 0.f);
+        __syncwarp();                          // exchange free for the next row
+    }
+}
+
+// ------------------------------------------------------------------ K4w ----
+template <class PL>
+__global__ void __launch_bounds__(32 * ROWW_WARPS, 2)
+    k4w_pair_rows(const float2* __restrict__ Q, unsigned long long* __restrict__ keys, int pair0,
+                  int npairs, const float2* __restrict__ tw2, const float2* __restrict__ twW) {
+    using RW = RowWarp<PL>;
+    constexpr int M = PL::M, H = PL::H;
+    extern __shared__ __align__(128) unsigned char smem_w[];
+    uint64_t* bars = reinterpret_cast<uint64_t*>(smem_w);
+    float2* tw2s = reinterpret_cast<float2*>(smem_w + RW::OFF_TW2);
+    float2* twWs = reinterpret_cast<float2*>(smem_w + RW::OFF_TWW);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned char* mine = smem_w + RW::OFF_WARP + warp * RW::WARP_K4;
+    const float2* land = reinterpret_cast<const float2*>(mine);
+    typename RW::IFft::Xc xc{reinterpret_cast<float2*>(mine + RW::QROW)};
+    uint64_t* bar = &bars[warp];
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+    }
+    rowwarp_tables<PL>(tw2s, twWs, tw2, twW);
+    __syncthreads();                           // the only CTA-wide barrier
+    const long long nrows = (long long)npairs * H;
+    const long long gw = (long long)blockIdx.x * ROWW_WARPS + warp, nw = (long long)gridDim.x * ROWW_WARPS;
+    const int r0 = (int)(nrows * gw / nw), r1 = (int)(nrows * (gw + 1) / nw);
+    auto issue = [&](int r) {
+        mbar_arrive_expect_tx(bar, RW::QROW);
+        bulk_g2s(mine, Q + (size_t)r * PL::WP, RW::QROW, bar);
+    };
+    auto flush = [&](int pair, float bv, uint32_t bi) {
+        unsigned long long key =
+            bv < 0.f ? 0ull : ((unsigned long long)__float_as_uint(bv) << 32) | (0xFFFFFFFFu - bi);
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) key = max(key, __shfl_xor_sync(0xFFFFFFFFu, key, o));
+        if (lane == 0) atomicMax(&keys[pair0 + pair], key);
+    };
+    if (lane == 0 && r0 < r1) issue(r0);
+    ArgmaxDst acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
+    int cur = r0 < r1 ? r0 / H : -1;
+    int k = 0;
+    for (int r = r0; r < r1; ++r, ++k) {
+        const int pl = r / H, y = r - pl * H;
+        if (pl != cur) {                       // warp-uniform
+            flush(cur, acc.best_v, acc.best_i);
+            cur = pl;
+            acc.best_v = -1.f;
+            acc.best_i = 0xFFFFFFFFu;
+        }
+        acc.row_base = y;
+        mbar_wait(bar, k & 1);
+        struct Src {
+            const float2* x;
+            const float2* w;
+            __device__ __forceinline__ float2 load(int, int n) const {
+                const float2 xn = x[n];
+                const float2 xm = x[M - n];
+                const float2 d = make_float2(xn.x - xm.x, xn.y + xm.y);
+                const float2 o = cmulc(d, w[n]);
+                return make_float2(xn.x + xm.x - o.y, xn.y - xm.y + o.x);
+            }
+        } src{land, twWs};
+        auto prefetch = [&]() {
+            if (lane == 0 && r + 1 < r1) {
+                fence_proxy_async();
+                issue(r + 1);
+            }
+        };
+        RW::IFft::run(src, xc, acc, tw2s, lane, prefetch);
+        __syncwarp();                          // exchange free for the next row
+    }
+    if (cur >= 0) flush(cur, acc.best_v, acc.best_i);
+}
+
+}  // namespace stitch
