@@ -67,6 +67,12 @@ struct WarpFft2<Radix<N, R0, R1>, SIGN, PAD> {
 };
 
 constexpr int ROWW_WARPS = 8;   // warps per CTA of the warp-per-line kernels
+#ifndef ROWW_MINB1
+#define ROWW_MINB1 2            // CTAs per SM the registers are budgeted for (K1w)
+#endif
+#ifndef ROWW_MINB4
+#define ROWW_MINB4 2            // (K4w)
+#endif
 
 template <class PL>
 struct RowWarp {
@@ -96,7 +102,7 @@ __device__ __forceinline__ void rowwarp_tables(float2* tw2s, float2* twWs, const
 
 // ------------------------------------------------------------------ K1w ----
 template <class PL>
-__global__ void __launch_bounds__(32 * ROWW_WARPS, 2)
+__global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB1)
     k1w_fwd_rows(const uint16_t* __restrict__ raw, float2* __restrict__ G, int tile0, int ntiles,
                  const float2* __restrict__ tw2, const float2* __restrict__ twW) {
     using RW = RowWarp<PL>;
@@ -159,7 +165,7 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, 2)
 
 // ------------------------------------------------------------------ K4w ----
 template <class PL>
-__global__ void __launch_bounds__(32 * ROWW_WARPS, 2)
+__global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
     k4w_pair_rows(const float2* __restrict__ Q, unsigned long long* __restrict__ keys, int pair0,
                   int npairs, const float2* __restrict__ tw2, const float2* __restrict__ twW) {
     using RW = RowWarp<PL>;
