@@ -8,7 +8,7 @@ Workloads (BASELINE.json ``configs``):
   config 1: 3x3 grid of 256x192 tiles (oracle runs in seconds)
   config 2: 18x22 grid of 1392x1040 tiles
   config 3: 42x59 grid of 1392x1040 tiles (headline)
-  config 4: 161 scans x 2 channels x 18x22 (streamed; not a round-1 bench line)
+  config 4: 161 scans x 2 channels x 18x22 (streamed: bench.py --config 4, stream.py)
   config 5: 100x100 grid of 1392x1040 tiles
 
 Geometry: with step
@@ -37,6 +37,8 @@ CONFIGS = {
     1: dict(name="3x3@256x192", n=3, m=3, H=192, W=256, overlap=0.10, delta=4),
     2: dict(name="18x22@1392x1040", n=18, m=22, H=1040, W=1392, overlap=0.10, delta=12),
     3: dict(name="42x59@1392x1040", n=42, m=59, H=1040, W=1392, overlap=0.10, delta=12),
+    4: dict(name="161x2x(18x22)@1392x1040", n=18, m=22, H=1040, W=1392, overlap=0.10, delta=12,
+            scans=161, channels=2),
     5: dict(name="100x100@1392x1040", n=100, m=100, H=1040, W=1392, overlap=0.10, delta=12),
 }
 

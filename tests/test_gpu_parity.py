@@ -269,3 +269,27 @@ def test_config2_full_size_sampled():
 @pytest.mark.slow
 def test_config3_headline_full_size_sampled():
     sampled_full_size(3, 8)
+
+
+def test_stream_time_series_matches_per_grid():
+    """f1 streaming: grids of a synthetic time series (scans x channels) pushed through two
+    slots give exactly the per-grid results, and one of them matches the oracle."""
+    from paper_conf_icpp_blattnerkcsbz14_b200.stream import GridStream
+    n, m, H, W = 3, 4, 192, 256
+    series = [(s, c) for s in range(3) for c in range(2)]
+    grids = {i: synthgrid.make_grid(n, m, H, W, scan=s, channel=c, seed=41).tiles
+             for i, (s, c) in enumerate(series)}
+    got = {}
+
+    def fill(i, host):
+        host[...] = grids[i]
+
+    with GridStream(n, m, H, W, slots=2) as gs:
+        count = gs.run(range(len(series)), fill, lambda r: got.__setitem__(r.index, r))
+    assert count == len(series) and sorted(got) == list(range(len(series)))
+    for i, tiles in grids.items():
+        w, nn, _ = run_gpu(tiles)
+        assert got[i].west.tobytes() == w.tobytes() and got[i].north.tobytes() == nn.tobytes()
+    ow, on = oracle.grid(grids[3])
+    assert np.array_equal(got[3].west["dx"][:, 1:], ow["dx"][:, 1:])
+    assert np.array_equal(got[3].north["dy"][1:], on["dy"][1:])
