@@ -245,6 +245,8 @@ def main():
     ap.add_argument("--chunk-tiles", type=int, default=0)
     ap.add_argument("--e2e-steps", type=int, default=3)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--compose", action="store_true",
+                    help="also time phase 2 (positions) and phase 3 (overlay composite)")
     ap.add_argument("--ts-grids", type=int, default=24, help="config 4: grids streamed (timed)")
     ap.add_argument("--ts-slots", type=int, default=2, help="config 4: grid slots in flight")
     ap.add_argument("--no-exchange", action="store_true",
@@ -397,6 +399,27 @@ def main():
     h2d = (e - halo) * T
     d2h = pairs_local * 64
 
+    # ---- optional: stitching phases 2 + 3 on the result (NEXT rows f3, f4) -------------
+    phase23 = None
+    if args.compose and world == 1:
+        from paper_conf_icpp_blattnerkcsbz14_b200 import compose_overlay, global_positions
+        t0 = time.perf_counter()
+        pos, _ = global_positions(west, north)
+        t_p2 = time.perf_counter() - t0
+        dev_tiles = torch.empty((n, m, H, W), dtype=torch.uint16, device="cuda")
+        dev_tiles.copy_(host)
+        canvas = compose_overlay(dev_tiles, pos)            # warm (allocates the canvas)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        compose_overlay(dev_tiles, pos, canvas)
+        torch.cuda.synchronize()
+        t_p3 = time.perf_counter() - t0
+        truth = synthgrid.origins(n, m, H, W, cfg["overlap"], cfg["delta"])
+        phase23 = {"phase2_ms": t_p2 * 1e3, "phase3_ms": t_p3 * 1e3,
+                   "canvas": list(canvas.shape), "canvas_GB": canvas.numel() * 2 / 1e9,
+                   "positions_exact": bool(np.array_equal(pos, truth - truth[0, 0]))}
+        del canvas, dev_tiles
+
     # ---- oracle on the host cores (rank 0, N = 1 only) ----------------------------------
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
@@ -425,6 +448,8 @@ def main():
             "gpu_launches": launches,
             "clocks": clocks,
         }
+        if phase23 is not None:
+            line["phase23"] = phase23
         print(json.dumps(line), flush=True)
     bp.close()
     if world > 1:

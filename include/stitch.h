@@ -190,6 +190,33 @@ stitch_status stitch_set_timing(stitch_ctx* ctx, int enabled);
  * Valid after stitch_synchronize / stitch_get_translations. */
 stitch_status stitch_kernel_timings(stitch_ctx* ctx, float* ms6, int64_t* launches6);
 
+/*
+ * Phase 2 (NEXT row f3): absolute tile positions from the phase-1
+ * translations.  The paper names no algorithm (reading C19): the translations
+ * of a MAXIMUM SPANNING TREE of the tile graph weighted by CCF are kept (Kruskal, ties by
+ * pair index) and positions are path sums from the root tile along the tree.
+ *   west, north: [n*m] as filled by stitch_compute_translations (candidate 0 = no edge)
+ *   pos_xy:      out [n*m][2] (x, y) of each tile's origin; the smallest tile of each
+ *                connected component is its origin (0, 0)
+ *   parent:      optional out [n*m] tree parent (-1 for a root); may be NULL
+ * Host-only (no device work).  Errors: INVALID_ARG.
+ */
+stitch_status stitch_global_positions(int32_t n, int32_t m, const stitch_pair* west,
+                                      const stitch_pair* north, int64_t* pos_xy, int32_t* parent);
+
+/*
+ * Phase 3 (NEXT row f4; Fig. 13 overlay L1446): compose the stitched
+ * image on the device by overlay blend -- in an overlap the later tile (row-major) is on
+ * top; every canvas pixel is written exactly once (deterministic, no atomics).
+ *   dev_tiles:  device uint16 [n][m][H][W];  host_pos_xy: [n*m][2] tile origins (canvas px)
+ *   dev_canvas: device uint16 [canvas_h][canvas_w], caller-owned; pixels no tile covers are
+ *               left untouched;  stream: cudaStream_t (NULL = legacy default stream)
+ * Synchronous.  Errors: INVALID_ARG, UNSUPPORTED (n*m > 65535), CUDA.
+ */
+stitch_status stitch_compose_overlay(const uint16_t* dev_tiles, int32_t n, int32_t m, int32_t H,
+                                     int32_t W, const int64_t* host_pos_xy, int64_t canvas_w,
+                                     int64_t canvas_h, uint16_t* dev_canvas, void* stream);
+
 /* Message for the last error on ctx (valid until the next call on ctx). */
 const char* stitch_last_error(stitch_ctx* ctx);
 

@@ -58,7 +58,8 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_debug_spectrum", "stitch_synchronize", "stitch_last_counts",
            "stitch_last_timings", "stitch_set_timing", "stitch_last_error", "stitch_destroy",
            "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings",
-           "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async"]
+           "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async",
+           "stitch_global_positions", "stitch_compose_overlay"]
 
 _lib = None
 
@@ -98,6 +99,8 @@ def load_library():
         "stitch_forward_range_async": (ctypes.c_int, [vp, i32, i32]),
         "stitch_spectra_range": (ctypes.c_int, [vp, i32, i32, P(vp), P(ctypes.c_size_t)]),
         "stitch_pairs_async": (ctypes.c_int, [vp]),
+        "stitch_global_positions": (ctypes.c_int, [i32, i32, vp, vp, vp, vp]),
+        "stitch_compose_overlay": (ctypes.c_int, [vp, i32, i32, i32, i32, vp, i64, i64, vp, vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -127,6 +130,39 @@ def pair_count(cfg: Config) -> int:
     if st:
         raise StitchError(st, "stitch_pair_count")
     return c.value
+
+
+def global_positions(west: np.ndarray, north: np.ndarray):
+    """Phase 2 (f3): absolute tile origins [n, m, 2] (x, y) from the translations, and the
+    maximum-spanning-tree parent of each tile (-1 at a root).  Host-only C code."""
+    n, m = west.shape
+    w = np.ascontiguousarray(west.reshape(-1), dtype=PAIR_DTYPE)
+    nn = np.ascontiguousarray(north.reshape(-1), dtype=PAIR_DTYPE)
+    pos = np.zeros((n * m, 2), np.int64)
+    parent = np.zeros(n * m, np.int32)
+    st = load_library().stitch_global_positions(n, m, w.ctypes.data, nn.ctypes.data,
+                                                pos.ctypes.data, parent.ctypes.data)
+    if st:
+        raise StitchError(st, "stitch_global_positions")
+    return pos.reshape(n, m, 2), parent.reshape(n, m)
+
+
+def compose_overlay(tiles, pos_xy: np.ndarray, canvas=None):
+    """Phase 3 (f4): overlay-blend composite of a device tile grid (torch CUDA uint16
+    [n, m, H, W]) at integer origins pos_xy [n, m, 2]; returns the torch canvas."""
+    import torch
+    n, m, H, W = tiles.shape
+    p = np.ascontiguousarray(pos_xy.reshape(-1, 2), dtype=np.int64)
+    p = p - p.min(axis=0)
+    cw, ch = int(p[:, 0].max()) + W, int(p[:, 1].max()) + H
+    if canvas is None:
+        canvas = torch.zeros((ch, cw), dtype=torch.uint16, device=tiles.device)
+    st = load_library().stitch_compose_overlay(
+        tiles.data_ptr(), n, m, H, W, p.ctypes.data, cw, ch, canvas.data_ptr(),
+        torch.cuda.current_stream(tiles.device).cuda_stream)
+    if st:
+        raise StitchError(st, "stitch_compose_overlay")
+    return canvas
 
 
 class PciamGrid:
