@@ -249,6 +249,8 @@ def main():
                     help="also time phase 2 (positions) and phase 3 (overlay composite)")
     ap.add_argument("--ts-grids", type=int, default=24, help="config 4: grids streamed (timed)")
     ap.add_argument("--ts-slots", type=int, default=2, help="config 4: grid slots in flight")
+    ap.add_argument("--precision", default="f32", choices=["f32", "f64"],
+                    help="arithmetic of steps 2-5 (f64: the optional fp64 path, SURVEY 8 f2)")
     ap.add_argument("--no-exchange", action="store_true",
                     help="N > 1: recompute the halo row's spectra instead of receiving them")
     args = ap.parse_args()
@@ -284,7 +286,8 @@ def main():
     first = r0 * m
 
     bp = BandPciam(n, m, H, W, rank, world, device=local, exchange=not args.no_exchange,
-                   chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles)
+                   chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles,
+                   precision=1 if args.precision == "f64" else 0)
     pg = bp.grid
     stream = pg.stream          # the stream the library enqueues on (events must be recorded here)
     pg.load_tiles(host, first)
@@ -355,6 +358,11 @@ def main():
         "k4_pair_rows": S,             # Q in (the surface is never stored)
         "k5_ccf_moments": 2 * T,       # the four candidate overlaps of A and B (HW pixels each)
         "k6_finalize": 8 + 160 + 64}
+    if args.precision == "f64":
+        # fp64 path (D1..D4, pciam_fp64.cuh): complex intermediates are 2S, the resident
+        # unit phasor is 2S (double2 per bin); D4's per-block argmax partials are ~0
+        alg_bytes_per_unit.update({"k1_fwd_rows": T + 2 * S, "k2_fwd_cols": 4 * S,
+                                   "k3_pair_cols": 6 * S, "k4_pair_rows": 2 * S})
     kd = kt_sum[dom]
     nsteps_k = max(1, min(args.steps, 5))
     fwd_tiles = (e - b) if bp.use_exchange else (e - halo)   # halo received or recomputed
@@ -380,7 +388,7 @@ def main():
     roofline["step_frac"] = roofline["step_alg_GBps"] / pk["hbm_gbs"]
     roofline["survey_2pass_GBps"] = survey_2pass / (dev_ms / 1e3) / 1e9
     traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(traffic_path):
+    if os.path.exists(traffic_path) and args.precision == "f32":   # captured on the fp32 kernels
         with open(traffic_path) as f:
             tr = json.load(f).get(dom)
         if tr:
@@ -433,7 +441,7 @@ def main():
             "scaling": "strong", "vs_baseline": value / PAPER_PAIRS_PER_S,
             "vs_baseline_ref": "paper Pipelined-GPU 1xC2070, 42x59 in 49.7 s (Table II, P:L1208)"
                                " = 97.7 pairs/s; other hardware, end-to-end incl. TIFF reads",
-            "dtype": "f32", "data": "synthetic",
+            "dtype": args.precision, "data": "synthetic",
             "config": {"workload": f"{cfg['name']} (BASELINE.json configs[{args.config - 1}])",
                        "grid": f"{n}x{m}", "tile": f"{W}x{H} uint16", "pairs": int(total_pairs),
                        "tiles": n * m, "grid_wall_ms": ms, "parallelism": f"row-bands x{world}",

@@ -58,7 +58,10 @@ typedef struct {
     int32_t tile_end;     /* one past the last owned tile; 0 => n*m */
     int32_t chunk_pairs;  /* pairs per inverse-transform chunk (L2-resident intermediate); 0 => default */
     int32_t chunk_tiles;  /* tiles per forward-transform chunk; 0 => default */
-    int32_t reserved;
+    int32_t precision;    /* arithmetic of steps 2-5: 0 = fp32 (default), 1 = fp64 (the paper's "double
+                             complex" transforms; north_star's optional fp64 path).
+                             The CCF (steps 6-7) is exact integer moments -> fp64 either way.
+                             Anything else -> STITCH_ERR_INVALID_ARG. */
     void* stream;         /* cudaStream_t to enqueue on (e.g. torch's current stream); NULL => library-created */
     void* workspace;      /* caller-owned device memory of >= stitch_workspace_size bytes (e.g. a torch
                              tensor), 256-byte aligned; NULL => the library allocates with cudaMalloc */
@@ -166,6 +169,16 @@ stitch_status stitch_pairs_async(stitch_ctx* ctx);
  * stitch_forward_async / compute.  Synchronous.
  */
 stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_out);
+
+/*
+ * Test hook of the fp64 path (precision = 1): tile t's complex
+ * half spectrum F(ky, kx) (step 2; "double complex") as
+ * [H][W/2+1][2] doubles, recomputed by the same fp64 forward kernels.  The
+ * context's resident store holds F/|F| (the only part step 3 uses).
+ * Synchronous.  STITCH_ERR_STATE on an fp32 context (and stitch_debug_spectrum
+ * returns STITCH_ERR_STATE on an fp64 one).
+ */
+stitch_status stitch_debug_spectrum_f64(stitch_ctx* ctx, int32_t tile, double* host_out);
 
 /* Wait for all work enqueued on the context stream. */
 stitch_status stitch_synchronize(stitch_ctx* ctx);

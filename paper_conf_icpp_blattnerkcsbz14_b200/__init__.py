@@ -47,7 +47,7 @@ class Config(ctypes.Structure):
                 ("grid_rows", ctypes.c_int32), ("grid_cols", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("tile_begin", ctypes.c_int32),
                 ("tile_end", ctypes.c_int32), ("chunk_pairs", ctypes.c_int32),
-                ("chunk_tiles", ctypes.c_int32), ("reserved", ctypes.c_int32),
+                ("chunk_tiles", ctypes.c_int32), ("precision", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
                 ("workspace_bytes", ctypes.c_size_t)]
 
@@ -59,7 +59,7 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_last_timings", "stitch_set_timing", "stitch_last_error", "stitch_destroy",
            "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings",
            "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async",
-           "stitch_global_positions", "stitch_compose_overlay"]
+           "stitch_global_positions", "stitch_compose_overlay", "stitch_debug_spectrum_f64"]
 
 _lib = None
 
@@ -87,6 +87,7 @@ def load_library():
         "stitch_get_translations": (ctypes.c_int, [vp, vp, vp]),
         "stitch_forward_async": (ctypes.c_int, [vp]),
         "stitch_debug_spectrum": (ctypes.c_int, [vp, i32, vp]),
+        "stitch_debug_spectrum_f64": (ctypes.c_int, [vp, i32, vp]),
         "stitch_synchronize": (ctypes.c_int, [vp]),
         "stitch_last_counts": (ctypes.c_int, [vp, P(i64), P(i64), P(i64)]),
         "stitch_last_timings": (ctypes.c_int, [vp, P(ctypes.c_float)]),
@@ -111,8 +112,9 @@ def load_library():
 
 
 def make_config(n, m, H, W, device=0, tile_begin=0, tile_end=0, chunk_pairs=0, chunk_tiles=0,
-                stream=None, workspace=None, workspace_bytes=0) -> Config:
-    return Config(W, H, n, m, device, tile_begin, tile_end, chunk_pairs, chunk_tiles, 0,
+                stream=None, workspace=None, workspace_bytes=0, precision=0) -> Config:
+    """precision: 0 = fp32 transforms (default), 1 = fp64."""
+    return Config(W, H, n, m, device, tile_begin, tile_end, chunk_pairs, chunk_tiles, precision,
                   stream, workspace, workspace_bytes)
 
 
@@ -171,13 +173,15 @@ class PciamGrid:
 
     def __init__(self, n: int, m: int, H: int, W: int, device: int = 0, tile_begin: int = 0,
                  tile_end: int = 0, chunk_pairs: int = 0, chunk_tiles: int = 0,
-                 use_torch: bool = True):
+                 use_torch: bool = True, precision: int = 0):
         self.lib = load_library()
         self.n, self.m, self.H, self.W = n, m, H, W
         self.device = device
         self._ctx = ctypes.c_void_p(None)
         self._ws = None
-        cfg = make_config(n, m, H, W, device, tile_begin, tile_end, chunk_pairs, chunk_tiles)
+        self.precision = precision
+        cfg = make_config(n, m, H, W, device, tile_begin, tile_end, chunk_pairs, chunk_tiles,
+                          precision=precision)
         self.stream = None
         if use_torch:
             import torch
@@ -296,7 +300,13 @@ class PciamGrid:
         return west.reshape(self.n, self.m), north.reshape(self.n, self.m)
 
     def spectrum(self, tile: int) -> np.ndarray:
-        """Resident half spectrum of a tile, complex64 [H, W//2 + 1] (test hook)."""
+        """Half spectrum of a tile, [H, W//2 + 1], complex64 (fp32 context) or complex128
+        (fp64 context), recomputed by the context's forward kernels (test hook)."""
+        if self.precision:
+            out = np.empty((self.H, self.W // 2 + 1), np.complex128)
+            self._check(self.lib.stitch_debug_spectrum_f64(self._ctx, tile, out.ctypes.data),
+                        "spectrum")
+            return out
         out = np.empty((self.H, self.W // 2 + 1), np.complex64)
         self._check(self.lib.stitch_debug_spectrum(self._ctx, tile, out.ctypes.data), "spectrum")
         return out

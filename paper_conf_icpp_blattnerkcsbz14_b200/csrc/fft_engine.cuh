@@ -29,6 +29,13 @@ __device__ __forceinline__ float2 cmul(float2 a, float2 b) {
 __device__ __forceinline__ float2 cmulc(float2 a, float2 b) {  // a * conj(b)
     return make_float2(fmaf(a.x, b.x, a.y * b.y), fmaf(a.y, b.x, -a.x * b.y));
 }
+// fp64 twins (the f2 path instantiates the engine with C = double2)
+__device__ __forceinline__ double2 cmul(double2 a, double2 b) {
+    return make_double2(fma(a.x, b.x, -a.y * b.y), fma(a.x, b.y, a.y * b.x));
+}
+__device__ __forceinline__ double2 cmulc(double2 a, double2 b) {
+    return make_double2(fma(a.x, b.x, a.y * b.y), fma(a.y, b.x, -a.x * b.y));
+}
 
 // Butterfly id g -> (line, b).  Row map: consecutive threads walk one line.
 struct RowMap {
@@ -48,29 +55,29 @@ struct ColMap {
 };
 
 // Exchange buffer for row lines: line-major, each line an R1 x (R0+PAD) matrix.
-template <int R0, int R1, int PAD>
+template <int R0, int R1, int PAD, class C = float2>
 struct RowXchg {
-    float2* s;
+    C* s;
     static constexpr int LSTRIDE = R1 * (R0 + PAD);
-    __device__ __forceinline__ float2& at(int line, int u, int v) const {
+    __device__ __forceinline__ C& at(int line, int u, int v) const {
         return s[line * LSTRIDE + v * (R0 + PAD) + u];
     }
     // element n of the transform in natural order: the slot stage 2 read it from
     // (u = n mod R0, v = n / R0), so stage 2 may write its outputs back in place
-    __device__ __forceinline__ float2& nat(int line, int n) const {
+    __device__ __forceinline__ C& nat(int line, int n) const {
         if constexpr (PAD == 0)
             return s[line * LSTRIDE + n];       // v * R0 + u == n
         else
             return at(line, n % R0, n / R0);
     }
-    __device__ __forceinline__ void store(int line, int n, float2 v) const { nat(line, n) = v; }
+    __device__ __forceinline__ void store(int line, int n, C v) const { nat(line, n) = v; }
 };
 // Exchange buffer for a panel of P columns: element (u, v) of column c at
 // (v*(R0+PAD) + u)*P + c, so a warp's 8-byte accesses span all 32 banks.
-template <int R0, int R1, int PAD, int P>
+template <int R0, int R1, int PAD, int P, class C = float2>
 struct ColXchg {
-    float2* s;
-    __device__ __forceinline__ float2& at(int line, int u, int v) const {
+    C* s;
+    __device__ __forceinline__ C& at(int line, int u, int v) const {
         return s[(v * (R0 + PAD) + u) * P + line];
     }
 };
@@ -91,18 +98,19 @@ struct Radix {
     static constexpr int count = sizeof...(Rs);
 };
 
-template <class RX, int SIGN, int L, int T, class Map, bool TW_SMEM = false>
+// C: the complex element type (float2, or double2 for the fp64 path f2)
+template <class RX, int SIGN, int L, int T, class Map, bool TW_SMEM = false, class C = float2>
 struct FftRun;
 
 // One stage: N = R0, no twiddles, source -> destination.
-template <int N, int R0, int SIGN, int L, int T, class Map, bool TW_SMEM>
-struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM> {
+template <int N, int R0, int SIGN, int L, int T, class Map, bool TW_SMEM, class C>
+struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM, C> {
     static_assert(N == R0, "single-stage plan");
     static constexpr int R1 = 1;
     template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid,
               class AfterLoads = NoMid>
     static __device__ __forceinline__ void run(const Src& src, const Xc&, Dst& dst,
-                                               const float2* __restrict__, const Mid& mid = Mid(),
+                                               const C* __restrict__, const Mid& mid = Mid(),
                                                const AfterLoads& after_loads = AfterLoads()) {
         // one butterfly per line (the source is consumed inside the loop; `mid` runs after it)
         constexpr int TOTAL = L;
@@ -112,7 +120,7 @@ struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM> {
             const int g = threadIdx.x + it * T;
             if (TOTAL % T == 0 || g < TOTAL) {
                 const int line = g;
-                float2 v[R0];
+                C v[R0];
 #pragma unroll
                 for (int j = 0; j < R0; ++j) v[j] = src.load(line, j);
                 Dft<R0, SIGN>::run(v);
@@ -127,8 +135,8 @@ struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM> {
 };
 
 // Two stages: N = R0 * R1, one exchange through shared memory.
-template <int N, int R0_, int R1_, int SIGN, int L, int T, class Map, bool TW_SMEM>
-struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
+template <int N, int R0_, int R1_, int SIGN, int L, int T, class Map, bool TW_SMEM, class C>
+struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
     static constexpr int R0 = R0_, R1 = R1_;
     static_assert(N == R0 * R1, "radices must multiply to N");
     // Stage 1: radix R0 over R1 butterflies per line, source -> exchange.  IN_PLACE: the
@@ -140,7 +148,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
         constexpr int TOTAL = L * R1;
         constexpr int ITER = (TOTAL + T - 1) / T;
         if constexpr (IN_PLACE) {
-            float2 v[ITER][R0];
+            C v[ITER][R0];
 #pragma unroll
             for (int it = 0; it < ITER; ++it) {
                 const int g = threadIdx.x + it * T;
@@ -171,7 +179,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
                 if (TOTAL % T == 0 || g < TOTAL) {
                     int line, b;
                     Map::template map<R1, L>(g, line, b);
-                    float2 v[R0];
+                    C v[R0];
 #pragma unroll
                     for (int j = 0; j < R0; ++j) v[j] = src.load(line, b + j * R1);
                     Dft<R0, SIGN>::run(v);
@@ -187,7 +195,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
     template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid,
               class AfterLoads = NoMid>
     static __device__ __forceinline__ void run(const Src& src, const Xc& xc, Dst& dst,
-                                               const float2* __restrict__ tw2,
+                                               const C* __restrict__ tw2,
                                                const Mid& mid = Mid(),
                                                const AfterLoads& after_loads = AfterLoads()) {
         stage1<IN_PLACE>(src, xc, after_loads);
@@ -204,13 +212,13 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM> {
                 if (TOTAL % T == 0 || g < TOTAL) {
                     int line, b;
                     Map::template map<R0, L>(g, line, b);
-                    float2 v[R1];
+                    C v[R1];
 #pragma unroll
                     for (int j = 0; j < R1; ++j) v[j] = xc.at(line, b, j);
-                    const float2* tw = tw2 + b * (R1 - 1);
+                    const C* tw = tw2 + b * (R1 - 1);
 #pragma unroll
                     for (int j = 1; j < R1; ++j) {
-                        const float2 w = TW_SMEM ? tw[j - 1] : __ldg(tw + (j - 1));
+                        const C w = TW_SMEM ? tw[j - 1] : __ldg(tw + (j - 1));
                         v[j] = SIGN < 0 ? cmul(v[j], w) : cmulc(v[j], w);
                     }
                     Dft<R1, SIGN>::run(v);

@@ -1,17 +1,19 @@
 #!/usr/bin/env python3
-"""Generate straight-line fp32 DFT codelets (codelets.cuh) for the CUDA FFT engine.
+"""Generate straight-line fp32 and fp64 DFT codelets (codelets.cuh) for the CUDA FFT engine.
 
 Each codelet computes, in registers, an unnormalised length-R DFT
     X[k] = sum_j x[j] exp(SIGN * 2 pi i j k / R),   SIGN = -1 (forward) or +1 (inverse)
 in place on a float2[R] array.  Primes use the symmetric (x_j +- x_{R-j}) form,
 composites a Cooley-Tukey split R = R1*R2 with constant twiddles (trivial ones --
 multiples of pi/4 -- special-cased).  Constants are computed in double here and
-rounded once to float literals.
+rounded once to float literals (fp32) or kept as double literals (fp64 path, f2: the same
+straight-line program with every float replaced by double).
 
 This is part of the CUDA product path only (it shares nothing with oracle/).
 Run:  python gen_codelets.py > codelets.cuh
 """
 import math
+import re
 import sys
 
 RADICES = [2, 3, 4, 5, 6, 8, 10, 12, 13, 16, 20, 24, 26, 29, 40]
@@ -250,17 +252,34 @@ def codelet(n, sign):
     return "\n".join(lines)
 
 
+_FLIT = re.compile(r"\(([-+0-9.e]+)f\)")
+
+
+def to_double(src: str) -> str:
+    """The fp64 twin of an fp32 codelet: double temporaries, fma, full-precision literals
+    (flit printed the double constant before appending 'f')."""
+    src = src.replace("const float ", "const double ").replace("fmaf(", "fma(")
+    src = src.replace("float2*", "double2*").replace("make_float2(", "make_double2(")
+    src = re.sub(r"void dft(\d+)([mp])\(", r"void dft\1\2_d(", src)
+    src = _FLIT.sub(r"(\1)", src)
+    return src.replace("0.0f", "0.0")
+
+
 def main():
     out = ["// GENERATED by gen_codelets.py -- do not edit.",
-           "// Straight-line fp32 DFT codelets: v[k] <- sum_j v[j] exp(SIGN 2 pi i j k / R).",
+           "// Straight-line fp32 / fp64 DFT codelets: v[k] <- sum_j v[j] exp(SIGN 2 pi i j k / R).",
            "#pragma once", "", "namespace stitch {", "",
            "template <int R, int SIGN> struct Dft;", ""]
     for r in RADICES:
         for sign in (-1, 1):
-            out.append(codelet(r, sign))
+            c = codelet(r, sign)
+            out.append(c)
+            out.append(to_double(c))
             tag = "m" if sign < 0 else "p"
-            out.append(f"template <> struct Dft<{r}, {sign}> {{ static __device__ __forceinline__ "
-                       f"void run(float2* v) {{ dft{r}{tag}(v); }} }};")
+            out.append(f"template <> struct Dft<{r}, {sign}> {{\n"
+                       f"    static __device__ __forceinline__ void run(float2* v) {{ dft{r}{tag}(v); }}\n"
+                       f"    static __device__ __forceinline__ void run(double2* v) {{ dft{r}{tag}_d(v); }}\n"
+                       f"}};")
             out.append("")
     out.append("}  // namespace stitch")
     sys.stdout.write("\n".join(out) + "\n")

@@ -1,0 +1,274 @@
+// pciam_fp64.cuh — the fp64 path: PCIAM steps 2-5 in double precision.
+//
+// The paper computes its transforms in "double complex" and the CCF in double
+// (Fig. 3); north_star makes fp64 the optional tighter-tolerance path (CCF within
+// 1e-9 of the oracle).  Same method, same FFT engine (fft_engine.cuh instantiated with
+// C = double2 and the fp64 twins of the generated codelets), same pair list, CCF (K5) and
+// selection (K6) as the fp32 path; what differs:
+//   * the resident spectrum is the unit phasor U = F/|F| (0 where F = 0) as double2 -- step 3
+//     F_A conj(F_B) / |F_A conj(F_B)| = U_A conj(U_B) exactly in real arithmetic (reading C4),
+//     and a 64-bit phase code would need a double-precision sincos per bin;
+//   * the argmax (step 5) compares doubles: per row block a (max |c|, smallest index) partial,
+//     then one warp per pair reduces the partials into the same 64-bit key K5/K6 consume
+//     (the key's value field carries |c| rounded to float, used only for the reported peak).
+// Kernels (plain CTA-per-block launches, coalesced global loads; no TMA: the fp64 path is
+// FP64-issue-bound on B200 long before it is HBM-bound):
+//   D1 fwd_rows   raw -> Gd   R2C along x (uint16 -> double fused into the load)
+//   D2 fwd_cols   Gd -> U     C2C along y, epilogue: unit phasor (or the complex spectrum
+//                             back into Gd for the parity hook)
+//   D3 pair_cols  U -> Qd     step 3 (U_A conj U_B) fused into the inverse C2C along y
+//   D4 pair_rows  Qd -> part  C2R along x, |.| + per-block argmax (surface never stored)
+//   D5 argmax     part -> key per-pair reduction of the block partials
+#pragma once
+#include "pciam_kernels.cuh"
+
+namespace stitch {
+
+template <class PL>
+struct Plan64 {
+    static constexpr int W = PL::W, H = PL::H, M = PL::M, WP = PL::WP;
+    using Row = typename PL::Row;
+    using Col = typename PL::Col;
+    using RI = typename PL::RI;
+    using CI = typename PL::CI;
+    static constexpr int ROW_L = PL::ROW_L, ROW_T = PL::ROW_T;
+    using RowX = RowXchg<RI::R0, RI::R1, PL::ROW_PAD, double2>;
+    static constexpr size_t ROW_SMEM = sizeof(double2) * ROW_L * RowX::LSTRIDE;
+    static constexpr int NBLK = H / ROW_L;    // row blocks (argmax partials) per pair
+    // column panels: 4 columns of double2 = 64-byte row segments
+    static constexpr int COL_P = 4;
+    static constexpr int COL_WORK = CI::STAGES == 1 ? COL_P
+                                                    : (COL_P * CI::R1 > COL_P * CI::R0
+                                                           ? COL_P * CI::R1
+                                                           : COL_P * CI::R0);
+    static constexpr int COL_T = (COL_WORK + 31) / 32 * 32;
+    using ColX = ColXchg<CI::R0, CI::R1, PL::COL_PAD, COL_P, double2>;
+    static constexpr size_t COL_SMEM =
+        CI::STAGES == 1 ? 16 : sizeof(double2) * COL_P * CI::R1 * (CI::R0 + PL::COL_PAD);
+    static_assert(WP % COL_P == 0, "fp64 column panel must divide the pitch");
+    static_assert(ROW_SMEM <= 200 * 1024 && COL_SMEM <= 200 * 1024, "fp64 shared memory");
+};
+
+// ------------------------------------------------------------------ D1 ----
+template <class PL>
+struct U16RowSrcD {  // z[n] = x[2n] + i x[2n+1] (exact in double)
+    const uint32_t* p;
+    __device__ __forceinline__ double2 load(int line, int n) const {
+        const uint32_t u = __ldg(p + line * (PL::W / 2) + n);
+        return make_double2((double)(u & 0xFFFFu), (double)(u >> 16));
+    }
+};
+
+// R2C post-processing of one line in double (the fp32 r2c_post_line, pciam_kernels.cuh):
+//   E = (Z[q] + conj Z[M-q]) / 2,  O = (Z[q] - conj Z[M-q]) / (2i)
+//   X[q] = E + w_W^q O,   X[M-q] = conj(E - w_W^q O)
+template <class PL, class Xc>
+__device__ __forceinline__ void r2c_post_line_d(const Xc& xc, int line, double2* __restrict__ out,
+                                                const double2* __restrict__ twW) {
+    constexpr int M = PL::M;
+    for (int q = threadIdx.x; q <= M / 2; q += PL::ROW_T) {
+        const double2 zq = xc.nat(line, q);
+        const double2 zm = xc.nat(line, q == 0 ? 0 : M - q);
+        const double2 E = make_double2(0.5 * (zq.x + zm.x), 0.5 * (zq.y - zm.y));
+        const double2 O = make_double2(0.5 * (zq.y + zm.y), -0.5 * (zq.x - zm.x));
+        const double2 wo = cmul(__ldg(&twW[q]), O);
+        out[q] = make_double2(E.x + wo.x, E.y + wo.y);
+        if (2 * q != M) out[M - q] = make_double2(E.x - wo.x, wo.y - E.y);
+    }
+    for (int q = M + 1 + threadIdx.x; q < PL::WP; q += PL::ROW_T) out[q] = make_double2(0.0, 0.0);
+}
+
+template <class PL>
+__global__ void __launch_bounds__(PL::ROW_T) d1_fwd_rows(const uint16_t* __restrict__ raw,
+                                                         double2* __restrict__ G, int tile0,
+                                                         const double2* __restrict__ tw2,
+                                                         const double2* __restrict__ twW) {
+    using P64 = Plan64<PL>;
+    extern __shared__ __align__(16) unsigned char smem64[];
+    constexpr int L = P64::ROW_L, T = P64::ROW_T;
+    const size_t t = (size_t)tile0 + blockIdx.y;
+    const int y0 = blockIdx.x * L;
+    U16RowSrcD<PL> src{reinterpret_cast<const uint32_t*>(raw + (t * PL::H + y0) * PL::W)};
+    typename P64::RowX xc{reinterpret_cast<double2*>(smem64)};
+    FftRun<typename P64::Row, -1, L, T, RowMap, false, double2>::run(src, xc, xc, tw2);
+    __syncthreads();
+#pragma unroll 1
+    for (int line = 0; line < L; ++line)
+        r2c_post_line_d<PL>(xc, line, G + ((size_t)blockIdx.y * PL::H + y0 + line) * PL::WP, twW);
+}
+
+// ------------------------------------------------------------------ D2 ----
+template <class PL>
+struct PanelIOD {  // a panel of columns of one [H][WP] double2 array
+    double2* p;
+    __device__ __forceinline__ double2 load(int line, int n) const {
+        return p[(size_t)n * PL::WP + line];
+    }
+    __device__ __forceinline__ void store(int line, int n, double2 v) const {
+        p[(size_t)n * PL::WP + line] = v;
+    }
+};
+
+template <class PL>
+struct UnitDst {  // resident spectrum: U = F/|F|, 0 where F = 0 (reading C4)
+    double2* p;
+    __device__ __forceinline__ void store(int line, int n, double2 v) const {
+        const double m2 = fma(v.x, v.x, v.y * v.y);
+        const double r = m2 > 0.0 ? rsqrt(m2) : 0.0;
+        p[(size_t)n * PL::WP + line] = make_double2(v.x * r, v.y * r);
+    }
+};
+
+// Every stage-1 read of the panel precedes the barrier before stage 2 (or, single-stage,
+// each butterfly owns its whole column), so the complex output may overwrite Gd in place.
+template <class PL, bool UNIT_OUT>
+__global__ void __launch_bounds__(Plan64<PL>::COL_T) d2_fwd_cols(double2* __restrict__ G,
+                                                                 double2* __restrict__ U,
+                                                                 int tile0,
+                                                                 const double2* __restrict__ tw2) {
+    using P64 = Plan64<PL>;
+    extern __shared__ __align__(16) unsigned char smem64[];
+    const int tl = blockIdx.y, c0 = blockIdx.x * P64::COL_P;
+    PanelIOD<PL> src{G + (size_t)tl * PL::H * PL::WP + c0};
+    typename P64::ColX xc{reinterpret_cast<double2*>(smem64)};
+    using Run = FftRun<typename P64::Col, -1, P64::COL_P, P64::COL_T, ColMap, false, double2>;
+    if constexpr (UNIT_OUT) {
+        UnitDst<PL> dst{U + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
+        Run::run(src, xc, dst, tw2);
+    } else {
+        Run::run(src, xc, src, tw2);
+    }
+}
+
+// ------------------------------------------------------------------ D3 ----
+template <class PL>
+struct NcpsUnitSrc {  // step 3: U_A conj(U_B) = F_A conj(F_B) / |F_A conj(F_B)| (0 if either is 0)
+    const double2* a;
+    const double2* b;
+    __device__ __forceinline__ double2 load(int line, int n) const {
+        const size_t o = (size_t)n * PL::WP + line;
+        return cmulc(__ldg(a + o), __ldg(b + o));
+    }
+};
+
+template <class PL>
+__global__ void __launch_bounds__(Plan64<PL>::COL_T) d3_pair_cols(const double2* __restrict__ U,
+                                                                  double2* __restrict__ Q,
+                                                                  const PairIdx* __restrict__ pairs,
+                                                                  int pair0,
+                                                                  const double2* __restrict__ tw2) {
+    using P64 = Plan64<PL>;
+    extern __shared__ __align__(16) unsigned char smem64[];
+    const PairIdx pr = pairs[pair0 + blockIdx.y];
+    const int c0 = blockIdx.x * P64::COL_P;
+    NcpsUnitSrc<PL> src{U + (size_t)pr.a * PL::H * PL::WP + c0,
+                        U + (size_t)pr.b * PL::H * PL::WP + c0};
+    PanelIOD<PL> dst{Q + (size_t)blockIdx.y * PL::H * PL::WP + c0};
+    typename P64::ColX xc{reinterpret_cast<double2*>(smem64)};
+    FftRun<typename P64::Col, +1, P64::COL_P, P64::COL_T, ColMap, false, double2>::run(src, xc, dst,
+                                                                                      tw2);
+}
+
+// ------------------------------------------------------------------ D4 ----
+template <class PL>
+struct C2RSrcD {  // complex-to-real pre-processing of row X[0..M] into Z[0..M) (as C2RSrc)
+    const double2* rows;
+    const double2* twW;
+    __device__ __forceinline__ double2 load(int line, int n) const {
+        const double2* r = rows + (size_t)line * PL::WP;
+        const double2 xn = r[n];
+        const double2 xm = r[PL::M - n];
+        const double2 w = __ldg(&twW[n]);
+        const double2 d = make_double2(xn.x - xm.x, xn.y + xm.y);
+        const double2 o = cmulc(d, w);
+        return make_double2(xn.x + xm.x - o.y, xn.y - xm.y + o.x);
+    }
+};
+
+struct ArgmaxDstD {  // step 5 in double: running (max |x|, smallest index at that max)
+    double best_v;     // -1 before the first value
+    uint32_t best_i;
+    int row_base, W;
+    __device__ __forceinline__ void take(double a, uint32_t idx) {
+        if (a > best_v || (a == best_v && idx < best_i)) {
+            best_v = a;
+            best_i = idx;
+        }
+    }
+    __device__ __forceinline__ void store(int line, int n, double2 v) {
+        const uint32_t idx = (uint32_t)((row_base + line) * W + 2 * n);
+        take(fabs(v.x), idx);
+        take(fabs(v.y), idx + 1);
+    }
+};
+
+// (v, i) beats (v2, i2): larger value, then the smaller row-major index (reading C6)
+__device__ __forceinline__ void argmax_merge(double& v, uint32_t& i, double v2, uint32_t i2) {
+    if (v2 > v || (v2 == v && i2 < i)) {
+        v = v2;
+        i = i2;
+    }
+}
+
+__device__ __forceinline__ void warp_argmax(double& v, uint32_t& i) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        const double v2 = __shfl_xor_sync(0xFFFFFFFFu, v, o);
+        const uint32_t i2 = __shfl_xor_sync(0xFFFFFFFFu, i, o);
+        argmax_merge(v, i, v2, i2);
+    }
+}
+
+template <class PL>
+__global__ void __launch_bounds__(PL::ROW_T) d4_pair_rows(const double2* __restrict__ Q,
+                                                          double* __restrict__ part_v,
+                                                          uint32_t* __restrict__ part_i,
+                                                          int pair0,
+                                                          const double2* __restrict__ tw2,
+                                                          const double2* __restrict__ twW) {
+    using P64 = Plan64<PL>;
+    extern __shared__ __align__(16) unsigned char smem64[];
+    __shared__ double rv[(PL::ROW_T + 31) / 32];
+    __shared__ uint32_t ri[(PL::ROW_T + 31) / 32];
+    constexpr int L = P64::ROW_L, T = P64::ROW_T;
+    const int y0 = blockIdx.x * L;
+    C2RSrcD<PL> src{Q + ((size_t)blockIdx.y * PL::H + y0) * PL::WP, twW};
+    ArgmaxDstD dst{-1.0, 0xFFFFFFFFu, y0, PL::W};
+    typename P64::RowX xc{reinterpret_cast<double2*>(smem64)};
+    FftRun<typename P64::Row, +1, L, T, RowMap, false, double2>::run(src, xc, dst, tw2);
+    double v = dst.best_v;
+    uint32_t i = dst.best_i;
+    warp_argmax(v, i);
+    const int w = threadIdx.x >> 5;
+    if ((threadIdx.x & 31) == 0) {
+        rv[w] = v;
+        ri[w] = i;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int k = 1; k < (T + 31) / 32; ++k) argmax_merge(v, i, rv[k], ri[k]);
+        const size_t o = (size_t)(pair0 + blockIdx.y) * P64::NBLK + blockIdx.x;
+        part_v[o] = v;
+        part_i[o] = i;
+    }
+}
+
+// ------------------------------------------------------------------ D5 ----
+// One warp per pair: reduce the NBLK block partials and emit the K5/K6 key
+// (bits(float(max)) << 32 | (2^32 - 1 - index)); the index is the exact double argmax.
+__global__ void d5_argmax_keys(const double* __restrict__ part_v, const uint32_t* __restrict__ part_i,
+                               unsigned long long* __restrict__ keys, int nblk, int npairs) {
+    const int p = blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5);
+    const int lane = threadIdx.x & 31;
+    if (p >= npairs) return;   // warp-uniform
+    double v = -1.0;
+    uint32_t i = 0xFFFFFFFFu;
+    for (int k = lane; k < nblk; k += 32)
+        argmax_merge(v, i, part_v[(size_t)p * nblk + k], part_i[(size_t)p * nblk + k]);
+    warp_argmax(v, i);
+    if (lane == 0)
+        keys[p] = v < 0.0 ? 0ull
+                          : ((unsigned long long)__float_as_uint((float)v) << 32) | (0xFFFFFFFFu - i);
+}
+
+}  // namespace stitch

@@ -20,6 +20,7 @@
 
 #include "../../include/stitch.h"
 #include "pciam_kernels.cuh"
+#include "pciam_fp64.cuh"
 
 using namespace stitch;
 
@@ -53,6 +54,14 @@ struct PlanOps {
     void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, cudaStream_t);
     void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
+               cudaStream_t);
+    // fp64 path (f2, pciam_fp64.cuh)
+    int nblk64, colp64;
+    cudaError_t (*d_setup)();
+    void (*d1)(const uint16_t*, double2*, int, int, const double2*, const double2*, cudaStream_t);
+    void (*d2)(double2*, double2*, int, int, const double2*, bool, cudaStream_t);
+    void (*d3)(const double2*, double2*, const PairIdx*, int, int, const double2*, cudaStream_t);
+    void (*d4)(const double2*, double*, uint32_t*, int, int, const double2*, const double2*,
                cudaStream_t);
 };
 
@@ -201,13 +210,57 @@ void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long lo
         raw, pairs, keys, mom, p0);
 }
 
+// ---- fp64 path launchers (f2)
+template <class PL>
+cudaError_t d_setup() {
+    using P64 = Plan64<PL>;
+    cudaError_t e;
+    if ((e = max_smem(d1_fwd_rows<PL>, P64::ROW_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(d4_pair_rows<PL>, P64::ROW_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(d2_fwd_cols<PL, true>, P64::COL_SMEM)) != cudaSuccess) return e;
+    if ((e = max_smem(d2_fwd_cols<PL, false>, P64::COL_SMEM)) != cudaSuccess) return e;
+    return max_smem(d3_pair_cols<PL>, P64::COL_SMEM);
+}
+template <class PL>
+void launch_d1(const uint16_t* raw, double2* G, int t0, int nt, const double2* tw2,
+               const double2* twW, cudaStream_t s) {
+    using P64 = Plan64<PL>;
+    d1_fwd_rows<PL><<<dim3(P64::NBLK, nt), P64::ROW_T, P64::ROW_SMEM, s>>>(raw, G, t0, tw2, twW);
+}
+template <class PL>
+void launch_d2(double2* G, double2* U, int t0, int nt, const double2* tw2, bool unit_out,
+               cudaStream_t s) {
+    using P64 = Plan64<PL>;
+    const dim3 grid(PL::WP / P64::COL_P, nt);
+    if (unit_out)
+        d2_fwd_cols<PL, true><<<grid, P64::COL_T, P64::COL_SMEM, s>>>(G, U, t0, tw2);
+    else
+        d2_fwd_cols<PL, false><<<grid, P64::COL_T, P64::COL_SMEM, s>>>(G, U, t0, tw2);
+}
+template <class PL>
+void launch_d3(const double2* U, double2* Q, const PairIdx* pairs, int p0, int np,
+               const double2* tw2, cudaStream_t s) {
+    using P64 = Plan64<PL>;
+    d3_pair_cols<PL><<<dim3(PL::WP / P64::COL_P, np), P64::COL_T, P64::COL_SMEM, s>>>(U, Q, pairs,
+                                                                                      p0, tw2);
+}
+template <class PL>
+void launch_d4(const double2* Q, double* pv, uint32_t* pi, int p0, int np, const double2* tw2,
+               const double2* twW, cudaStream_t s) {
+    using P64 = Plan64<PL>;
+    d4_pair_rows<PL><<<dim3(P64::NBLK, np), P64::ROW_T, P64::ROW_SMEM, s>>>(Q, pv, pi, p0, tw2,
+                                                                            twW);
+}
+
 template <class PL>
 PlanOps make_ops() {
     return PlanOps{PL::W,       PL::H,         PL::M,          PL::WC,        PL::WP,
                    PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
                    PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
                    launch_k2p<PL>, launch_k3p<PL>, launch_k1w<PL>, launch_k4w<PL>, launch_k1<PL>,
-                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>};
+                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>, Plan64<PL>::NBLK,
+                   Plan64<PL>::COL_P, d_setup<PL>, launch_d1<PL>, launch_d2<PL>, launch_d3<PL>,
+                   launch_d4<PL>};
 }
 
 const PlanOps* find_plan(int W, int H) {
@@ -229,7 +282,9 @@ struct Layout {
     int h_begin, t_begin, t_end, nlocal;
     int64_t npairs;
     int chunk_pairs, chunk_tiles;
-    size_t off_raw, off_spec, off_g, off_q, off_pairs, off_keys, off_mom, off_res, off_tw, total;
+    int prec;   // 0 fp32, 1 fp64 (f2)
+    size_t off_raw, off_spec, off_g, off_q, off_pairs, off_keys, off_mom, off_res, off_tw,
+        off_part, total;
 };
 
 stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L) {
@@ -243,20 +298,28 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     int64_t np = 0;
     for (int t = L->t_begin; t < L->t_end; ++t) np += (t % m >= 1) + (t / m >= 1);
     L->npairs = np;
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 64;
-    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : 32;
+    if (c->precision != 0 && c->precision != 1) return STITCH_ERR_INVALID_ARG;
+    L->prec = c->precision;
+    // fp64 chunks of 8 keep the 94 MB intermediate (8 x H x WP x 16 B at 1392x1040) in L2
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : (L->prec ? 8 : 64);
+    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : (L->prec ? 8 : 32);
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
+    // resident spectrum: u32 phase code (fp32) or double2 unit phasor (fp64)
+    const size_t spec_el = L->prec ? sizeof(double2) : sizeof(uint32_t);
+    const size_t cplx = L->prec ? sizeof(double2) : sizeof(float2);
     size_t o = 0;
     L->off_raw = o;   o += align256((size_t)L->nlocal * H * W * sizeof(uint16_t));
-    L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * sizeof(uint32_t));
-    L->off_g = o;     o += align256((size_t)L->chunk_tiles * H * WP * sizeof(float2));
-    L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * sizeof(float2));
+    L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * spec_el);
+    L->off_g = o;     o += align256((size_t)L->chunk_tiles * H * WP * cplx);
+    L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * cplx);
     L->off_pairs = o; o += align256((size_t)(np > 0 ? np : 1) * sizeof(PairIdx));
     L->off_keys = o;  o += align256((size_t)(np > 0 ? np : 1) * sizeof(unsigned long long));
     L->off_mom = o;   o += align256((size_t)(np > 0 ? np : 1) * 20 * sizeof(unsigned long long));
     L->off_res = o;   o += align256((size_t)(np > 0 ? np : 1) * sizeof(stitch_pair));
-    L->off_tw = o;    o += align256((size_t)(tw_count(ops)) * sizeof(float2));
+    L->off_tw = o;    o += align256((size_t)(tw_count(ops)) * cplx);
+    L->off_part = o;  // fp64 argmax partials: double [pairs][nblk] then u32 [pairs][nblk]
+    if (L->prec) o += align256((size_t)(np > 0 ? np : 1) * ops->nblk64 * (8 + 4));
     L->total = o;
     return STITCH_OK;
 }
@@ -286,6 +349,11 @@ struct stitch_ctx {
     uint16_t* raw;
     uint32_t* spec;                   // resident phase spectra [nlocal][H][WP]
     float2 *G, *Q, *twM, *twH, *twW;  // chunk intermediates, twiddles
+    int prec = 0;                     // 1: fp64 path (f2): the buffers below are used instead
+    double2 *Gd = nullptr, *Qd = nullptr, *Ud = nullptr;   // Ud: resident unit phasors
+    double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
+    double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
+    uint32_t* part_i = nullptr;
     CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (phase codes)
     PairIdx* pairs;
     unsigned long long *keys, *mom;
@@ -445,6 +513,8 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     if ((e = ops->setup(&ctx->grid_k1p, &ctx->grid_k4p, &ctx->grid_k1w, &ctx->grid_k4w)) !=
         cudaSuccess)
         return bail(STITCH_ERR_CUDA);
+    ctx->prec = L.prec;
+    if (ctx->prec && (e = ops->d_setup()) != cudaSuccess) return bail(STITCH_ERR_CUDA);
     {
         const char* wenv = std::getenv("STITCH_ROWWARP");   // STITCH_ROWWARP=0: CTA row kernels
         if (wenv && wenv[0] == '0') ctx->grid_k1w = ctx->grid_k4w = 0;
@@ -460,7 +530,7 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         const char* genv = std::getenv("STITCH_GRAPH");   // STITCH_GRAPH=0: direct launches
         ctx->use_graph = !(genv && genv[0] == '0');
         const char* cenv = std::getenv("STITCH_CONCURRENT");  // STITCH_CONCURRENT=0: one stream
-        ctx->concurrent = !(cenv && cenv[0] == '0');
+        ctx->concurrent = !(cenv && cenv[0] == '0') && !ctx->prec;
         if (ctx->concurrent) {
             for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf})
                 if (cudaStreamCreateWithFlags(st, cudaStreamNonBlocking) != cudaSuccess)
@@ -513,9 +583,21 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     ctx->twM = (float2*)(b + L.off_tw);
     ctx->twH = ctx->twM + tw_row(ops);
     ctx->twW = ctx->twH + tw_col(ops);
+    if (ctx->prec) {
+        ctx->Ud = (double2*)(b + L.off_spec);
+        ctx->Gd = (double2*)(b + L.off_g);
+        ctx->Qd = (double2*)(b + L.off_q);
+        ctx->twMd = (double2*)(b + L.off_tw);
+        ctx->twHd = ctx->twMd + tw_row(ops);
+        ctx->twWd = ctx->twHd + tw_col(ops);
+        const size_t np1 = (size_t)(L.npairs > 0 ? L.npairs : 1) * ops->nblk64;
+        ctx->part_v = (double*)(b + L.off_part);
+        ctx->part_i = (uint32_t*)(b + L.off_part + np1 * sizeof(double));
+    }
 
-    // TMA descriptors (driver entry point through the runtime; no libcuda link needed)
-    {
+    // TMA descriptors (driver entry point through the runtime; no libcuda link needed);
+    // the fp64 path uses plain loads
+    if (!ctx->prec) {
         void* fn = nullptr;
         cudaDriverEntryPointQueryResult q;
         if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) !=
@@ -600,8 +682,27 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
             mx = std::max(mx, std::max(pl[(size_t)p].a, pl[(size_t)p].b));
         ctx->pair_need.push_back(mx / L.chunk_tiles);
     }
-    if ((e = cudaMemcpyAsync(ctx->twM, tw.data(), tw.size() * sizeof(float2),
-                             cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
+    // fp64 twiddles: the same tables, rounded once to double
+    std::vector<double2> twd;
+    if (ctx->prec) {
+        twd.resize(tw_count(ops));
+        auto wd = [](long e2, long N) {
+            const double a = -2.0 * M_PI * (double)(e2 % N) / (double)N;
+            return make_double2(std::cos(a), std::sin(a));
+        };
+        auto fill2d = [&](double2* dst, int r0, int r1) {
+            const int N = r0 * r1;
+            for (int bb = 0; bb < r0; ++bb)
+                for (int j = 1; j < r1; ++j) dst[(size_t)bb * (r1 - 1) + j - 1] = wd((long)j * bb, N);
+        };
+        fill2d(twd.data(), ops->row_r0, ops->row_r1);
+        fill2d(twd.data() + tw_row(ops), ops->col_r0, ops->col_r1);
+        for (int k = 0; k < ops->W; ++k) twd[tw_row(ops) + tw_col(ops) + k] = wd(k, ops->W);
+        if ((e = cudaMemcpyAsync(ctx->twMd, twd.data(), twd.size() * sizeof(double2),
+                                 cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
+            return bail(STITCH_ERR_CUDA);
+    } else if ((e = cudaMemcpyAsync(ctx->twM, tw.data(), tw.size() * sizeof(float2),
+                                    cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
         return bail(STITCH_ERR_CUDA);
     if (!pl.empty() &&
         (e = cudaMemcpyAsync(ctx->pairs, pl.data(), pl.size() * sizeof(PairIdx),
@@ -689,6 +790,14 @@ static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
     const int ct = ctx->L.chunk_tiles;
     for (int t0 = lt0; t0 < lt0 + count; t0 += ct) {
         const int nt = lt0 + count - t0 < ct ? lt0 + count - t0 : ct;
+        if (ctx->prec) {   // fp64 path (f2): D1, D2
+            o->d1(ctx->raw, ctx->Gd, t0, nt, ctx->twMd, ctx->twWd, ctx->stream);
+            CK(mark(ctx, 0), "event");
+            o->d2(ctx->Gd, ctx->Ud, t0, nt, ctx->twHd, true, ctx->stream);
+            CK(mark(ctx, 1), "event");
+            ctx->launches += 2;
+            continue;
+        }
         launch_k1_any(ctx, t0, nt, ctx->stream);
         CK(mark(ctx, 0), "event");
         if (ctx->grid_colp > 0)
@@ -714,6 +823,14 @@ static stitch_status pairs_impl(stitch_ctx* ctx) {
         const int cp = ctx->L.chunk_pairs;
         for (int64_t p0 = 0; p0 < np; p0 += cp) {
             const int npc = (int)(np - p0 < cp ? np - p0 : cp);
+            if (ctx->prec) {   // fp64 path (f2): D3, D4 (block argmax partials)
+                o->d3(ctx->Ud, ctx->Qd, ctx->pairs, (int)p0, npc, ctx->twHd, s);
+                CK(mark(ctx, 2), "event");
+                o->d4(ctx->Qd, ctx->part_v, ctx->part_i, (int)p0, npc, ctx->twMd, ctx->twWd, s);
+                CK(mark(ctx, 3), "event");
+                ctx->launches += 2;
+                continue;
+            }
             if (ctx->grid_colp > 0)
                 o->k3p(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, ctx->grid_colp, s);
             else
@@ -722,6 +839,12 @@ static stitch_status pairs_impl(stitch_ctx* ctx) {
             launch_k4_any(ctx, (int)p0, npc, s);
             CK(mark(ctx, 3), "event");
             ctx->launches += 2;
+        }
+        if (ctx->prec) {   // D5: per-pair reduction of the partials into the K5/K6 key
+            d5_argmax_keys<<<(unsigned)((np + 7) / 8), 256, 0, s>>>(ctx->part_v, ctx->part_i,
+                                                                   ctx->keys, o->nblk64, (int)np);
+            CK(mark(ctx, 3), "event");
+            ctx->launches += 1;
         }
         CK(cudaGetLastError(), "pair launch");
     }
@@ -910,7 +1033,8 @@ stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t 
     if (!ctx || !dev_ptr || !bytes) return STITCH_ERR_INVALID_ARG;
     if (count < 0 || first_tile < ctx->L.h_begin || first_tile + (int64_t)count > ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
-    const size_t per = (size_t)ctx->H * ctx->ops->WP * sizeof(uint32_t);
+    const size_t per =
+        (size_t)ctx->H * ctx->ops->WP * (ctx->prec ? sizeof(double2) : sizeof(uint32_t));
     *dev_ptr = reinterpret_cast<char*>(ctx->spec) + (size_t)(first_tile - ctx->L.h_begin) * per;
     *bytes = (size_t)count * per;
     return STITCH_OK;
@@ -976,6 +1100,7 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
     if (tile < ctx->L.h_begin || tile >= ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
+    if (ctx->prec) return fail(ctx, STITCH_ERR_STATE, "fp64 context: use stitch_debug_spectrum_f64");
     // The resident store keeps phase codes; recompute the complex spectrum of this tile
     // with the same K1 + K2 kernels into the chunk buffer G (slot 0) and copy it out.
     const int lt = tile - ctx->L.h_begin;
@@ -985,6 +1110,28 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
     CK(cudaGetLastError(), "spectrum launch");
     CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->G,
                          ctx->ops->WP * sizeof(float2), ctx->ops->WC * sizeof(float2), ctx->H,
+                         cudaMemcpyDeviceToHost, ctx->stream),
+       "copy spectrum");
+    CK(cudaStreamSynchronize(ctx->stream), "synchronize");
+    return STITCH_OK;
+}
+
+stitch_status stitch_debug_spectrum_f64(stitch_ctx* ctx, int32_t tile, double* host_out) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!host_out) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output");
+    if (!ctx->prec) return fail(ctx, STITCH_ERR_STATE, "fp32 context: use stitch_debug_spectrum");
+    if (tile < ctx->L.h_begin || tile >= ctx->L.t_end)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
+    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
+    // the resident store keeps unit phasors: recompute this tile's complex spectrum with the
+    // same D1 + D2 kernels into chunk slot 0 of Gd (D2 writing complex values in place)
+    const int lt = tile - ctx->L.h_begin;
+    const PlanOps* o = ctx->ops;
+    o->d1(ctx->raw, ctx->Gd, lt, 1, ctx->twMd, ctx->twWd, ctx->stream);
+    o->d2(ctx->Gd, ctx->Ud, lt, 1, ctx->twHd, false, ctx->stream);
+    CK(cudaGetLastError(), "spectrum launch");
+    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(double2), ctx->Gd,
+                         ctx->ops->WP * sizeof(double2), ctx->ops->WC * sizeof(double2), ctx->H,
                          cudaMemcpyDeviceToHost, ctx->stream),
        "copy spectrum");
     CK(cudaStreamSynchronize(ctx->stream), "synchronize");

@@ -85,6 +85,23 @@ def test_workspace_size_matches_layout(lib):
     assert raw + spec + chunks < ws < raw + spec + chunks + 5 * 2**20
 
 
+def test_fp64_workspace_and_precision_validation(lib):
+    """precision = 1 (f2): resident unit phasors and chunk intermediates in double2, plus the
+    per-row-block argmax partials; any other precision value is rejected."""
+    cfg = pkg.make_config(42, 59, 1040, 1392, chunk_pairs=8, chunk_tiles=8, precision=1)
+    ws = pkg.workspace_size(cfg)
+    H, W, WP = 1040, 1392, 704
+    raw = 2478 * H * W * 2
+    spec = 2478 * H * WP * 16         # resident unit phasors (double2)
+    chunks = 2 * 8 * H * WP * 16      # Gd + Qd
+    part = 4855 * (H // 4) * 12       # (double, u32) per pair and 4-row block
+    assert raw + spec + chunks + part < ws < raw + spec + chunks + part + 5 * 2**20
+    b = ctypes.c_size_t()
+    for bad in (2, -1):
+        cfg = pkg.make_config(3, 3, 192, 256, precision=bad)
+        assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 1
+
+
 def _eval_codelet(body, x):
     def fmaf(a, b, c):
         return a * b + c
@@ -93,14 +110,16 @@ def _eval_codelet(body, x):
     for line in body.split("\n"):
         line = line.strip().rstrip(";")
         line = re.sub(r"\((-?[0-9.e+-]+)f\)", r"(\1)", line).replace("0.0f", "0.0")
-        if line.startswith("const float"):
-            line = line[len("const float "):]
-            if "v[" in line:
-                py.extend(line.split(", "))
-            else:
-                py.append(line)
-        elif line.startswith("v["):
-            mm = re.match(r"v\[(\d+)\] = make_float2\((.*), (.*)\)", line)
+        line = line.replace("fma(", "fmaf(")
+        for ty in ("const float ", "const double "):
+            if line.startswith(ty):
+                line = line[len(ty):]
+                if "v[" in line:
+                    py.extend(line.split(", "))
+                else:
+                    py.append(line)
+        if line.startswith("v["):
+            mm = re.match(r"v\[(\d+)\] = make_(?:float|double)2\((.*), (.*)\)", line)
             py.append(f"out[{mm.group(1)}] = complex({mm.group(2)}, {mm.group(3)})")
 
     class F:
@@ -125,6 +144,26 @@ def test_generated_codelets_are_dfts():
         j = np.arange(n)
         ref = np.exp(sign * 2j * math.pi * np.outer(j, j) / n) @ x
         assert np.abs(got - ref).max() <= 1e-6 * np.abs(ref).max(), (n, tag)
+
+
+def test_generated_fp64_codelets_are_dfts():
+    """The fp64 twins (f2 path) are the same programs with double temporaries and
+    full-precision constants: evaluated in Python doubles they are the DFT to ~1e-15."""
+    src = open(os.path.join(ROOT, "paper_conf_icpp_blattnerkcsbz14_b200", "csrc",
+                            "codelets.cuh")).read()
+    funcs = re.findall(r"void dft(\d+)([mp])_d\(double2\* __restrict__ v\) \{\n(.*?)\n\}", src,
+                       re.S)
+    assert len(funcs) >= 20
+    assert not any("float" in body or "fmaf" in body for _, _, body in funcs)
+    rng = np.random.default_rng(1)
+    for n, tag, body in funcs:
+        n = int(n)
+        sign = -1 if tag == "m" else 1
+        x = rng.standard_normal(n) + 1j * rng.standard_normal(n)
+        got = _eval_codelet(body, x)
+        j = np.arange(n)
+        ref = np.exp(sign * 2j * math.pi * np.outer(j, j) / n) @ x
+        assert np.abs(got - ref).max() <= 1e-13 * np.abs(ref).max(), (n, tag)
 
 
 def test_phase_code_polynomial_matches_atan2():
