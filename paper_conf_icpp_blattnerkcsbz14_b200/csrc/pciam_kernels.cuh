@@ -141,7 +141,7 @@ __global__ void __launch_bounds__(PL::ROW_T) k1_fwd_rows(const uint16_t* __restr
                                                          const float2* __restrict__ tw2,
                                                          const float2* __restrict__ twW) {
     extern __shared__ float2 smem[];
-    constexpr int L = PL::ROW_L, T = PL::ROW_T, M = PL::M;
+    constexpr int L = PL::ROW_L, T = PL::ROW_T;
     const size_t t = (size_t)tile0 + blockIdx.y;
     const int y0 = blockIdx.x * L;
     U16RowSrc<PL> src{reinterpret_cast<const uint32_t*>(raw + (t * PL::H + y0) * PL::W)};
@@ -218,6 +218,24 @@ __device__ __forceinline__ void tma_panel(void* land, const CUtensorMap* map, in
         tma_load_2d(d + (size_t)y * PL::COL_P * elem_bytes, map, x, row0 + y, bar);
 }
 
+// The column kernels' stage-2 twiddle table (COL_TW2N float2) joins the panel's TMA
+// transaction as one bulk copy: a per-thread LDG -> STS loop here serialised an L2 round trip
+// per iteration at the start of every CTA (a quarter of K3's stall samples, ncu r01).
+template <class PL>
+struct ColTw {
+    static constexpr bool BULK = PL::COL_TW2N > 0 && (PL::COL_TW2N * 8) % 16 == 0;
+    static constexpr uint32_t BYTES = BULK ? (uint32_t)(PL::COL_TW2N * 8) : 0u;
+    // thread 0, inside the panel's transaction (the global table is 16-byte aligned)
+    static __device__ __forceinline__ void issue(float2* tws, const float2* tw2, uint64_t* bar) {
+        if constexpr (BULK) bulk_g2s(tws, tw2, BYTES, bar);
+    }
+    // every thread, if the table could not go by bulk copy
+    static __device__ __forceinline__ void fallback(float2* tws, const float2* tw2) {
+        if constexpr (!BULK)
+            for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    }
+};
+
 // K2: column FFT of a chunk of row-transformed tiles (G, complex, L2-resident), panel of
 // COL_P columns landed by TMA; writes the resident phase spectrum (or, for the test hook,
 // the complex spectrum back into G).
@@ -234,12 +252,13 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         fence_mbar_init();
     }
     __syncthreads();
-    if (threadIdx.x == 0) {
-        mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C);
-        tma_panel<PL>(csmem, &tmG, 2 * c0, tl * PL::H, 8, &bar);
-    }
     float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
-    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    if (threadIdx.x == 0) {
+        mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C + ColTw<PL>::BYTES);
+        tma_panel<PL>(csmem, &tmG, 2 * c0, tl * PL::H, 8, &bar);
+        ColTw<PL>::issue(tws, tw2, &bar);
+    }
+    ColTw<PL>::fallback(tws, tw2);
     mbar_wait(&bar, 0);
     LandSrc<PL> src{reinterpret_cast<const float2*>(csmem)};
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
@@ -284,13 +303,14 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         fence_mbar_init();
     }
     __syncthreads();
+    float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
     if (threadIdx.x == 0) {
-        mbar_arrive_expect_tx(&bar, (uint32_t)(2 * PL::H * PL::COL_P * 4));
+        mbar_arrive_expect_tx(&bar, (uint32_t)(2 * PL::H * PL::COL_P * 4) + ColTw<PL>::BYTES);
         tma_panel<PL>(la, &tmS, c0, pr.a * PL::H, 4, &bar);
         tma_panel<PL>(lb, &tmS, c0, pr.b * PL::H, 4, &bar);
+        ColTw<PL>::issue(tws, tw2, &bar);
     }
-    float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
-    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    ColTw<PL>::fallback(tws, tw2);
     mbar_wait(&bar, 0);
     NcpsPhaseSrc<PL> src{la, lb};
     PanelIO<PL> dst{Q + (size_t)blockIdx.y * PL::H * PL::WP + c0};
@@ -528,7 +548,7 @@ __global__ void __launch_bounds__(PL::ROW_T) k1p_fwd_rows(const uint16_t* __rest
                                                           const float2* __restrict__ twW) {
     using RP = RowPersist<PL>;
     extern __shared__ __align__(16) unsigned char smem_raw[];
-    constexpr int L = PL::ROW_L, T = PL::ROW_T, M = PL::M, BPT = PL::H / L;
+    constexpr int L = PL::ROW_L, T = PL::ROW_T, BPT = PL::H / L;
     uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + RP::OFF_BAR);
     float2* tw2s = reinterpret_cast<float2*>(smem_raw + RP::OFF_TW2);
     float2* twWs = reinterpret_cast<float2*>(smem_raw + RP::OFF_TWW);

@@ -274,8 +274,9 @@ const PlanOps* find_plan(int W, int H) {
 size_t align256(size_t x) { return (x + 255) / 256 * 256; }
 
 // twiddle tables: row stage-2 [r0*(r1-1)], column stage-2 [c0*(c1-1)], R2C/C2R w_W [W]
-size_t tw_row(const PlanOps* o) { return (size_t)o->row_r0 * (o->row_r1 - 1); }
-size_t tw_col(const PlanOps* o) { return (size_t)o->col_r0 * (o->col_r1 - 1); }
+// (slot counts rounded up to even, so every table starts 16-byte aligned for bulk copies)
+size_t tw_row(const PlanOps* o) { return ((size_t)o->row_r0 * (o->row_r1 - 1) + 1) & ~(size_t)1; }
+size_t tw_col(const PlanOps* o) { return ((size_t)o->col_r0 * (o->col_r1 - 1) + 1) & ~(size_t)1; }
 size_t tw_count(const PlanOps* o) { return tw_row(o) + tw_col(o) + o->W + 2; }
 
 struct Layout {
