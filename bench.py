@@ -396,11 +396,18 @@ def main():
 
     # ---- e2e: through the C ABI from pinned host buffers ------------------------------
     e2e_steps = max(1, args.e2e_steps)
+    pipelined = not bp.use_exchange           # whole-band contexts: H2D pipelined under compute
+    if pipelined:
+        pg.compute_from_host_async(host, first)     # warm: captures this buffer's graph
+        pg.get_translations()
     barrier()
     t0 = time.perf_counter()
     for _ in range(e2e_steps):
-        pg.load_tiles(host, first)                  # H2D of this rank's tile rows
-        bp.step_async()
+        if pipelined:   # per chunk: H2D of its tiles, then its transforms (stitch.h)
+            pg.compute_from_host_async(host, first)
+        else:
+            pg.load_tiles(host, first)              # H2D of this rank's tile rows
+            bp.step_async()
         west, north = pg.get_translations()         # D2H of the results, synchronous
     torch.cuda.synchronize()
     e2e_s = max_over_ranks((time.perf_counter() - t0) / e2e_steps)
@@ -452,7 +459,11 @@ def main():
             "roofline": roofline,
             "cpu_baseline": cpu,
             "e2e": {"value": total_pairs / e2e_s, "unit": "pairs/s", "h2d_bytes_per_step": h2d,
-                    "d2h_bytes_per_step": d2h, "grid_wall_ms": e2e_s * 1e3},
+                    "d2h_bytes_per_step": d2h, "grid_wall_ms": e2e_s * 1e3,
+                    "h2d_GBps": h2d / e2e_s / 1e9,
+                    "api": ("stitch_compute_translations_from_host_async (H2D pipelined per "
+                            "forward chunk) + stitch_get_translations" if pipelined else
+                            "stitch_load_tiles + step + stitch_get_translations")},
             "gpu_launches": launches,
             "clocks": clocks,
         }

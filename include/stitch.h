@@ -141,6 +141,20 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx);
  */
 stitch_status stitch_compute_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north);
 
+/*
+ * Steps 1-7 with step 1 pipelined (the paper's read/copier stages feeding its GPU stages,
+ * P:L1030-1040): `tiles` is a HOST run of consecutive tiles starting at `first_tile`
+ * covering the resident range (as stitch_load_tiles).  Each forward chunk's tiles are
+ * copied host-to-device on their own stream right before that chunk's transforms, so the
+ * copy of later chunks overlaps the transforms and pairs of earlier ones.  Asynchronous:
+ * the host buffer must stay valid and unmodified until stitch_get_translations /
+ * stitch_synchronize returns.  Pinned (page-locked) memory is needed for the overlap
+ * (pageable memory works, without it).  fp64 or timing contexts load, then compute.
+ * Errors: INVALID_ARG (null pointer, range does not cover the resident tiles); CUDA.
+ */
+stitch_status stitch_compute_translations_from_host_async(stitch_ctx* ctx, const uint16_t* tiles,
+                                                         int32_t first_tile, int32_t count);
+
 /* Copy the results of the last compute to the host (same layout as above). Synchronous. */
 stitch_status stitch_get_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north);
 

@@ -59,7 +59,8 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_last_timings", "stitch_set_timing", "stitch_last_error", "stitch_destroy",
            "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings",
            "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async",
-           "stitch_global_positions", "stitch_compose_overlay", "stitch_debug_spectrum_f64"]
+           "stitch_global_positions", "stitch_compose_overlay", "stitch_debug_spectrum_f64",
+           "stitch_compute_translations_from_host_async"]
 
 _lib = None
 
@@ -88,6 +89,7 @@ def load_library():
         "stitch_forward_async": (ctypes.c_int, [vp]),
         "stitch_debug_spectrum": (ctypes.c_int, [vp, i32, vp]),
         "stitch_debug_spectrum_f64": (ctypes.c_int, [vp, i32, vp]),
+        "stitch_compute_translations_from_host_async": (ctypes.c_int, [vp, vp, i32, i32]),
         "stitch_synchronize": (ctypes.c_int, [vp]),
         "stitch_last_counts": (ctypes.c_int, [vp, P(i64), P(i64), P(i64)]),
         "stitch_last_timings": (ctypes.c_int, [vp, P(ctypes.c_float)]),
@@ -250,6 +252,24 @@ class PciamGrid:
                 raise ValueError("tiles must be a contiguous torch.uint16 tensor")
             ptr, dev = tiles.data_ptr(), int(tiles.is_cuda)
         self._check(self.lib.stitch_load_tiles(self._ctx, ptr, first_tile, count, dev), "load")
+
+    def compute_from_host_async(self, tiles, first_tile: int = 0) -> None:
+        """Steps 1-7 with the host-to-device copy pipelined under the transforms: `tiles` is a
+        HOST run of consecutive tiles from `first_tile` (numpy or pinned torch CPU tensor,
+        [k, H, W] or [rows, m, H, W]) covering resident_range().  Keep it alive and unmodified
+        until get_translations() / synchronize()."""
+        if isinstance(tiles, np.ndarray):
+            if tiles.dtype != np.uint16 or not tiles.flags.c_contiguous:
+                raise ValueError("tiles must be C-contiguous uint16")
+            ptr, count = tiles.ctypes.data, tiles.size // (self.H * self.W)
+        else:
+            if tiles.is_cuda or not tiles.is_contiguous() or tiles.element_size() != 2:
+                raise ValueError("tiles must be a contiguous 16-bit host tensor")
+            ptr, count = tiles.data_ptr(), tiles.numel() // (self.H * self.W)
+        self._keep = tiles
+        self._check(self.lib.stitch_compute_translations_from_host_async(self._ctx, ptr,
+                                                                         first_tile, count),
+                    "compute from host")
 
     # -- steps 2-7 -------------------------------------------------------------
     def compute_translations_async(self) -> None:

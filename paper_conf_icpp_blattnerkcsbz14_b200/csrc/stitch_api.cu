@@ -379,7 +379,8 @@ struct stitch_ctx {
     // concurrent schedule (timing off): forward chunks, pair chunks and CCF chunks on three
     // internal streams joined by events, so compute-bound and memory-bound kernels overlap
     bool concurrent = true;
-    cudaStream_t s_fwd = nullptr, s_pair = nullptr, s_ccf = nullptr;
+    cudaStream_t s_fwd = nullptr, s_pair = nullptr, s_ccf = nullptr, s_h2d = nullptr;
+    std::vector<cudaEvent_t> ev_h2d;          // per forward chunk: its tiles have landed
     std::vector<cudaEvent_t> ev_fwd, ev_k4;   // per forward chunk / per pair chunk
     cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
     std::vector<int> pair_need;               // forward chunk completing each pair chunk's tiles
@@ -474,10 +475,12 @@ void stitch_destroy(stitch_ctx* ctx) {
         if (e) cudaEventDestroy(e);
     for (auto& e : ctx->ev_k4)
         if (e) cudaEventDestroy(e);
+    for (auto& e : ctx->ev_h2d)
+        if (e) cudaEventDestroy(e);
     if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
     for (auto& e : ctx->ev_join)
         if (e) cudaEventDestroy(e);
-    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf})
+    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d})
         if (st) cudaStreamDestroy(st);
     if (ctx->own_mem && ctx->mem) cudaFree(ctx->mem);
     if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
@@ -533,13 +536,17 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         const char* cenv = std::getenv("STITCH_CONCURRENT");  // STITCH_CONCURRENT=0: one stream
         ctx->concurrent = !(cenv && cenv[0] == '0') && !ctx->prec;
         if (ctx->concurrent) {
-            for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf})
+            for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf, &ctx->s_h2d})
                 if (cudaStreamCreateWithFlags(st, cudaStreamNonBlocking) != cudaSuccess)
                     return bail(STITCH_ERR_CUDA);
             const int nf = (L.nlocal + L.chunk_tiles - 1) / L.chunk_tiles;
             const int nc = (int)((L.npairs + L.chunk_pairs - 1) / L.chunk_pairs);
             ctx->ev_fwd.assign(nf, nullptr);
+            ctx->ev_h2d.assign(nf, nullptr);
             ctx->ev_k4.assign(nc, nullptr);
+            for (auto& e : ctx->ev_h2d)
+                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                    return bail(STITCH_ERR_CUDA);
             for (auto& e : ctx->ev_fwd)
                 if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
                     return bail(STITCH_ERR_CUDA);
@@ -893,7 +900,11 @@ static stitch_status step_begin(stitch_ctx* ctx) {
 // records an event per chunk; s_pair runs the pair chunks (K3, K4), each waiting for the
 // forward chunk that completes the tiles it reads; s_ccf runs K5 per pair chunk behind
 // its K4, then K6.  Buffers G (s_fwd) and Q (s_pair) are only touched by one stream.
-static stitch_status compute_concurrent(stitch_ctx* ctx) {
+// host_src (optional): the caller's host copy of the resident tiles [h_begin, t_end); each
+// forward chunk's tiles are copied on a fourth stream just before that chunk's K1, so the
+// H2D of later chunks overlaps the transforms and pairs of earlier ones (step 1 pipelined
+// with steps 2-7, as the paper's read/copier stages feed its GPU stages).
+static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_src = nullptr) {
     const PlanOps* o = ctx->ops;
     cudaStream_t m = ctx->stream;
     const int64_t np = ctx->L.npairs;
@@ -903,11 +914,20 @@ static stitch_status compute_concurrent(stitch_ctx* ctx) {
         CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), m), "memset");
     }
     CK(cudaEventRecord(ctx->ev_fork, m), "fork");
-    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf})
+    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d})
         CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
     cudaStream_t sf = ctx->s_fwd, sp = ctx->s_pair, sk = ctx->s_ccf;
+    const size_t tile_px = (size_t)ctx->H * ctx->W;
     for (int f = 0, t0 = 0; t0 < nl; ++f, t0 += ct) {
         const int nt = nl - t0 < ct ? nl - t0 : ct;
+        if (host_src) {
+            CK(cudaMemcpyAsync(ctx->raw + (size_t)t0 * tile_px, host_src + (size_t)t0 * tile_px,
+                               (size_t)nt * tile_px * sizeof(uint16_t), cudaMemcpyHostToDevice,
+                               ctx->s_h2d),
+               "chunk H2D");
+            CK(cudaEventRecord(ctx->ev_h2d[f], ctx->s_h2d), "event");
+            CK(cudaStreamWaitEvent(sf, ctx->ev_h2d[f], 0), "wait H2D");
+        }
         launch_k1_any(ctx, t0, nt, sf);
         if (ctx->grid_colp > 0)
             o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, sf);
@@ -941,6 +961,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx) {
         ctx->launches += 1;
     }
     CK(cudaGetLastError(), "concurrent launch");
+    // (s_h2d's last copy is ordered before the last K1 on s_fwd, so joining s_fwd covers it)
     cudaStream_t ss[3] = {sf, sp, sk};
     for (int i = 0; i < 3; ++i) {
         CK(cudaEventRecord(ctx->ev_join[i], ss[i]), "join");
@@ -1025,6 +1046,32 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
         if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
         return pairs_impl(ctx);
     });
+    if (st == STITCH_OK) ctx->computed = true;
+    return st;
+}
+
+stitch_status stitch_compute_translations_from_host_async(stitch_ctx* ctx, const uint16_t* tiles,
+                                                         int32_t first_tile, int32_t count) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!tiles) return fail(ctx, STITCH_ERR_INVALID_ARG, "null tiles pointer");
+    if (first_tile > ctx->L.h_begin || first_tile + (int64_t)count < ctx->L.t_end || first_tile < 0)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range does not cover [halo_begin, tile_end)");
+    const uint16_t* src = tiles + (size_t)(ctx->L.h_begin - first_tile) * ctx->H * ctx->W;
+    cudaPointerAttributes pa;
+    const bool pinned = cudaPointerGetAttributes(&pa, tiles) == cudaSuccess &&
+                        pa.type == cudaMemoryTypeHost;
+    cudaGetLastError();   // clear a pointer-query error on pageable memory
+    if (!ctx->concurrent || ctx->timing || !pinned) {   // no pipelining: load, then the step
+        stitch_status st = stitch_load_tiles(ctx, tiles, first_tile, count, 0);
+        if (st != STITCH_OK) return st;
+        return stitch_compute_translations_async(ctx);
+    }
+    stitch_status st = step_begin(ctx);
+    if (st != STITCH_OK) return st;
+    ctx->loaded = true;
+    // one captured graph per host buffer address (the copies' source is baked into it)
+    const uint64_t key = (4ull << 60) ^ (uint64_t)reinterpret_cast<uintptr_t>(src);
+    st = run_graphed(ctx, key, [&]() { return compute_concurrent(ctx, src); });
     if (st == STITCH_OK) ctx->computed = true;
     return st;
 }

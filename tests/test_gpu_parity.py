@@ -293,3 +293,36 @@ def test_stream_time_series_matches_per_grid():
     ow, on = oracle.grid(grids[3])
     assert np.array_equal(got[3].west["dx"][:, 1:], ow["dx"][:, 1:])
     assert np.array_equal(got[3].north["dy"][1:], on["dy"][1:])
+
+
+def test_compute_from_host_pipelined_matches_load_then_compute():
+    """Step 1 pipelined under steps 2-7 (stitch_compute_translations_from_host_async): the
+    per-chunk H2D copies on their own stream give bit-identical results to load + compute,
+    from pinned memory (pipelined, graph-captured, replayed) and from pageable memory
+    (load-then-compute fallback)."""
+    g = synthgrid.make_grid(5, 6, 192, 256, seed=51)
+    ref = run_gpu(g.tiles, chunk_tiles=4, chunk_pairs=8)
+    pinned = torch.empty(g.tiles.shape, dtype=torch.uint16, pin_memory=True)
+    pinned.numpy()[...] = g.tiles
+    with PciamGrid(5, 6, 192, 256, chunk_tiles=4, chunk_pairs=8) as pg:
+        for src in (pinned, pinned, g.tiles):
+            pg.compute_from_host_async(src, 0)
+            w, n = pg.get_translations()
+            assert w.tobytes() == ref[0].tobytes() and n.tobytes() == ref[1].tobytes()
+        # a second pinned buffer (its own captured graph)
+        pinned2 = torch.empty(g.tiles.shape, dtype=torch.uint16, pin_memory=True)
+        pinned2.numpy()[...] = g.tiles
+        pg.compute_from_host_async(pinned2, 0)
+        w, n = pg.get_translations()
+        assert w.tobytes() == ref[0].tobytes()
+    with PciamGrid(5, 6, 192, 256, tile_begin=12, tile_end=30) as pg:
+        h0, _, _ = pg.resident_range()
+        band = torch.empty((30 - h0, 192, 256), dtype=torch.uint16, pin_memory=True)
+        band.numpy()[...] = g.tiles.reshape(-1, 192, 256)[h0:]
+        pg.compute_from_host_async(band, h0)
+        w = np.zeros(30, ref[0].dtype); nn = np.zeros(30, ref[1].dtype)
+        pg.get_translations(w, nn)
+        assert w[12:].tobytes() == ref[0].reshape(-1)[12:].tobytes()
+        assert nn[12:].tobytes() == ref[1].reshape(-1)[12:].tobytes()
+        with pytest.raises(StitchError):
+            pg.compute_from_host_async(band[1:], h0 + 1)     # does not cover the halo
