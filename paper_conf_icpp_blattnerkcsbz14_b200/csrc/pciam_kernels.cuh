@@ -324,8 +324,11 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
 // item's panel lands by TMA in its own buffer; stage 1 reads it into registers, and right
 // after that barrier the TMA for the next item is issued, so the fetch overlaps stage 1's
 // butterflies, the exchange and stage 2 of the current item.
-template <class PL, bool PHASE_OUT>
-__global__ void __launch_bounds__(PL::COL_T, 1)
+// MINB: CTAs per SM the kernel is register-budgeted for.  TWG: stage-2 twiddles read through
+// L1 from global memory instead of a shared copy (the narrow-panel "quad" plans, 4 columns
+// per panel, fit three CTAs per SM only without it: landing + exchange = 67 KB per CTA).
+template <class PL, bool PHASE_OUT, int MINB = 1, bool TWG = false>
+__global__ void __launch_bounds__(PL::COL_T, MINB)
     k2p_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
                  uint32_t* __restrict__ spec, int tile0, int ntiles,
                  const float2* __restrict__ tw2) {
@@ -345,10 +348,12 @@ __global__ void __launch_bounds__(PL::COL_T, 1)
         mbar_init(&bar, 1);
         fence_mbar_init();
     }
-    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    if constexpr (!TWG)
+        for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    const float2* twp = TWG ? tw2 : tws;
     __syncthreads();
     if (threadIdx.x == 0 && (int)blockIdx.x < nitems) issue(blockIdx.x);
-    using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, true>;
+    using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, !TWG>;
     int k = 0;
     for (int item = blockIdx.x; item < nitems; item += gridDim.x, ++k) {
         mbar_wait(&bar, k & 1);
@@ -363,16 +368,16 @@ __global__ void __launch_bounds__(PL::COL_T, 1)
         LandSrc<PL> src{reinterpret_cast<const float2*>(csmem)};
         if constexpr (PHASE_OUT) {
             PhaseDst<PL> dst{spec + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
-            Run::template run<true>(src, xc, dst, tws, NoMid(), after_loads);
+            Run::template run<true>(src, xc, dst, twp, NoMid(), after_loads);
         } else {
             PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
-            Run::template run<true>(src, xc, dst, tws, NoMid(), after_loads);
+            Run::template run<true>(src, xc, dst, twp, NoMid(), after_loads);
         }
     }
 }
 
-template <class PL>
-__global__ void __launch_bounds__(PL::COL_T, 1)
+template <class PL, int MINB = 1, bool TWG = false>
+__global__ void __launch_bounds__(PL::COL_T, MINB)
     k3p_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
                   const PairIdx* __restrict__ pairs, int pair0, int npairs,
                   const float2* __restrict__ tw2) {
@@ -396,10 +401,12 @@ __global__ void __launch_bounds__(PL::COL_T, 1)
         mbar_init(&bar, 1);
         fence_mbar_init();
     }
-    for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    if constexpr (!TWG)
+        for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
+    const float2* twp = TWG ? tw2 : tws;
     __syncthreads();
     if (threadIdx.x == 0 && (int)blockIdx.x < nitems) issue(blockIdx.x);
-    using Run = FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, true>;
+    using Run = FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, !TWG>;
     int k = 0;
     for (int item = blockIdx.x; item < nitems; item += gridDim.x, ++k) {
         mbar_wait(&bar, k & 1);
@@ -413,7 +420,7 @@ __global__ void __launch_bounds__(PL::COL_T, 1)
         };
         NcpsPhaseSrc<PL> src{la, lb};
         PanelIO<PL> dst{Q + (size_t)pl * PL::H * PL::WP + c0};
-        Run::template run<true>(src, xc, dst, tws, NoMid(), after_loads);
+        Run::template run<true>(src, xc, dst, twp, NoMid(), after_loads);
     }
 }
 

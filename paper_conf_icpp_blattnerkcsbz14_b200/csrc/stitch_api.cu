@@ -16,6 +16,7 @@
 #include <map>
 #include <new>
 #include <string>
+#include <type_traits>
 #include <vector>
 
 #include "../../include/stitch.h"
@@ -33,6 +34,19 @@ using P1392 = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 
 using P256 = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 8, 128, 1, 1>;
 using P48 = Plan<48, 40, Radix<24, 24>, Radix<40, 40>, 8, 32, 8, 32, 0, 0>;
 using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 32, 8, 32, 0, 0>;
+
+// "Quad" column plans: the same transforms on 4-column panels, run by the persistent column
+// kernels with three CTAs per SM, each prefetching its next panel by TMA while it computes
+// (the one-panel-per-CTA kernels spend ~30 % of their stall samples waiting for their panel,
+// ncu r01c).  void: no quad variant for that plan.
+template <class PL> struct QuadOf { using type = void; };
+template <> struct QuadOf<P1392> {
+    using type = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 4, 160, 0, 1>;
+};
+template <> struct QuadOf<P256> {
+    using type = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 4, 64, 1, 1>;
+};
+constexpr int QUAD_MINB = 3;
 
 struct PlanOps {
     int W, H, M, WC, WP, row_l, col_p;
@@ -55,6 +69,12 @@ struct PlanOps {
     void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
                cudaStream_t);
+    // quad column plans (col_p_q = 0: none); setup returns the persistent grid
+    int col_p_q;
+    cudaError_t (*setup_q)(int* grid);
+    void (*k2q)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, int, cudaStream_t);
+    void (*k3q)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
+                cudaStream_t);
     // fp64 path (f2, pciam_fp64.cuh)
     int nblk64, colp64;
     cudaError_t (*d_setup)();
@@ -210,6 +230,57 @@ void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long lo
         raw, pairs, keys, mom, p0);
 }
 
+// ---- quad column plans
+template <class PL>
+cudaError_t setup_q(int* grid) {
+    *grid = 0;
+    using Q = typename QuadOf<PL>::type;
+    if constexpr (!std::is_void<Q>::value) {
+        cudaError_t e;
+        int dev = 0, sms = 0, nb2 = 0, nb3 = 0;
+        if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+        if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+            return e;
+        auto k2 = k2p_fwd_cols<Q, true, QUAD_MINB, true>;
+        auto k3 = k3p_pair_cols<Q, QUAD_MINB, true>;
+        if ((e = max_smem(k2, Q::COLP_TOFF)) != cudaSuccess) return e;
+        if ((e = max_smem(k3, Q::COLP_TOFF)) != cudaSuccess) return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb2, k2, Q::COL_T, Q::COLP_TOFF)) !=
+            cudaSuccess)
+            return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb3, k3, Q::COL_T, Q::COLP_TOFF)) !=
+            cudaSuccess)
+            return e;
+        *grid = std::min(nb2, nb3) * sms;
+    }
+    return cudaSuccess;
+}
+template <class PL>
+void launch_k2q(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt,
+                const float2* tw2, int grid, cudaStream_t s) {
+    using Q = typename QuadOf<PL>::type;
+    if constexpr (!std::is_void<Q>::value) {
+        const int items = nt * (Q::WP / Q::COL_P);
+        k2p_fwd_cols<Q, true, QUAD_MINB, true><<<grid < items ? grid : items, Q::COL_T,
+                                                 Q::COLP_TOFF, s>>>(tmG, G, spec, t0, nt, tw2);
+    }
+}
+template <class PL>
+void launch_k3q(const CUtensorMap& tmS, float2* Q_, const PairIdx* pairs, int p0, int np,
+                const float2* tw2, int grid, cudaStream_t s) {
+    using Q = typename QuadOf<PL>::type;
+    if constexpr (!std::is_void<Q>::value) {
+        const int items = np * (Q::WP / Q::COL_P);
+        k3p_pair_cols<Q, QUAD_MINB, true><<<grid < items ? grid : items, Q::COL_T, Q::COLP_TOFF,
+                                            s>>>(tmS, Q_, pairs, p0, np, tw2);
+    }
+}
+template <class PL>
+constexpr int quad_col_p() {
+    using Q = typename QuadOf<PL>::type;
+    if constexpr (std::is_void<Q>::value) return 0; else return Q::COL_P;
+}
+
 // ---- fp64 path launchers (f2)
 template <class PL>
 cudaError_t d_setup() {
@@ -258,7 +329,8 @@ PlanOps make_ops() {
                    PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
                    PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
                    launch_k2p<PL>, launch_k3p<PL>, launch_k1w<PL>, launch_k4w<PL>, launch_k1<PL>,
-                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>, Plan64<PL>::NBLK,
+                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>, quad_col_p<PL>(), setup_q<PL>,
+                   launch_k2q<PL>, launch_k3q<PL>, Plan64<PL>::NBLK,
                    Plan64<PL>::COL_P, d_setup<PL>, launch_d1<PL>, launch_d2<PL>, launch_d3<PL>,
                    launch_d4<PL>};
 }
@@ -356,6 +428,8 @@ struct stitch_ctx {
     double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
     uint32_t* part_i = nullptr;
     CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (phase codes)
+    CUtensorMap tmG4, tmS4;           // the same with the quad plans' 4-column boxes
+    int grid_colq = 0;                // quad persistent column kernels (0: not used)
     PairIdx* pairs;
     unsigned long long *keys, *mom;
     stitch_pair* res;
@@ -531,6 +605,14 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         int sms = 0;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
         ctx->grid_colp = (env && env[0] == '1') ? sms : 0;
+        // quad persistent column kernels (STITCH_COLQ=1; measured slower on B200, ncu r01q:
+        // the panel prefetch removes the TMA wait (30 % -> 3 % of K3's stall samples) but the
+        // 104-of-160-thread stage 1 leaves 22 % at barriers and the L1 twiddle loads another
+        // ~20 %: K3 11.2 -> 15.6 ms per step)
+        const char* qenv = std::getenv("STITCH_COLQ");
+        if (!ctx->prec && ops->col_p_q > 0 && qenv && qenv[0] == '1') {
+            if ((e = ops->setup_q(&ctx->grid_colq)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+        }
         const char* genv = std::getenv("STITCH_GRAPH");   // STITCH_GRAPH=0: direct launches
         ctx->use_graph = !(genv && genv[0] == '0');
         const char* cenv = std::getenv("STITCH_CONCURRENT");  // STITCH_CONCURRENT=0: one stream
@@ -614,26 +696,26 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
         const cuuint32_t boxh = (cuuint32_t)(ops->H / ((ops->H + 255) / 256));
         const cuuint32_t estr[2] = {1, 1};
-        {
-            const cuuint64_t dims[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
-            const cuuint64_t strides[1] = {(cuuint64_t)ops->WP * 8};
-            const cuuint32_t box[2] = {(cuuint32_t)2 * ops->col_p, boxh};
-            if (encode(&ctx->tmG, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, dims, strides, box,
-                       estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                       CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-                return bail(STITCH_ERR_CUDA);
-        }
-        {
-            const cuuint64_t dims[2] = {(cuuint64_t)ops->WP, (cuuint64_t)L.nlocal * ops->H};
-            const cuuint64_t strides[1] = {(cuuint64_t)ops->WP * 4};
-            const cuuint32_t box[2] = {(cuuint32_t)ops->col_p, boxh};
-            if (encode(&ctx->tmS, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->spec, dims, strides, box,
-                       estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                       CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                       CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
-                return bail(STITCH_ERR_CUDA);
-        }
+        // G: complex chunk [chunk_tiles*H][WP] as floats; spec: u32 phase codes [nlocal*H][WP]
+        auto encode_pair = [&](CUtensorMap* mg, CUtensorMap* ms, int colp) {
+            const cuuint64_t gd[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
+            const cuuint64_t gs[1] = {(cuuint64_t)ops->WP * 8};
+            const cuuint32_t gb[2] = {(cuuint32_t)2 * colp, boxh};
+            const cuuint64_t sd[2] = {(cuuint64_t)ops->WP, (cuuint64_t)L.nlocal * ops->H};
+            const cuuint64_t ss[1] = {(cuuint64_t)ops->WP * 4};
+            const cuuint32_t sb[2] = {(cuuint32_t)colp, boxh};
+            return encode(mg, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, gd, gs, gb, estr,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS &&
+                   encode(ms, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->spec, sd, ss, sb, estr,
+                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+        };
+        if (!encode_pair(&ctx->tmG, &ctx->tmS, ops->col_p)) return bail(STITCH_ERR_CUDA);
+        if (ctx->grid_colq > 0 && !encode_pair(&ctx->tmG4, &ctx->tmS4, ops->col_p_q))
+            return bail(STITCH_ERR_CUDA);
     }
 
     // Twiddles w_N^e = exp(-2 pi i e / N), computed in double, rounded once.
@@ -792,6 +874,27 @@ static void launch_k4_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s) {
         o->k4(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, s);
 }
 
+// Column kernels: quad persistent (3 CTAs/SM, TMA prefetch) where available, else the
+// persistent single-CTA variant if requested, else one CTA per panel.
+static void launch_k2_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
+    const PlanOps* o = ctx->ops;
+    if (ctx->grid_colq > 0)
+        o->k2q(ctx->tmG4, ctx->G, ctx->spec, t0, nt, ctx->twH, ctx->grid_colq, s);
+    else if (ctx->grid_colp > 0)
+        o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, s);
+    else
+        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, s);
+}
+static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s) {
+    const PlanOps* o = ctx->ops;
+    if (ctx->grid_colq > 0)
+        o->k3q(ctx->tmS4, ctx->Q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colq, s);
+    else if (ctx->grid_colp > 0)
+        o->k3p(ctx->tmS, ctx->Q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colp, s);
+    else
+        o->k3(ctx->tmS, ctx->Q, ctx->pairs, p0, np, ctx->twH, s);
+}
+
 // Forward transforms (K1 + K2) of the resident tiles with local indices [lt0, lt0 + count).
 static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
     const PlanOps* o = ctx->ops;
@@ -808,10 +911,7 @@ static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
         }
         launch_k1_any(ctx, t0, nt, ctx->stream);
         CK(mark(ctx, 0), "event");
-        if (ctx->grid_colp > 0)
-            o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, ctx->stream);
-        else
-            o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->stream);
+        launch_k2_any(ctx, t0, nt, ctx->stream);
         CK(mark(ctx, 1), "event");
         ctx->launches += 2;
     }
@@ -839,10 +939,7 @@ static stitch_status pairs_impl(stitch_ctx* ctx) {
                 ctx->launches += 2;
                 continue;
             }
-            if (ctx->grid_colp > 0)
-                o->k3p(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, ctx->grid_colp, s);
-            else
-                o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, s);
+            launch_k3_any(ctx, (int)p0, npc, s);
             CK(mark(ctx, 2), "event");
             launch_k4_any(ctx, (int)p0, npc, s);
             CK(mark(ctx, 3), "event");
@@ -929,10 +1026,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
             CK(cudaStreamWaitEvent(sf, ctx->ev_h2d[f], 0), "wait H2D");
         }
         launch_k1_any(ctx, t0, nt, sf);
-        if (ctx->grid_colp > 0)
-            o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, sf);
-        else
-            o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, sf);
+        launch_k2_any(ctx, t0, nt, sf);
         CK(cudaEventRecord(ctx->ev_fwd[f], sf), "event");
         ctx->launches += 2;
     }
@@ -945,10 +1039,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
             CK(cudaStreamWaitEvent(sp, ctx->ev_fwd[need], 0), "wait forward");
             waited = need;
         }
-        if (ctx->grid_colp > 0)
-            o->k3p(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, ctx->grid_colp, sp);
-        else
-            o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p0, npc, ctx->twH, sp);
+        launch_k3_any(ctx, (int)p0, npc, sp);
         launch_k4_any(ctx, (int)p0, npc, sp);
         CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
         CK(cudaStreamWaitEvent(sk, ctx->ev_k4[c], 0), "wait k4");
