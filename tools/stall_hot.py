@@ -1,3 +1,5 @@
+"""The SASS instructions with the most warp-stall samples in an ncu source-page CSV.
+Usage: python tools/stall_hot.py src.csv [top_n]"""
 import csv, sys
 rows = list(csv.reader(open(sys.argv[1])))
 # find header

@@ -1,3 +1,6 @@
+"""Warp-stall samples of an ncu source-page CSV (--page source --csv --print-source sass), summed
+over the SASS between barriers / mbarrier waits (or every N instructions), with the top stall
+reasons of each phase.  Usage: python tools/stall_phases.py src.csv [N]"""
 import csv,sys
 rows=list(csv.reader(open(sys.argv[1])))
 hi=next(i for i,r in enumerate(rows) if r and r[0]=="Address")
