@@ -24,6 +24,7 @@ from __future__ import annotations
 
 import argparse
 import json
+import math
 import os
 import subprocess
 import sys
@@ -38,6 +39,7 @@ sys.path.insert(0, ROOT)
 import synthgrid  # noqa: E402
 from paper_conf_icpp_blattnerkcsbz14_b200.parallel import band as parallel_band  # noqa: E402
 
+HBM_SPEC_GBPS = 8000.0             # B200 HBM3e spec (report fractions of both)
 PAPER_PAIRS_PER_S = 4855 / 49.7   # Pipelined-GPU, 1x Tesla C2070, Table II: context
 REASON_BITS = {0x1: "gpu_idle", 0x2: "applications_clocks_setting", 0x4: "sw_power_cap",
                0x8: "hw_slowdown", 0x10: "sync_boost", 0x20: "sw_thermal_slowdown",
@@ -387,6 +389,20 @@ def main():
     roofline["step_alg_GBps"] = design_bytes / (dev_ms / 1e3) / 1e9
     roofline["step_frac"] = roofline["step_alg_GBps"] / pk["hbm_gbs"]
     roofline["survey_2pass_GBps"] = survey_2pass / (dev_ms / 1e3) / 1e9
+    roofline["spec_frac"] = roofline["step_alg_GBps"] / HBM_SPEC_GBPS       # vs the ~8 TB/s spec
+    # FFT FLOP/s (north_star "FFT FLOP/s against the fp32 peak"): the nominal
+    # 2.5 N log2 N per real 2-D transform (N = HW), one per tile (forward) and one per pair
+    # (inverse), against 2 FLOP x 128 FP32 lanes x SMs x the SM clock measured under load
+    nominal = 2.5 * H * W * math.log2(H * W) * (fwd_tiles + pairs_local)
+    sm_mhz = clocks.get("sm_mhz") or pk.get("sm_max_mhz", 1965.0)
+    n_sm = torch.cuda.get_device_properties(local).multi_processor_count
+    fp_peak = 2 * 128 * n_sm * sm_mhz * 1e6 / 1e12
+    fft = {"nominal_flop_per_step": nominal, "achieved_tflops": nominal / (dev_ms / 1e3) / 1e12,
+           "peak_tflops": fp_peak, "peak": "fp64" if args.precision == "f64" else "fp32",
+           "sm_mhz": sm_mhz, "convention": "2.5 N log2 N per real 2-D transform, N = H*W"}
+    if args.precision == "f64":   # B200 FP64 vector rate: half the FP32 rate
+        fft["peak_tflops"] = fp_peak / 2
+    fft["frac"] = fft["achieved_tflops"] / fft["peak_tflops"]
     traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     if os.path.exists(traffic_path) and args.precision == "f32":   # captured on the fp32 kernels
         with open(traffic_path) as f:
@@ -457,6 +473,7 @@ def main():
                        "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)",
                        "overlap": cfg["overlap"], "seed": synthgrid.SEED},
             "roofline": roofline,
+            "fft_flops": fft,
             "cpu_baseline": cpu,
             "e2e": {"value": total_pairs / e2e_s, "unit": "pairs/s", "h2d_bytes_per_step": h2d,
                     "d2h_bytes_per_step": d2h, "grid_wall_ms": e2e_s * 1e3,

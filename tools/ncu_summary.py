@@ -36,6 +36,14 @@ def main():
             if k in h:
                 i = h.index(k)
                 print(f"  {k:66s} {v[i]:>16s} {u[i]}")
+        # counted FP32 FLOP rate (fadd + fmul + 2 ffma per thread instruction) vs the FFMA peak
+        fk = {k: f"smsp__sass_thread_inst_executed_op_{k}_pred_on.sum.per_cycle_elapsed"
+              for k in ("fadd", "fmul", "ffma")}
+        pk = "sm__sass_thread_inst_executed_op_ffma_pred_on.sum.peak_sustained"
+        if all(x in h for x in fk.values()) and pk in h:
+            fl = sum(float(v[h.index(fk[k])]) * (2 if k == "ffma" else 1) for k in fk)
+            peak = 2 * float(v[h.index(pk)])
+            print(f"  fp32 FLOP/cycle (fadd+fmul+2ffma) {fl:.0f} of peak {peak:.0f} = {fl / peak:.3f}")
         stalls = [(float(v[i]), h[i]) for i in range(len(h))
                   if h[i].startswith("smsp__average_warps_issue_stalled_")
                   and h[i].endswith("_per_issue_active.ratio") and v[i]]

@@ -6,7 +6,9 @@ SMOKE='import __graft_entry__ as g; g.smoke()'
 BIG='import numpy as np, synthgrid; from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid
 g = synthgrid.make_grid(2, 2, 1040, 1392)
 p = PciamGrid(2, 2, 1040, 1392, chunk_pairs=2, chunk_tiles=2); p.load_grid(g.tiles); w, n = p.compute_translations()
-print("big ok", w["dx"].tolist(), n["dy"].tolist())'
+q = PciamGrid(2, 2, 1040, 1392, precision=1); q.load_grid(g.tiles); w2, n2 = q.compute_translations()
+assert (w["dx"] == w2["dx"]).all() and (n["dy"] == n2["dy"]).all()
+print("big ok (fp32 + fp64)", w["dx"].tolist(), n["dy"].tolist())'
 for tool in memcheck racecheck synccheck initcheck; do
   echo "== $tool (config 1)"
   timeout 900 compute-sanitizer --tool $tool --print-limit 20 python -c "$SMOKE" 2>&1 | tail -6
