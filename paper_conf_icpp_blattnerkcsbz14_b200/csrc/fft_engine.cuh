@@ -92,6 +92,26 @@ struct NoMid {
     __device__ __forceinline__ void operator()() const {}
 };
 
+// A destination may take a whole butterfly's outputs at once (element b + j*STRIDE gets
+// v[j]) by defining store_batch<R, STRIDE>(line, b, v); otherwise they are stored one by one.
+template <class D, class = void>
+struct HasBatch {
+    static constexpr bool value = false;
+};
+template <class D>
+struct HasBatch<D, decltype((void)&D::BATCH)> {
+    static constexpr bool value = true;
+};
+template <int R, int STRIDE, class Dst, class C>
+__device__ __forceinline__ void store_butterfly(Dst& dst, int line, int b, C (&v)[R]) {
+    if constexpr (HasBatch<Dst>::value) {
+        dst.template store_batch<R, STRIDE>(line, b, v);
+    } else {
+#pragma unroll
+        for (int j = 0; j < R; ++j) dst.store(line, b + j * STRIDE, v[j]);
+    }
+}
+
 template <int N_, int... Rs>
 struct Radix {
     static constexpr int N = N_;
@@ -124,8 +144,7 @@ struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM, C> {
 #pragma unroll
                 for (int j = 0; j < R0; ++j) v[j] = src.load(line, j);
                 Dft<R0, SIGN>::run(v);
-#pragma unroll
-                for (int j = 0; j < R0; ++j) dst.store(line, j, v[j]);
+                store_butterfly<R0, 1>(dst, line, 0, v);
             }
         }
         __syncthreads();
@@ -222,8 +241,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
                         v[j] = SIGN < 0 ? cmul(v[j], w) : cmulc(v[j], w);
                     }
                     Dft<R1, SIGN>::run(v);
-#pragma unroll
-                    for (int j = 0; j < R1; ++j) dst.store(line, b + j * R0, v[j]);
+                    store_butterfly<R1, R0>(dst, line, b, v);
                 }
             }
         }

@@ -460,6 +460,28 @@ struct ArgmaxDst {  // step 5: running max of |x| with its row-major index, neve
         take(fabsf(v.x), idx);       // x[2n]
         take(fabsf(v.y), idx + 1);   // x[2n+1]
     }
+    // A whole butterfly (elements b + j*STRIDE): its max |x| by FMNMX (one instruction per
+    // value instead of compare + two selects), and only when that reaches the running best
+    // (rare once a line is under way) the smallest index holding it.  Same result as `store`
+    // value by value: the best value, ties to the smallest index (reading C6).
+    static constexpr bool BATCH = true;
+    template <int R, int STRIDE>
+    __device__ __forceinline__ void store_batch(int line, int b, const float2 (&v)[R]) {
+        float m = fmaxf(fabsf(v[0].x), fabsf(v[0].y));
+#pragma unroll
+        for (int j = 1; j < R; ++j) m = fmaxf(m, fmaxf(fabsf(v[j].x), fabsf(v[j].y)));
+        if (m >= best_v) {
+            const uint32_t base = (uint32_t)((row_base + line) * W + 2 * b);
+            uint32_t idx = 0xFFFFFFFFu;
+#pragma unroll
+            for (int j = R - 1; j >= 0; --j) {   // ends on the smallest index holding m
+                if (fabsf(v[j].y) == m) idx = base + 2 * j * STRIDE + 1;
+                if (fabsf(v[j].x) == m) idx = base + 2 * j * STRIDE;
+            }
+            if (m > best_v || idx < best_i) best_i = idx;
+            best_v = m;
+        }
+    }
     // packed key: larger |x| wins, then the smaller index (reading C6)
     __device__ __forceinline__ unsigned long long key() const {
         if (best_v < 0.f) return 0ull;

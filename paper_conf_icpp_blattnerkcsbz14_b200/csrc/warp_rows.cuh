@@ -60,8 +60,7 @@ struct WarpFft2<Radix<N, R0, R1>, SIGN, PAD> {
 #pragma unroll
             for (int j = 1; j < R1; ++j) v[j] = SIGN < 0 ? cmul(v[j], tw[j - 1]) : cmulc(v[j], tw[j - 1]);
             Dft<R1, SIGN>::run(v);
-#pragma unroll
-            for (int j = 0; j < R1; ++j) dst.store(0, lane + j * R0, v[j]);
+            store_butterfly<R1, R0>(dst, 0, lane, v);
         }
     }
 };
@@ -164,6 +163,41 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB1)
 }
 
 // ------------------------------------------------------------------ K4w ----
+// Step 5 for a warp that walks consecutive rows of one correlation surface: the running
+// (max |x|, smallest index) is kept warp-uniform.  Per row, each stage-2 lane reduces its
+// butterfly's outputs with FMNMX3 (two values per instruction) and one REDUX gives the row
+// maximum; only when that beats the running best does a lane holding it look up its index
+// (smallest among equal values, then REDUX-min over the lanes).  A later row cannot win a
+// tie: its indices are larger (reading C6).  |x| >= 0, so its float bits order as unsigned.
+template <int NLANES>
+struct WarpArgmaxDst {
+    float best_v;      // -1 before the first row
+    uint32_t best_i;
+    int row_base, W;
+    static constexpr unsigned MASK = NLANES >= 32 ? 0xFFFFFFFFu : ((1u << NLANES) - 1u);
+    static constexpr bool BATCH = true;
+    template <int R, int STRIDE>
+    __device__ __forceinline__ void store_batch(int line, int b, const float2 (&v)[R]) {
+        float m = fmaxf(fabsf(v[0].x), fabsf(v[0].y));
+#pragma unroll
+        for (int j = 1; j < R; ++j) m = fmaxf(m, fmaxf(fabsf(v[j].x), fabsf(v[j].y)));
+        const float M = __uint_as_float(__reduce_max_sync(MASK, __float_as_uint(m)));
+        if (M > best_v) {                      // warp-uniform
+            uint32_t idx = 0xFFFFFFFFu;
+            if (m == M) {
+                const uint32_t base = (uint32_t)((row_base + line) * W + 2 * b);
+#pragma unroll
+                for (int j = R - 1; j >= 0; --j) {
+                    if (fabsf(v[j].y) == M) idx = base + 2 * j * STRIDE + 1;
+                    if (fabsf(v[j].x) == M) idx = base + 2 * j * STRIDE;
+                }
+            }
+            best_i = __reduce_min_sync(MASK, idx);
+            best_v = M;
+        }
+    }
+};
+
 template <class PL>
 __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
     k4w_pair_rows(const float2* __restrict__ Q, unsigned long long* __restrict__ keys, int pair0,
@@ -200,7 +234,7 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
         if (lane == 0) atomicMax(&keys[pair0 + pair], key);
     };
     if (lane == 0 && r0 < r1) issue(r0);
-    ArgmaxDst acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
+    WarpArgmaxDst<RW::RI::R0> acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
     int cur = r0 < r1 ? r0 / H : -1;
     int k = 0;
     for (int r = r0; r < r1; ++r, ++k) {
