@@ -326,3 +326,26 @@ def test_compute_from_host_pipelined_matches_load_then_compute():
         assert nn[12:].tobytes() == ref[1].reshape(-1)[12:].tobytes()
         with pytest.raises(StitchError):
             pg.compute_from_host_async(band[1:], h0 + 1)     # does not cover the halo
+
+
+@pytest.mark.parametrize("env", [
+    {"STITCH_ROWWARP": "0"},                         # CTA row kernels (K1p/K4p)
+    {"STITCH_COL_PERSIST": "1"},                     # persistent column kernels (K2p/K3p)
+    {"STITCH_COLQ": "1"},                            # quad column plans (4-column panels)
+    {"STITCH_GRAPH": "0"},                           # direct launches
+    {"STITCH_CONCURRENT": "0"},                      # one stream
+    {"STITCH_ROWWARP": "0", "STITCH_COL_PERSIST": "1", "STITCH_GRAPH": "0"},
+])
+def test_launch_variants_bit_identical(env, monkeypatch):
+    """Every measured kernel / schedule variant (selected by environment at
+    stitch_init) gives bit-identical results to the default path, on the 256x192 plan and on
+    the headline 1392x1040 plan."""
+    for n, m, H, W, seed in [(3, 4, 192, 256, 61), (2, 3, 1040, 1392, 62)]:
+        g = synthgrid.make_grid(n, m, H, W, seed=seed)
+        ref = run_gpu(g.tiles, chunk_pairs=4, chunk_tiles=3)
+        for k, v in env.items():
+            monkeypatch.setenv(k, v)
+        got = run_gpu(g.tiles, chunk_pairs=4, chunk_tiles=3)
+        for k in env:
+            monkeypatch.delenv(k)
+        assert got[0].tobytes() == ref[0].tobytes() and got[1].tobytes() == ref[1].tobytes()
