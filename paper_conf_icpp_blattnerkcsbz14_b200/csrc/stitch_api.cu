@@ -345,6 +345,14 @@ const PlanOps* find_plan(int W, int H) {
 
 size_t align256(size_t x) { return (x + 255) / 256 * 256; }
 
+// Dual pair schedule (STITCH_DUAL=1): K3 and K4 on separate streams with two Q slots, and K4's
+// persistent grid limited to STITCH_DUAL_K4 CTAs per SM (default 1), so a K4 chunk and the next
+// chunk's K3 share every SM: the issue-bound row kernel fills the column kernel's TMA waits.
+int dual_pairs_env() {
+    const char* e = std::getenv("STITCH_DUAL");
+    return e && e[0] == '1';
+}
+
 // twiddle tables: row stage-2 [r0*(r1-1)], column stage-2 [c0*(c1-1)], R2C/C2R w_W [W]
 // (slot counts rounded up to even, so every table starts 16-byte aligned for bulk copies)
 size_t tw_row(const PlanOps* o) { return ((size_t)o->row_r0 * (o->row_r1 - 1) + 1) & ~(size_t)1; }
@@ -356,6 +364,7 @@ struct Layout {
     int64_t npairs;
     int chunk_pairs, chunk_tiles;
     int prec;   // 0 fp32, 1 fp64 (f2)
+    int q_slots;  // pair-chunk intermediates: 2 = K3(c+1) may run beside K4(c) (dual schedule)
     size_t off_raw, off_spec, off_g, off_q, off_pairs, off_keys, off_mom, off_res, off_tw,
         off_part, total;
 };
@@ -385,7 +394,8 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     L->off_raw = o;   o += align256((size_t)L->nlocal * H * W * sizeof(uint16_t));
     L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * spec_el);
     L->off_g = o;     o += align256((size_t)L->chunk_tiles * H * WP * cplx);
-    L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * cplx);
+    L->q_slots = (!L->prec && dual_pairs_env()) ? 2 : 1;
+    L->off_q = o;     o += align256((size_t)L->q_slots * L->chunk_pairs * H * WP * cplx);
     L->off_pairs = o; o += align256((size_t)(np > 0 ? np : 1) * sizeof(PairIdx));
     L->off_keys = o;  o += align256((size_t)(np > 0 ? np : 1) * sizeof(unsigned long long));
     L->off_mom = o;   o += align256((size_t)(np > 0 ? np : 1) * 20 * sizeof(unsigned long long));
@@ -422,6 +432,10 @@ struct stitch_ctx {
     uint16_t* raw;
     uint32_t* spec;                   // resident phase spectra [nlocal][H][WP]
     float2 *G, *Q, *twM, *twH, *twW;  // chunk intermediates, twiddles
+    float2* Q2 = nullptr;             // second pair-chunk slot (dual schedule)
+    int grid_k4w_dual = 0;            // K4w grid beside K3 (dual schedule)
+    cudaStream_t s_pair4 = nullptr;   // K4 stream (dual schedule)
+    std::vector<cudaEvent_t> ev_k3;   // per pair chunk: its Q is complete (dual schedule)
     int prec = 0;                     // 1: fp64 path (f2): the buffers below are used instead
     double2 *Gd = nullptr, *Qd = nullptr, *Ud = nullptr;   // Ud: resident unit phasors
     double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
@@ -551,6 +565,9 @@ void stitch_destroy(stitch_ctx* ctx) {
         if (e) cudaEventDestroy(e);
     for (auto& e : ctx->ev_h2d)
         if (e) cudaEventDestroy(e);
+    for (auto& e : ctx->ev_k3)
+        if (e) cudaEventDestroy(e);
+    if (ctx->s_pair4) cudaStreamDestroy(ctx->s_pair4);
     if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
     for (auto& e : ctx->ev_join)
         if (e) cudaEventDestroy(e);
@@ -629,6 +646,19 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
             for (auto& e : ctx->ev_h2d)
                 if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
                     return bail(STITCH_ERR_CUDA);
+            if (L.q_slots == 2 && ctx->grid_k4w > 0) {
+                if (cudaStreamCreateWithFlags(&ctx->s_pair4, cudaStreamNonBlocking) != cudaSuccess)
+                    return bail(STITCH_ERR_CUDA);
+                ctx->ev_k3.assign(nc, nullptr);
+                for (auto& e : ctx->ev_k3)
+                    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
+                        return bail(STITCH_ERR_CUDA);
+                const char* ke = std::getenv("STITCH_DUAL_K4");
+                const int per_sm = ke ? std::max(1, std::atoi(ke)) : 1;
+                int sms = 0;
+                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
+                ctx->grid_k4w_dual = std::min(ctx->grid_k4w, per_sm * sms);
+            }
             for (auto& e : ctx->ev_fwd)
                 if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
                     return bail(STITCH_ERR_CUDA);
@@ -666,6 +696,7 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     ctx->spec = (uint32_t*)(b + L.off_spec);
     ctx->G = (float2*)(b + L.off_g);
     ctx->Q = (float2*)(b + L.off_q);
+    if (L.q_slots == 2) ctx->Q2 = ctx->Q + (size_t)L.chunk_pairs * ops->H * ops->WP;
     ctx->pairs = (PairIdx*)(b + L.off_pairs);
     ctx->keys = (unsigned long long*)(b + L.off_keys);
     ctx->mom = (unsigned long long*)(b + L.off_mom);
@@ -864,14 +895,16 @@ static void launch_k1_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
     else
         o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, s);
 }
-static void launch_k4_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s) {
+static void launch_k4_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
+                          const float2* Qp = nullptr, int grid_w = 0) {
     const PlanOps* o = ctx->ops;
+    const float2* q = Qp ? Qp : ctx->Q;
     if (ctx->grid_k4w > 0)
-        o->k4w(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, ctx->grid_k4w, s);
+        o->k4w(q, ctx->keys, p0, np, ctx->twM, ctx->twW, grid_w > 0 ? grid_w : ctx->grid_k4w, s);
     else if (ctx->grid_k4p > 0)
-        o->k4p(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, ctx->grid_k4p, s);
+        o->k4p(q, ctx->keys, p0, np, ctx->twM, ctx->twW, ctx->grid_k4p, s);
     else
-        o->k4(ctx->Q, ctx->keys, p0, np, ctx->twM, ctx->twW, s);
+        o->k4(q, ctx->keys, p0, np, ctx->twM, ctx->twW, s);
 }
 
 // Column kernels: quad persistent (3 CTAs/SM, TMA prefetch) where available, else the
@@ -885,14 +918,16 @@ static void launch_k2_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
     else
         o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, s);
 }
-static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s) {
+static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
+                          float2* Qp = nullptr) {
     const PlanOps* o = ctx->ops;
+    float2* q = Qp ? Qp : ctx->Q;
     if (ctx->grid_colq > 0)
-        o->k3q(ctx->tmS4, ctx->Q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colq, s);
+        o->k3q(ctx->tmS4, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colq, s);
     else if (ctx->grid_colp > 0)
-        o->k3p(ctx->tmS, ctx->Q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colp, s);
+        o->k3p(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colp, s);
     else
-        o->k3(ctx->tmS, ctx->Q, ctx->pairs, p0, np, ctx->twH, s);
+        o->k3(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, s);
 }
 
 // Forward transforms (K1 + K2) of the resident tiles with local indices [lt0, lt0 + count).
@@ -1011,8 +1046,8 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
         CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), m), "memset");
     }
     CK(cudaEventRecord(ctx->ev_fork, m), "fork");
-    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d})
-        CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
+    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d, ctx->s_pair4})
+        if (st) CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
     cudaStream_t sf = ctx->s_fwd, sp = ctx->s_pair, sk = ctx->s_ccf;
     const size_t tile_px = (size_t)ctx->H * ctx->W;
     for (int f = 0, t0 = 0; t0 < nl; ++f, t0 += ct) {
@@ -1039,9 +1074,19 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
             CK(cudaStreamWaitEvent(sp, ctx->ev_fwd[need], 0), "wait forward");
             waited = need;
         }
-        launch_k3_any(ctx, (int)p0, npc, sp);
-        launch_k4_any(ctx, (int)p0, npc, sp);
-        CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
+        if (ctx->s_pair4) {   // dual schedule: slot c&1, K3 and K4 on their own streams
+            float2* q = (c & 1) ? ctx->Q2 : ctx->Q;
+            if (c >= 2) CK(cudaStreamWaitEvent(sp, ctx->ev_k4[c - 2], 0), "wait slot");
+            launch_k3_any(ctx, (int)p0, npc, sp, q);
+            CK(cudaEventRecord(ctx->ev_k3[c], sp), "event");
+            CK(cudaStreamWaitEvent(ctx->s_pair4, ctx->ev_k3[c], 0), "wait k3");
+            launch_k4_any(ctx, (int)p0, npc, ctx->s_pair4, q, ctx->grid_k4w_dual);
+            CK(cudaEventRecord(ctx->ev_k4[c], ctx->s_pair4), "event");
+        } else {
+            launch_k3_any(ctx, (int)p0, npc, sp);
+            launch_k4_any(ctx, (int)p0, npc, sp);
+            CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
+        }
         CK(cudaStreamWaitEvent(sk, ctx->ev_k4[c], 0), "wait k4");
         o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, sk);
         ctx->launches += 3;
@@ -1052,7 +1097,8 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
         ctx->launches += 1;
     }
     CK(cudaGetLastError(), "concurrent launch");
-    // (s_h2d's last copy is ordered before the last K1 on s_fwd, so joining s_fwd covers it)
+    // (s_h2d's last copy is ordered before the last K1 on s_fwd, and every K4 on s_pair4 before
+    // a K5 on s_ccf, so joining s_fwd, s_pair and s_ccf covers all streams)
     cudaStream_t ss[3] = {sf, sp, sk};
     for (int i = 0; i < 3; ++i) {
         CK(cudaEventRecord(ctx->ev_join[i], ss[i]), "join");
