@@ -1036,7 +1036,9 @@ static stitch_status step_begin(stitch_ctx* ctx) {
 // forward chunk's tiles are copied on a fourth stream just before that chunk's K1, so the
 // H2D of later chunks overlaps the transforms and pairs of earlier ones (step 1 pipelined
 // with steps 2-7, as the paper's read/copier stages feed its GPU stages).
-static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_src = nullptr) {
+// forward = false: steps 3-7 only (the split multi-GPU step: spectra already resident).
+static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_src = nullptr,
+                                        bool forward = true) {
     const PlanOps* o = ctx->ops;
     cudaStream_t m = ctx->stream;
     const int64_t np = ctx->L.npairs;
@@ -1050,7 +1052,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
         if (st) CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
     cudaStream_t sf = ctx->s_fwd, sp = ctx->s_pair, sk = ctx->s_ccf;
     const size_t tile_px = (size_t)ctx->H * ctx->W;
-    for (int f = 0, t0 = 0; t0 < nl; ++f, t0 += ct) {
+    for (int f = 0, t0 = 0; forward && t0 < nl; ++f, t0 += ct) {
         const int nt = nl - t0 < ct ? nl - t0 : ct;
         if (host_src) {
             CK(cudaMemcpyAsync(ctx->raw + (size_t)t0 * tile_px, host_src + (size_t)t0 * tile_px,
@@ -1070,7 +1072,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
         const int64_t p0 = (int64_t)c * cp;
         const int npc = (int)(np - p0 < cp ? np - p0 : cp);
         const int need = ctx->pair_need[c];
-        if (need > waited) {
+        if (forward && need > waited) {
             CK(cudaStreamWaitEvent(sp, ctx->ev_fwd[need], 0), "wait forward");
             waited = need;
         }
@@ -1166,7 +1168,11 @@ stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, in
 stitch_status stitch_pairs_async(stitch_ctx* ctx) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "pairs before load");
-    stitch_status st = run_graphed(ctx, 3ull << 60, [&]() { return pairs_impl(ctx); });
+    stitch_status st = run_graphed(ctx, 3ull << 60, [&]() {
+        // K5 on its own stream beside the K3/K4 chunks, as in the whole step
+        if (ctx->concurrent && !ctx->timing) return compute_concurrent(ctx, nullptr, false);
+        return pairs_impl(ctx);
+    });
     if (st == STITCH_OK) ctx->computed = true;
     return st;
 }
