@@ -210,7 +210,9 @@ stitch_status stitch_last_counts(stitch_ctx* ctx, int64_t* launches, int64_t* fo
 stitch_status stitch_last_timings(stitch_ctx* ctx, float* ms4);
 
 /* Event timing mode: 0 off (default), 1 per-stage events, 2 per-stage + one event after
- * every kernel launch (for per-kernel durations; perturbs the timeline slightly). */
+ * every kernel launch (for per-kernel durations; one stream, perturbs the timeline
+ * slightly), 3 the concurrent schedule launched directly with an event pair around every
+ * launch (stitch_timeline).  Anything else: INVALID_ARG. */
 stitch_status stitch_set_timing(stitch_ctx* ctx, int enabled);
 
 /* Mode-2 timings of the last compute per kernel K1..K6: summed device ms and launch counts.
@@ -245,6 +247,16 @@ stitch_status stitch_compose_overlay(const uint16_t* dev_tiles, int32_t n, int32
                                      int64_t canvas_h, uint16_t* dev_canvas, void* stream);
 
 /* Message for the last error on ctx (valid until the next call on ctx). */
+/*
+ * Measurement hook: after a compute with stitch_set_timing(ctx, 3) (the concurrent schedule
+ * launched directly, with an event pair around every launch) and stitch_synchronize /
+ * stitch_get_translations, the launch timeline: kernel id (0..5 = K1..K6), stream (0 forward,
+ * 1 pairs, 2 CCF), start and end in ms from the step's start.  Up to `capacity` records are
+ * written; *count = the number of records.  STATE if no timeline was collected.
+ */
+stitch_status stitch_timeline(stitch_ctx* ctx, int32_t* kernel, int32_t* stream, float* start_ms,
+                              float* end_ms, int64_t capacity, int64_t* count);
+
 const char* stitch_last_error(stitch_ctx* ctx);
 
 /* Release everything the context owns.  NULL-safe. */

@@ -60,7 +60,7 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings",
            "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async",
            "stitch_global_positions", "stitch_compose_overlay", "stitch_debug_spectrum_f64",
-           "stitch_compute_translations_from_host_async"]
+           "stitch_compute_translations_from_host_async", "stitch_timeline"]
 
 _lib = None
 
@@ -90,6 +90,7 @@ def load_library():
         "stitch_debug_spectrum": (ctypes.c_int, [vp, i32, vp]),
         "stitch_debug_spectrum_f64": (ctypes.c_int, [vp, i32, vp]),
         "stitch_compute_translations_from_host_async": (ctypes.c_int, [vp, vp, i32, i32]),
+        "stitch_timeline": (ctypes.c_int, [vp, vp, vp, vp, vp, i64, P(i64)]),
         "stitch_synchronize": (ctypes.c_int, [vp]),
         "stitch_last_counts": (ctypes.c_int, [vp, P(i64), P(i64), P(i64)]),
         "stitch_last_timings": (ctypes.c_int, [vp, P(ctypes.c_float)]),
@@ -341,7 +342,7 @@ class PciamGrid:
         return {"launches": a.value, "forward_ffts": b.value, "pairs": c.value}
 
     def set_timing(self, mode: int) -> None:
-        """0 off, 1 per-stage events, 2 per-stage + per-launch events."""
+        """0 off, 1 per-stage events, 2 per-stage + per-launch events, 3 timeline."""
         self._check(self.lib.stitch_set_timing(self._ctx, int(mode)), "timing")
 
     def kernel_timings(self) -> dict:
@@ -352,6 +353,21 @@ class PciamGrid:
         names = ["k1_fwd_rows", "k2_fwd_cols", "k3_pair_cols", "k4_pair_rows",
                  "k5_ccf_moments", "k6_finalize"]
         return {n: {"ms": ms[i], "launches": cnt[i]} for i, n in enumerate(names)}
+
+    def timeline(self) -> dict:
+        """Timing-mode-3 launch timeline of the last compute: arrays kernel (0..5 = K1..K6),
+        stream (0 forward, 1 pairs, 2 CCF), start_ms, end_ms (from the step's start)."""
+        cnt = ctypes.c_int64(0)
+        self._check(self.lib.stitch_timeline(self._ctx, None, None, None, None, 0,
+                                             ctypes.byref(cnt)), "timeline")
+        k = np.zeros(cnt.value, np.int32)
+        st = np.zeros(cnt.value, np.int32)
+        a = np.zeros(cnt.value, np.float32)
+        b = np.zeros(cnt.value, np.float32)
+        self._check(self.lib.stitch_timeline(self._ctx, k.ctypes.data, st.ctypes.data,
+                                             a.ctypes.data, b.ctypes.data, cnt.value,
+                                             ctypes.byref(cnt)), "timeline")
+        return {"kernel": k, "stream": st, "start_ms": a, "end_ms": b}
 
     def last_timings(self) -> dict:
         ms = (ctypes.c_float * 4)()

@@ -472,7 +472,17 @@ struct stitch_ctx {
     std::vector<cudaEvent_t> ev_fwd, ev_k4;   // per forward chunk / per pair chunk
     cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
     std::vector<int> pair_need;               // forward chunk completing each pair chunk's tiles
-    int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events
+    int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events,
+                     // 3 timeline of the concurrent schedule (events around every launch)
+    struct TlRec {
+        int8_t kid, stream;
+        cudaEvent_t a, b;
+    };
+    std::vector<TlRec> tl;             // timing 3: one record per launch
+    std::vector<cudaEvent_t> tl_pool;  // reusable events
+    size_t tl_used = 0;
+    cudaEvent_t tl_origin = nullptr;
+    std::vector<float> tl_ms;          // [2 * records]: start, end relative to the fork
     cudaEvent_t ev[4] = {nullptr, nullptr, nullptr, nullptr};
     float ms[4] = {0, 0, 0, 0};
     std::vector<cudaEvent_t> kev;     // per-launch events (timing == 2)
@@ -481,6 +491,33 @@ struct stitch_ctx {
     int64_t kcount[6] = {0, 0, 0, 0, 0, 0};
     std::string err;
 };
+
+// Timeline (timing mode 3): an event pair around a launch on stream `s` (index si).
+static cudaError_t tl_event(stitch_ctx* ctx, cudaEvent_t* out) {
+    if (ctx->tl_used == ctx->tl_pool.size()) {
+        cudaEvent_t e;
+        cudaError_t r = cudaEventCreate(&e);
+        if (r != cudaSuccess) return r;
+        ctx->tl_pool.push_back(e);
+    }
+    *out = ctx->tl_pool[ctx->tl_used++];
+    return cudaSuccess;
+}
+template <class F>
+static cudaError_t tl_wrap(stitch_ctx* ctx, cudaStream_t s, int si, int kid, F launch) {
+    if (ctx->timing != 3) {
+        launch();
+        return cudaSuccess;
+    }
+    stitch_ctx::TlRec r{(int8_t)kid, (int8_t)si, nullptr, nullptr};
+    cudaError_t e;
+    if ((e = tl_event(ctx, &r.a)) != cudaSuccess || (e = tl_event(ctx, &r.b)) != cudaSuccess) return e;
+    if ((e = cudaEventRecord(r.a, s)) != cudaSuccess) return e;
+    launch();
+    if ((e = cudaEventRecord(r.b, s)) != cudaSuccess) return e;
+    ctx->tl.push_back(r);
+    return cudaSuccess;
+}
 
 // Per-launch event (timing mode 2): kid 0..5 = K1..K6.
 static cudaError_t mark(stitch_ctx* ctx, int kid) {
@@ -566,6 +603,8 @@ void stitch_destroy(stitch_ctx* ctx) {
     for (auto& e : ctx->ev_h2d)
         if (e) cudaEventDestroy(e);
     for (auto& e : ctx->ev_k3)
+        if (e) cudaEventDestroy(e);
+    for (auto& e : ctx->tl_pool)
         if (e) cudaEventDestroy(e);
     if (ctx->s_pair4) cudaStreamDestroy(ctx->s_pair4);
     if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
@@ -1047,6 +1086,12 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
         CK(cudaMemsetAsync(ctx->keys, 0, (size_t)np * sizeof(unsigned long long), m), "memset");
         CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), m), "memset");
     }
+    if (ctx->timing == 3) {
+        ctx->tl.clear();
+        ctx->tl_used = 0;
+        CK(tl_event(ctx, &ctx->tl_origin), "event");
+        CK(cudaEventRecord(ctx->tl_origin, m), "event");
+    }
     CK(cudaEventRecord(ctx->ev_fork, m), "fork");
     for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d, ctx->s_pair4})
         if (st) CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
@@ -1062,8 +1107,8 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
             CK(cudaEventRecord(ctx->ev_h2d[f], ctx->s_h2d), "event");
             CK(cudaStreamWaitEvent(sf, ctx->ev_h2d[f], 0), "wait H2D");
         }
-        launch_k1_any(ctx, t0, nt, sf);
-        launch_k2_any(ctx, t0, nt, sf);
+        CK(tl_wrap(ctx, sf, 0, 0, [&] { launch_k1_any(ctx, t0, nt, sf); }), "timeline");
+        CK(tl_wrap(ctx, sf, 0, 1, [&] { launch_k2_any(ctx, t0, nt, sf); }), "timeline");
         CK(cudaEventRecord(ctx->ev_fwd[f], sf), "event");
         ctx->launches += 2;
     }
@@ -1085,17 +1130,21 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
             launch_k4_any(ctx, (int)p0, npc, ctx->s_pair4, q, ctx->grid_k4w_dual);
             CK(cudaEventRecord(ctx->ev_k4[c], ctx->s_pair4), "event");
         } else {
-            launch_k3_any(ctx, (int)p0, npc, sp);
-            launch_k4_any(ctx, (int)p0, npc, sp);
+            CK(tl_wrap(ctx, sp, 1, 2, [&] { launch_k3_any(ctx, (int)p0, npc, sp); }), "timeline");
+            CK(tl_wrap(ctx, sp, 1, 3, [&] { launch_k4_any(ctx, (int)p0, npc, sp); }), "timeline");
             CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
         }
         CK(cudaStreamWaitEvent(sk, ctx->ev_k4[c], 0), "wait k4");
-        o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, sk);
+        CK(tl_wrap(ctx, sk, 2, 4, [&] {
+               o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, sk);
+           }), "timeline");
         ctx->launches += 3;
     }
     if (np > 0) {
-        k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(ctx->keys, ctx->mom, ctx->res,
-                                                                  ctx->H, ctx->W, (int)np);
+        CK(tl_wrap(ctx, sk, 2, 5, [&] {
+               k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
+                   ctx->keys, ctx->mom, ctx->res, ctx->H, ctx->W, (int)np);
+           }), "timeline");
         ctx->launches += 1;
     }
     CK(cudaGetLastError(), "concurrent launch");
@@ -1183,7 +1232,7 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
     st = run_graphed(ctx, 1ull << 60, [&]() {
-        if (ctx->concurrent && !ctx->timing) return compute_concurrent(ctx);
+        if (ctx->concurrent && (!ctx->timing || ctx->timing == 3)) return compute_concurrent(ctx);
         stitch_status s2 = forward_impl(ctx, 0, ctx->L.nlocal);
         if (s2 != STITCH_OK) return s2;
         if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
@@ -1233,6 +1282,17 @@ stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t 
 
 static cudaError_t collect_timings(stitch_ctx* ctx) {
     cudaError_t e = cudaSuccess;
+    if (ctx->timing == 3) {
+        ctx->tl_ms.assign(2 * ctx->tl.size(), 0.f);
+        for (size_t i = 0; i < ctx->tl.size(); ++i) {
+            if ((e = cudaEventElapsedTime(&ctx->tl_ms[2 * i], ctx->tl_origin, ctx->tl[i].a)) !=
+                    cudaSuccess ||
+                (e = cudaEventElapsedTime(&ctx->tl_ms[2 * i + 1], ctx->tl_origin, ctx->tl[i].b)) !=
+                    cudaSuccess)
+                return e;
+        }
+        return cudaSuccess;
+    }
     if (ctx->timing) {
         for (int i = 0; i < 3; ++i)
             if ((e = cudaEventElapsedTime(&ctx->ms[i], ctx->ev[i], ctx->ev[i + 1])) != cudaSuccess)
@@ -1362,8 +1422,23 @@ stitch_status stitch_last_timings(stitch_ctx* ctx, float* ms4) {
 
 stitch_status stitch_set_timing(stitch_ctx* ctx, int enabled) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
-    if (enabled < 0 || enabled > 2) return fail(ctx, STITCH_ERR_INVALID_ARG, "timing mode 0..2");
+    if (enabled < 0 || enabled > 3) return fail(ctx, STITCH_ERR_INVALID_ARG, "timing mode 0..3");
     ctx->timing = enabled;
+    return STITCH_OK;
+}
+
+stitch_status stitch_timeline(stitch_ctx* ctx, int32_t* kernel, int32_t* stream, float* start_ms,
+                              float* end_ms, int64_t capacity, int64_t* count) {
+    if (!ctx || !count) return STITCH_ERR_INVALID_ARG;
+    *count = (int64_t)ctx->tl.size();
+    if (ctx->tl_ms.size() != 2 * ctx->tl.size())
+        return fail(ctx, STITCH_ERR_STATE, "no collected timeline (timing 3, then synchronize)");
+    for (int64_t i = 0; i < *count && i < capacity; ++i) {
+        if (kernel) kernel[i] = ctx->tl[i].kid;
+        if (stream) stream[i] = ctx->tl[i].stream;
+        if (start_ms) start_ms[i] = ctx->tl_ms[2 * i];
+        if (end_ms) end_ms[i] = ctx->tl_ms[2 * i + 1];
+    }
     return STITCH_OK;
 }
 
