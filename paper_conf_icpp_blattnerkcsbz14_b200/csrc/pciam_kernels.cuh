@@ -218,6 +218,23 @@ __device__ __forceinline__ void tma_panel(void* land, const CUtensorMap* map, in
         tma_load_2d(d + (size_t)y * PL::COL_P * elem_bytes, map, x, row0 + y, bar);
 }
 
+template <class PL>
+__device__ __forceinline__ void l2_prefetch_panel(const CUtensorMap* map, int x, int row0) {
+#pragma unroll 1
+    for (int y = 0; y < PL::H; y += PL::BOXH) tma_prefetch_l2_2d(map, x, row0 + y);
+}
+
+// L2 prefetch for the CTA `ahead` launch slots later (about one wave of resident CTAs): its
+// panel is pulled from DRAM into L2 while this CTA computes, so its own TMA loads hit L2
+// (the column kernels spend ~30 % of their stall samples waiting for their panel, ncu r01c).
+// Returns the (panel, item) of that CTA, or item < 0 if it is past the end of the grid.
+__device__ __forceinline__ void ahead_cta(int ahead, int& panel, int& item) {
+    const int lin = blockIdx.y * gridDim.x + blockIdx.x + ahead;
+    panel = lin % gridDim.x;
+    item = lin / gridDim.x;
+    if (ahead <= 0 || item >= (int)gridDim.y) item = -1;
+}
+
 // The column kernels' stage-2 twiddle table (COL_TW2N float2) joins the panel's TMA
 // transaction as one bulk copy: a per-thread LDG -> STS loop here serialised an L2 round trip
 // per iteration at the start of every CTA (a quarter of K3's stall samples, ncu r01).
@@ -242,7 +259,8 @@ struct ColTw {
 template <class PL, bool PHASE_OUT>
 __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     k2t_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
-                 uint32_t* __restrict__ spec, int tile0, const float2* __restrict__ tw2) {
+                 uint32_t* __restrict__ spec, int tile0, const float2* __restrict__ tw2,
+                 int ahead = 0) {
     extern __shared__ __align__(128) unsigned char csmem[];
     __shared__ uint64_t bar;
     const int tl = blockIdx.y, c0 = blockIdx.x * PL::COL_P;
@@ -257,6 +275,9 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C + ColTw<PL>::BYTES);
         tma_panel<PL>(csmem, &tmG, 2 * c0, tl * PL::H, 8, &bar);
         ColTw<PL>::issue(tws, tw2, &bar);
+        int pn, it;
+        ahead_cta(ahead, pn, it);
+        if (it >= 0) l2_prefetch_panel<PL>(&tmG, 2 * pn * PL::COL_P, it * PL::H);
     }
     ColTw<PL>::fallback(tws, tw2);
     mbar_wait(&bar, 0);
@@ -290,7 +311,8 @@ struct NcpsPhaseSrc {  // step 3 from two landed phase panels: exp(i (phi_A - ph
 template <class PL>
 __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     k3t_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
-                  const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2) {
+                  const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2,
+                  int ahead = 0) {
     extern __shared__ __align__(128) unsigned char csmem[];
     __shared__ uint64_t bar;
     const PairIdx pr = pairs[pair0 + blockIdx.y];
@@ -309,6 +331,13 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         tma_panel<PL>(la, &tmS, c0, pr.a * PL::H, 4, &bar);
         tma_panel<PL>(lb, &tmS, c0, pr.b * PL::H, 4, &bar);
         ColTw<PL>::issue(tws, tw2, &bar);
+        int pn, it;
+        ahead_cta(ahead, pn, it);
+        if (it >= 0) {
+            const PairIdx nx = pairs[pair0 + it];
+            l2_prefetch_panel<PL>(&tmS, pn * PL::COL_P, nx.a * PL::H);
+            l2_prefetch_panel<PL>(&tmS, pn * PL::COL_P, nx.b * PL::H);
+        }
     }
     ColTw<PL>::fallback(tws, tw2);
     mbar_wait(&bar, 0);

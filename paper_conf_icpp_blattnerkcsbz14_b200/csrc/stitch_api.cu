@@ -65,8 +65,10 @@ struct PlanOps {
     void (*k4w)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
                 cudaStream_t);
     void (*k1)(const uint16_t*, float2*, int, int, const float2*, const float2*, cudaStream_t);
-    void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, cudaStream_t);
-    void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
+    void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, int,
+               cudaStream_t);
+    void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
+               cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
                cudaStream_t);
     // quad column plans (col_p_q = 0: none); setup returns the persistent grid
@@ -150,18 +152,18 @@ void launch_k1(const uint16_t* raw, float2* G, int t0, int nt, const float2* twM
 }
 template <class PL>
 void launch_k2(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt, const float2* tw2,
-               bool phase_out, cudaStream_t s) {
+               bool phase_out, int ahead, cudaStream_t s) {
     const dim3 grid(PL::WP / PL::COL_P, nt);
     if (phase_out)
-        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2);
+        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2, ahead);
     else
-        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2);
+        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2, 0);
 }
 template <class PL>
 void launch_k3(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
-               const float2* tw2, cudaStream_t s) {
-    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(tmS, Q, pairs,
-                                                                                    p0, tw2);
+               const float2* tw2, int ahead, cudaStream_t s) {
+    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(
+        tmS, Q, pairs, p0, tw2, ahead);
 }
 template <class PL>
 void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const float2* twM,
@@ -444,6 +446,8 @@ struct stitch_ctx {
     CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (phase codes)
     CUtensorMap tmG4, tmS4;           // the same with the quad plans' 4-column boxes
     int grid_colq = 0;                // quad persistent column kernels (0: not used)
+    int col_ahead = 0;                // K2 L2 prefetch distance in CTAs (0: off)
+    int col_ahead3 = 0;               // K3 L2 prefetch distance in CTAs (0: off)
     PairIdx* pairs;
     unsigned long long *keys, *mom;
     stitch_pair* res;
@@ -661,6 +665,16 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         int sms = 0;
         cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
         ctx->grid_colp = (env && env[0] == '1') ? sms : 0;
+        // K2 / K3: L2 prefetch of the panels of the CTA one wave ahead (STITCH_L2PF /
+        // STITCH_L2PF3 = <CTAs>, 0 = off).  Measured: K2 7.25 -> 6.85 ms at one wave (2 CTAs
+        // x SMs); K3 slower (11.18 -> 11.53 ms: its prefetch needs the next pair's tile
+        // indices, a dependent global load in the prologue), so off for K3 by default.
+        {
+            const char* pf = std::getenv("STITCH_L2PF");
+            ctx->col_ahead = pf ? std::atoi(pf) : 2 * sms;
+            const char* pf3 = std::getenv("STITCH_L2PF3");
+            ctx->col_ahead3 = pf3 ? std::atoi(pf3) : 0;
+        }
         // quad persistent column kernels (STITCH_COLQ=1; measured slower on B200, ncu r01q:
         // the panel prefetch removes the TMA wait (30 % -> 3 % of K3's stall samples) but the
         // 104-of-160-thread stage 1 leaves 22 % at barriers and the L1 twiddle loads another
@@ -955,7 +969,7 @@ static void launch_k2_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
     else if (ctx->grid_colp > 0)
         o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, s);
     else
-        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, s);
+        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->col_ahead, s);
 }
 static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
                           float2* Qp = nullptr) {
@@ -966,7 +980,7 @@ static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
     else if (ctx->grid_colp > 0)
         o->k3p(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colp, s);
     else
-        o->k3(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, s);
+        o->k3(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->col_ahead3, s);
 }
 
 // Forward transforms (K1 + K2) of the resident tiles with local indices [lt0, lt0 + count).
@@ -1357,7 +1371,7 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
     const int lt = tile - ctx->L.h_begin;
     const PlanOps* o = ctx->ops;
     launch_k1_any(ctx, lt, 1, ctx->stream);
-    o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->twH, false, ctx->stream);
+    o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->twH, false, 0, ctx->stream);
     CK(cudaGetLastError(), "spectrum launch");
     CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->G,
                          ctx->ops->WP * sizeof(float2), ctx->ops->WC * sizeof(float2), ctx->H,
