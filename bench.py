@@ -253,6 +253,9 @@ def main():
     ap.add_argument("--ts-slots", type=int, default=2, help="config 4: grid slots in flight")
     ap.add_argument("--precision", default="f32", choices=["f32", "f64"],
                     help="arithmetic of steps 2-5 (f64: the optional fp64 path, SURVEY 8 f2)")
+    ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
+                    help="gloo: logic check of the N > 1 path with ranks sharing GPUs (not a "
+                         "bench number; the halo goes through host memory)")
     ap.add_argument("--no-exchange", action="store_true",
                     help="N > 1: recompute the halo row's spectra instead of receiving them")
     args = ap.parse_args()
@@ -272,9 +275,17 @@ def main():
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world != args.gpus:
         raise SystemExit(f"--gpus {args.gpus} but WORLD_SIZE={world}")
+    if args.dist_backend == "gloo":
+        # logic check of the multi-rank path on fewer GPUs than ranks: ranks share devices,
+        # the halo exchange stages through host memory (parallel.exchange_halo)
+        local = local % torch.cuda.device_count()
     torch.cuda.set_device(local)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if args.dist_backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group("gloo")
+    red_dev = "cuda" if args.dist_backend == "nccl" else "cpu"
 
     n, m, H, W = cfg["n"], cfg["m"], cfg["H"], cfg["W"]
     b, e, halo = band(rank, world, n, m)
@@ -304,14 +315,14 @@ def main():
     def max_over_ranks(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64, device=red_dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
     def sum_over_ranks(x: float) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device="cuda")
+        t = torch.tensor([x], dtype=torch.float64, device=red_dev)
         dist.all_reduce(t, op=dist.ReduceOp.SUM)
         return float(t.item())
 
@@ -393,7 +404,8 @@ def main():
     # FFT FLOP/s (north_star "FFT FLOP/s against the fp32 peak"): the nominal
     # 2.5 N log2 N per real 2-D transform (N = HW), one per tile (forward) and one per pair
     # (inverse), against 2 FLOP x 128 FP32 lanes x SMs x the SM clock measured under load
-    nominal = 2.5 * H * W * math.log2(H * W) * (fwd_tiles + pairs_local)
+    # whole job: every rank's transforms (halo rows recomputed without the exchange count too)
+    nominal = 2.5 * H * W * math.log2(H * W) * sum_over_ranks(fwd_tiles + pairs_local)
     sm_mhz = clocks.get("sm_mhz") or pk.get("sm_max_mhz", 1965.0)
     n_sm = torch.cuda.get_device_properties(local).multi_processor_count
     fp_peak = 2 * 128 * n_sm * sm_mhz * 1e6 / 1e12
@@ -427,8 +439,8 @@ def main():
         west, north = pg.get_translations()         # D2H of the results, synchronous
     torch.cuda.synchronize()
     e2e_s = max_over_ranks((time.perf_counter() - t0) / e2e_steps)
-    h2d = (e - halo) * T
-    d2h = pairs_local * 64
+    h2d = sum_over_ranks((e - halo) * T)          # whole job: every rank's tile rows
+    d2h = sum_over_ranks(pairs_local * 64)
 
     # ---- optional: stitching phases 2 + 3 on the result (NEXT rows f3, f4) -------------
     phase23 = None

@@ -74,8 +74,20 @@ def halo_plan(rank: int, world: int, n: int, m: int) -> HaloPlan:
 
 
 def exchange_halo(send_buf, recv_buf, rank: int, world: int, group=None) -> None:
-    """Send `send_buf` to rank+1 and receive `recv_buf` from rank-1 (batched P2P)."""
+    """Send `send_buf` to rank+1 and receive `recv_buf` from rank-1 (batched P2P).  NCCL moves
+    device buffers GPU to GPU; under gloo (CPU tests, or the bench's --dist-backend gloo logic
+    check) device buffers are staged through host memory."""
     import torch.distributed as dist
+    if dist.get_backend(group) == "gloo" and any(b is not None and b.is_cuda
+                                                 for b in (send_buf, recv_buf)):
+        import torch
+        torch.cuda.current_stream().synchronize()
+        s_host = send_buf.cpu() if send_buf is not None else None
+        r_host = torch.empty_like(recv_buf, device="cpu") if recv_buf is not None else None
+        exchange_halo(s_host, r_host, rank, world, group)
+        if recv_buf is not None:
+            recv_buf.copy_(r_host)
+        return
     ops = []
     if send_buf is not None and rank + 1 < world:
         ops.append(dist.P2POp(dist.isend, send_buf, rank + 1, group))
