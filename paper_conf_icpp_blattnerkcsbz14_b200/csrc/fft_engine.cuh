@@ -118,13 +118,31 @@ struct Radix {
     static constexpr int count = sizeof...(Rs);
 };
 
-// C: the complex element type (float2, or double2 for the fp64 path f2)
-template <class RX, int SIGN, int L, int T, class Map, bool TW_SMEM = false, class C = float2>
+// The threads that run one transform batch: the whole CTA (default), or one of several
+// independent thread groups of a CTA (GroupOf<GT>: group g = threadIdx.x / GT synchronises on
+// named barrier 1 + g, so groups never wait for each other).
+struct CtaGrp {
+    static __device__ __forceinline__ int tid() { return threadIdx.x; }
+    static __device__ __forceinline__ void sync() { __syncthreads(); }
+};
+template <int GT>
+struct GroupOf {
+    static_assert(GT % 32 == 0, "thread groups are whole warps");
+    static __device__ __forceinline__ int tid() { return threadIdx.x % GT; }
+    static __device__ __forceinline__ int id() { return threadIdx.x / GT; }
+    static __device__ __forceinline__ void sync() {
+        asm volatile("bar.sync %0, %1;" ::"r"(1 + id()), "n"(GT) : "memory");
+    }
+};
+
+// C: the complex element type (float2, or double2 for the fp64 path f2); Grp: the thread group
+template <class RX, int SIGN, int L, int T, class Map, bool TW_SMEM = false, class C = float2,
+          class Grp = CtaGrp>
 struct FftRun;
 
 // One stage: N = R0, no twiddles, source -> destination.
-template <int N, int R0, int SIGN, int L, int T, class Map, bool TW_SMEM, class C>
-struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM, C> {
+template <int N, int R0, int SIGN, int L, int T, class Map, bool TW_SMEM, class C, class Grp>
+struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM, C, Grp> {
     static_assert(N == R0, "single-stage plan");
     static constexpr int R1 = 1;
     template <bool IN_PLACE = false, class Src, class Xc, class Dst, class Mid = NoMid,
@@ -137,7 +155,7 @@ struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM, C> {
         constexpr int ITER = (TOTAL + T - 1) / T;
 #pragma unroll
         for (int it = 0; it < ITER; ++it) {
-            const int g = threadIdx.x + it * T;
+            const int g = Grp::tid() + it * T;
             if (TOTAL % T == 0 || g < TOTAL) {
                 const int line = g;
                 C v[R0];
@@ -147,15 +165,16 @@ struct FftRun<Radix<N, R0>, SIGN, L, T, Map, TW_SMEM, C> {
                 store_butterfly<R0, 1>(dst, line, 0, v);
             }
         }
-        __syncthreads();
+        Grp::sync();
         after_loads();
         mid();
     }
 };
 
 // Two stages: N = R0 * R1, one exchange through shared memory.
-template <int N, int R0_, int R1_, int SIGN, int L, int T, class Map, bool TW_SMEM, class C>
-struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
+template <int N, int R0_, int R1_, int SIGN, int L, int T, class Map, bool TW_SMEM, class C,
+          class Grp>
+struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C, Grp> {
     static constexpr int R0 = R0_, R1 = R1_;
     static_assert(N == R0 * R1, "radices must multiply to N");
     // Stage 1: radix R0 over R1 butterflies per line, source -> exchange.  IN_PLACE: the
@@ -170,7 +189,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
             C v[ITER][R0];
 #pragma unroll
             for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
+                const int g = Grp::tid() + it * T;
                 if (TOTAL % T == 0 || g < TOTAL) {
                     int line, b;
                     Map::template map<R1, L>(g, line, b);
@@ -178,11 +197,11 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
                     for (int j = 0; j < R0; ++j) v[it][j] = src.load(line, b + j * R1);
                 }
             }
-            __syncthreads();
+            Grp::sync();
             after_loads();   // the source buffer is free from here on
 #pragma unroll
             for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
+                const int g = Grp::tid() + it * T;
                 if (TOTAL % T == 0 || g < TOTAL) {
                     int line, b;
                     Map::template map<R1, L>(g, line, b);
@@ -194,7 +213,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
         } else {
 #pragma unroll
             for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
+                const int g = Grp::tid() + it * T;
                 if (TOTAL % T == 0 || g < TOTAL) {
                     int line, b;
                     Map::template map<R1, L>(g, line, b);
@@ -218,7 +237,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
                                                const Mid& mid = Mid(),
                                                const AfterLoads& after_loads = AfterLoads()) {
         stage1<IN_PLACE>(src, xc, after_loads);
-        __syncthreads();
+        Grp::sync();
         mid();
         {   // stage 2: radix R1 over R0 butterflies per line, exchange -> destination
             constexpr int TOTAL = L * R0;
@@ -227,7 +246,7 @@ struct FftRun<Radix<N, R0_, R1_>, SIGN, L, T, Map, TW_SMEM, C> {
             // inside the instruction cache
 #pragma unroll 1
             for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
+                const int g = Grp::tid() + it * T;
                 if (TOTAL % T == 0 || g < TOTAL) {
                     int line, b;
                     Map::template map<R0, L>(g, line, b);

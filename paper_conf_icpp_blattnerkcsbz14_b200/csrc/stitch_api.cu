@@ -22,6 +22,7 @@
 #include "../../include/stitch.h"
 #include "pciam_kernels.cuh"
 #include "pciam_fp64.cuh"
+#include "col_groups.cuh"
 
 using namespace stitch;
 
@@ -71,6 +72,11 @@ struct PlanOps {
                cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
                cudaStream_t);
+    // two-group column kernels (K2g/K3g); setup_g returns the grid (0: none for this plan)
+    cudaError_t (*setup_g)(int* grid);
+    void (*k2g)(const CUtensorMap&, uint32_t*, int, int, const float2*, int, cudaStream_t);
+    void (*k3g)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
+                cudaStream_t);
     // quad column plans (col_p_q = 0: none); setup returns the persistent grid
     int col_p_q;
     cudaError_t (*setup_q)(int* grid);
@@ -232,6 +238,50 @@ void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long lo
         raw, pairs, keys, mom, p0);
 }
 
+// ---- two-group column kernels
+template <class PL>
+cudaError_t setup_g(int* grid) {
+    *grid = 0;
+    using CG = ColGroups<PL>;
+    if constexpr (CG::OK) {
+        cudaError_t e;
+        int dev = 0, sms = 0, nb2 = 0, nb3 = 0;
+        if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
+        if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
+            return e;
+        if ((e = max_smem(k2g_fwd_cols<PL>, CG::SMEM)) != cudaSuccess) return e;
+        if ((e = max_smem(k3g_pair_cols<PL>, CG::SMEM)) != cudaSuccess) return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb2, k2g_fwd_cols<PL>, CG::NT,
+                                                                CG::SMEM)) != cudaSuccess)
+            return e;
+        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb3, k3g_pair_cols<PL>, CG::NT,
+                                                                CG::SMEM)) != cudaSuccess)
+            return e;
+        *grid = std::min(nb2, nb3) * sms;
+    }
+    return cudaSuccess;
+}
+template <class PL>
+void launch_k2g(const CUtensorMap& tmG, uint32_t* spec, int t0, int nt, const float2* tw2,
+                int grid, cudaStream_t s) {
+    using CG = ColGroups<PL>;
+    if constexpr (CG::OK) {
+        const int items = nt * (PL::WP / PL::COL_P);
+        k2g_fwd_cols<PL><<<grid < items ? grid : items, CG::NT, CG::SMEM, s>>>(tmG, spec, t0, nt,
+                                                                              tw2);
+    }
+}
+template <class PL>
+void launch_k3g(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
+                const float2* tw2, int grid, cudaStream_t s) {
+    using CG = ColGroups<PL>;
+    if constexpr (CG::OK) {
+        const int items = np * (PL::WP / PL::COL_P);
+        k3g_pair_cols<PL><<<grid < items ? grid : items, CG::NT, CG::SMEM, s>>>(tmS, Q, pairs, p0,
+                                                                               np, tw2);
+    }
+}
+
 // ---- quad column plans
 template <class PL>
 cudaError_t setup_q(int* grid) {
@@ -331,7 +381,8 @@ PlanOps make_ops() {
                    PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
                    PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
                    launch_k2p<PL>, launch_k3p<PL>, launch_k1w<PL>, launch_k4w<PL>, launch_k1<PL>,
-                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>, quad_col_p<PL>(), setup_q<PL>,
+                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>, setup_g<PL>, launch_k2g<PL>,
+                   launch_k3g<PL>, quad_col_p<PL>(), setup_q<PL>,
                    launch_k2q<PL>, launch_k3q<PL>, Plan64<PL>::NBLK,
                    Plan64<PL>::COL_P, d_setup<PL>, launch_d1<PL>, launch_d2<PL>, launch_d3<PL>,
                    launch_d4<PL>};
@@ -446,6 +497,7 @@ struct stitch_ctx {
     CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (phase codes)
     CUtensorMap tmG4, tmS4;           // the same with the quad plans' 4-column boxes
     int grid_colq = 0;                // quad persistent column kernels (0: not used)
+    int grid_colg = 0;                // two-group column kernels (0: not used)
     int col_ahead = 0;                // K2 L2 prefetch distance in CTAs (0: off)
     int col_ahead3 = 0;               // K3 L2 prefetch distance in CTAs (0: off)
     PairIdx* pairs;
@@ -674,6 +726,12 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
             ctx->col_ahead = pf ? std::atoi(pf) : 2 * sms;
             const char* pf3 = std::getenv("STITCH_L2PF3");
             ctx->col_ahead3 = pf3 ? std::atoi(pf3) : 0;
+        }
+        // two-group persistent column kernels (STITCH_COLG=1)
+        {
+            const char* genv2 = std::getenv("STITCH_COLG");
+            if (!ctx->prec && genv2 && genv2[0] == '1')
+                if ((e = ops->setup_g(&ctx->grid_colg)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
         }
         // quad persistent column kernels (STITCH_COLQ=1; measured slower on B200, ncu r01q:
         // the panel prefetch removes the TMA wait (30 % -> 3 % of K3's stall samples) but the
@@ -964,7 +1022,9 @@ static void launch_k4_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
 // persistent single-CTA variant if requested, else one CTA per panel.
 static void launch_k2_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
     const PlanOps* o = ctx->ops;
-    if (ctx->grid_colq > 0)
+    if (ctx->grid_colg > 0)
+        o->k2g(ctx->tmG, ctx->spec, t0, nt, ctx->twH, ctx->grid_colg, s);
+    else if (ctx->grid_colq > 0)
         o->k2q(ctx->tmG4, ctx->G, ctx->spec, t0, nt, ctx->twH, ctx->grid_colq, s);
     else if (ctx->grid_colp > 0)
         o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, s);
@@ -975,7 +1035,9 @@ static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
                           float2* Qp = nullptr) {
     const PlanOps* o = ctx->ops;
     float2* q = Qp ? Qp : ctx->Q;
-    if (ctx->grid_colq > 0)
+    if (ctx->grid_colg > 0)
+        o->k3g(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colg, s);
+    else if (ctx->grid_colq > 0)
         o->k3q(ctx->tmS4, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colq, s);
     else if (ctx->grid_colp > 0)
         o->k3p(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colp, s);

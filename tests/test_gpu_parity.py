@@ -335,6 +335,7 @@ def test_compute_from_host_pipelined_matches_load_then_compute():
     {"STITCH_GRAPH": "0"},                           # direct launches
     {"STITCH_CONCURRENT": "0"},                      # one stream
     {"STITCH_DUAL": "1"},                            # K3 beside K4 on two Q slots
+    {"STITCH_COLG": "1"},                            # two-group column kernels, TMA ring
     {"STITCH_ROWWARP": "0", "STITCH_COL_PERSIST": "1", "STITCH_GRAPH": "0"},
 ])
 def test_launch_variants_bit_identical(env, monkeypatch):
