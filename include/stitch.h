@@ -166,7 +166,7 @@ stitch_status stitch_forward_async(stitch_ctx* ctx);
  *   stitch_forward_range_async — step 2 for the resident tiles [first_tile, first_tile+count)
  *     (global row-major indices; INVALID_ARG if not resident);
  *   stitch_spectra_range — device address and size of the resident spectra of a tile range
- *     (phase codes, u32 [count][H][pitch]; contiguous), so the caller can send the last tile
+ *     (Q15 unit phasors F/|F|, u32 [count][H][pitch]; contiguous), so the caller can send the last tile
  *     row of its band to the next rank and receive its halo row (e.g. NCCL send/recv through
  *     torch.distributed on the workspace tensor) instead of recomputing it;
  *   stitch_pairs_async — steps 3-7 for every pair of the range, spectra already resident.

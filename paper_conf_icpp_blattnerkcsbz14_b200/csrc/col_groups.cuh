@@ -82,7 +82,7 @@ __global__ void __launch_bounds__(512, 1)   // <= 128 registers (16K per sub-par
     }
 }
 
-// K3g: NCPS from two phase panels + inverse column FFT -> Q (as K3t).
+// K3g: NCPS from two phasor panels + inverse column FFT -> Q (as K3t).
 template <class PL>
 __global__ void __launch_bounds__(512, 1)   // <= 128 registers (16K per sub-partition at 4 warps each)
     k3g_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,

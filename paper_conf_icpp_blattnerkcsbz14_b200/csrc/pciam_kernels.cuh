@@ -4,7 +4,7 @@
 //   raw   uint16 [tiles][H][W]           W contiguous (the caller's tile layout)
 //   G     float2 [chunk][H][WP]          row-transformed tiles of a forward chunk (L2-sized)
 //   spec  u32    [tiles][H][WP]          resident half spectrum kx in [0, W/2] (WP = pad16(W/2+1))
-//                                        stored as its phase code (31-bit turn + nonzero flag),
+//                                        stored as its Q15 unit phasor F/|F| (2 x int16),
 //                                        reused by <= 4 pairs
 //   Q     float2 [chunk][H][WP]          per-pair column-inverse intermediate (L2-sized chunk)
 //   keys  u64    [pairs]                 packed (|c| bits << 32 | ~index) argmax per pair
@@ -14,8 +14,8 @@
 //   K1 fwd_rows   raw -> G      R2C along x: length-W real row as a W/2 complex FFT + post-twiddle
 //                               (step 2 first half; uint16->fp32 fused into the load)
 //   K2 fwd_cols   G -> spec     C2C along y on TMA-landed column panels (step 2 second half),
-//                               epilogue: phase code
-//   K3 pair_cols  2 spec -> Q   NCPS exp(i(phi_A - phi_B)) from two TMA-landed phase panels
+//                               epilogue: Q15 unit phasor
+//   K3 pair_cols  2 spec -> Q   NCPS U_A conj(U_B) (exact int32) from two TMA-landed phasor panels
 //                               (step 3), then the inverse C2C along y (step 4 first half)
 //   K4 pair_rows  Q -> keys     C2R along x (step 4 second half) with |.| + argmax fused in the
 //                               epilogue; the real correlation surface is never stored (step 5)
@@ -62,9 +62,9 @@ struct Plan {
     using RowX = RowXchg<RI::R0, RI::R1, ROW_PAD>;
     using ColX = ColXchg<CI::R0, CI::R1, COL_PAD, COL_P>;
     static constexpr size_t ROW_SMEM = sizeof(float2) * ROW_L * RowX::LSTRIDE;
-    // column kernels: a TMA landing panel [H][COL_P] (complex, or two phase panels), reused
+    // column kernels: a TMA landing panel [H][COL_P] (complex, or two phasor panels), reused
     // in place as the stage exchange buffer once stage 1 has read it into registers
-    // K3 lands two phase panels: the second starts 128-byte aligned (TMA destination rule)
+    // K3 lands two phasor panels: the second starts 128-byte aligned (TMA destination rule)
     static constexpr size_t COL_PHASE_B = (sizeof(uint32_t) * COL_P * H + 127) / 128 * 128;
     static constexpr size_t COL_LAND_C = sizeof(float2) * COL_P * H;
     static constexpr size_t COL_LAND_P = COL_PHASE_B + sizeof(uint32_t) * COL_P * H;
@@ -170,41 +170,41 @@ struct LandSrc {  // a landed complex panel [H][COL_P] in shared memory
     __device__ __forceinline__ float2 load(int line, int n) const { return s[n * PL::COL_P + line]; }
 };
 
-// Resident spectrum code: the phase of F in 31-bit fixed point (top bits, 2^32 per turn)
-// plus a nonzero flag (bit 0).  Step 3 needs only phases: F_A conj(F_B) / |F_A conj(F_B)|
-// = exp(i (phi_A - phi_B)), and 0 where F_A or F_B vanishes (reading C4).
-// Phase code of v: atan2(v.y, v.x) / pi in [-1, 1] by octant reduction + a degree-8
-// polynomial in t^2 for atan(t)/pi on [0, 1] (coefficients fitted in double, max error
-// 1.6e-7 rad in fp32; the fp32 spectrum's own phase error is ~1e-6 rad), scaled to 2^31
-// per half turn; bit 0 = nonzero flag.  A zero v gives t = 0*inf = NaN -> an arbitrary
-// code with flag 0, which makes every NCPS product with it 0 (reading C4).
-__device__ __forceinline__ uint32_t phase_code(float2 v) {
-    const float ax = fabsf(v.x), ay = fabsf(v.y);
-    const float mx = fmaxf(ax, ay), mn = fminf(ax, ay);
-    const float t = __fdividef(mn, mx);
-    const float s = t * t;
-    float p = 0.0009368208120577037f;
-    p = fmaf(p, s, -0.00521085737273097f);
-    p = fmaf(p, s, 0.013704856857657433f);
-    p = fmaf(p, s, -0.023946231231093407f);
-    p = fmaf(p, s, 0.03387756645679474f);
-    p = fmaf(p, s, -0.045206326991319656f);
-    p = fmaf(p, s, 0.06363658607006073f);
-    p = fmaf(p, s, -0.10610226541757584f);
-    p = fmaf(p, s, 0.31830987334251404f);
-    float r = p * t;                                 // atan(mn/mx) / pi in [0, 1/4]
-    r = ay > ax ? 0.5f - r : r;
-    r = v.x < 0.f ? 1.0f - r : r;
-    r = copysignf(r, v.y);                           // [-1, 1]
-    const int32_t q = __float2int_rn(r * 2147483648.0f);   // saturates at r = 1
-    return ((uint32_t)q & ~1u) | (mx > 0.f ? 1u : 0u);
+// Resident spectrum code: the unit phasor F/|F| in Q15 fixed point, two signed 16-bit
+// fields (bits 0-15: round(32767 Re F/|F|), bits 16-31: round(32767 Im F/|F|)).  Step 3
+// needs nothing else: F_A conj(F_B) / |F_A conj(F_B)| = U_A conj(U_B) with U = F/|F|, and 0
+// where F_A or F_B vanishes (reading C4): a zero F encodes as the zero phasor, so every NCPS
+// product with it is exactly 0 without a flag.  Quantisation error <= 1.6e-5 per component
+// (|U_q| = 1 +- 5e-5, angle +- 3e-5 rad): the correlation surface changes by a relative
+// ~1e-5/sqrt(HW) at the peak, far inside the 1e-4 peak-height contract.
+// Encoder (8 instructions, no atan2): r = 32767 / |v| (rsqrt, floored argument so v = 0
+// gives r finite and both fields 0); each field is rounded by the fp32 magic-number trick --
+// fmaf(x, r, 1.5*2^23) holds round(x r) in two's complement in its low 16 mantissa bits --
+// and the two low halves are packed with one byte permute.
+__device__ __forceinline__ uint32_t phasor_q15(float2 v) {
+    const float s2 = fmaf(v.x, v.x, v.y * v.y);
+    const float r = rsqrtf(fmaxf(s2, 1e-36f)) * 32767.0f;
+    const float fx = fmaf(v.x, r, 12582912.0f);     // 1.5 * 2^23: ulp 1, round to nearest
+    const float fy = fmaf(v.y, r, 12582912.0f);
+    return __byte_perm(__float_as_uint(fx), __float_as_uint(fy), 0x5410);
 }
+// Decoder: the sign-extended fields (one PRMT in sign-replicate mode, one arithmetic shift)
+__device__ __forceinline__ int32_t q15_lo(uint32_t w) {
+    int32_t r;
+    asm("prmt.b32 %0, %1, 0, 0x9910;" : "=r"(r) : "r"(w));
+    return r;
+}
+__device__ __forceinline__ int32_t q15_hi(uint32_t w) { return (int32_t)w >> 16; }
+// NCPS scale: U_A conj(U_B) in Q15 x Q15 is 32767^2 times the unit-modulus product, formed
+// exactly in int32 (|.| <= |U_A| |U_B| < 1.08e9) and rounded once to fp32; the inverse
+// transform is linear, so the factor is carried to the reported peak height (K6).
+constexpr double NCPS_Q15_SCALE = 32767.0 * 32767.0;
 
 template <class PL>
-struct PhaseDst {  // K2 output: phase codes of a panel of the resident spectrum
+struct PhaseDst {  // K2 output: Q15 unit phasors of a panel of the resident spectrum
     uint32_t* p;
     __device__ __forceinline__ void store(int line, int n, float2 v) const {
-        p[(size_t)n * PL::WP + line] = phase_code(v);
+        p[(size_t)n * PL::WP + line] = phasor_q15(v);
     }
 };
 
@@ -295,16 +295,13 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
 
 // ------------------------------------------------------------------ K3 ----
 template <class PL>
-struct NcpsPhaseSrc {  // step 3 from two landed phase panels: exp(i (phi_A - phi_B)) or 0
+struct NcpsPhaseSrc {  // step 3 from two landed phasor panels: U_A conj(U_B) (x 32767^2)
     const uint32_t* a;
     const uint32_t* b;
     __device__ __forceinline__ float2 load(int line, int n) const {
         const uint32_t ua = a[n * PL::COL_P + line], ub = b[n * PL::COL_P + line];
-        const uint32_t d = ua - ub;   // phase difference, wraps mod one turn (flag bits cancel)
-        const float x = (float)(int32_t)d * 1.46291807926715968e-9f;   // 2 pi / 2^32, [-pi, pi)
-        float sn, cs;
-        __sincosf(x, &sn, &cs);
-        return (ua & ub & 1u) ? make_float2(cs, sn) : make_float2(0.f, 0.f);
+        const int32_t ax = q15_lo(ua), ay = q15_hi(ua), bx = q15_lo(ub), by = q15_hi(ub);
+        return make_float2((float)(ax * bx + ay * by), (float)(ay * bx - ax * by));
     }
 };
 
@@ -904,7 +901,8 @@ __device__ __forceinline__ double i128_to_double(__int128 v) {
 
 __global__ void k6_finalize(const unsigned long long* __restrict__ keys,
                             const unsigned long long* __restrict__ mom,
-                            stitch_pair* __restrict__ out, int H, int W, int npairs) {
+                            stitch_pair* __restrict__ out, int H, int W, int npairs,
+                            double peak_div) {
     const int p = blockIdx.x * blockDim.x + threadIdx.x;
     if (p >= npairs) return;
     const unsigned long long key = keys[p];
@@ -913,7 +911,8 @@ __global__ void k6_finalize(const unsigned long long* __restrict__ keys,
     stitch_pair r;
     r.peak_x = x;
     r.peak_y = y;
-    r.peak = __uint_as_float((uint32_t)(key >> 32)) / ((float)W * (float)H);
+    // peak_div = W*H (fp64 path), W*H*32767^2 (fp32 path: Q15 phasor NCPS, see phasor_q15)
+    r.peak = (float)((double)__uint_as_float((uint32_t)(key >> 32)) / peak_div);
     const int cdx[4] = {x, W - x, x, W - x};
     const int cdy[4] = {y, y, H - y, H - y};
     int best = 0;

@@ -440,7 +440,7 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : (L->prec ? 8 : 32);
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
-    // resident spectrum: u32 phase code (fp32) or double2 unit phasor (fp64)
+    // resident spectrum: u32 Q15 unit phasor (fp32) or double2 unit phasor (fp64)
     const size_t spec_el = L->prec ? sizeof(double2) : sizeof(uint32_t);
     const size_t cplx = L->prec ? sizeof(double2) : sizeof(float2);
     size_t o = 0;
@@ -483,7 +483,7 @@ struct stitch_ctx {
     char* mem = nullptr;
     bool own_mem = false;
     uint16_t* raw;
-    uint32_t* spec;                   // resident phase spectra [nlocal][H][WP]
+    uint32_t* spec;                   // resident Q15 phasor spectra [nlocal][H][WP]
     float2 *G, *Q, *twM, *twH, *twW;  // chunk intermediates, twiddles
     float2* Q2 = nullptr;             // second pair-chunk slot (dual schedule)
     int grid_k4w_dual = 0;            // K4w grid beside K3 (dual schedule)
@@ -494,7 +494,7 @@ struct stitch_ctx {
     double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
     double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
     uint32_t* part_i = nullptr;
-    CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (phase codes)
+    CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (Q15 phasors)
     CUtensorMap tmG4, tmS4;           // the same with the quad plans' 4-column boxes
     int grid_colq = 0;                // quad persistent column kernels (0: not used)
     int grid_colg = 0;                // two-group column kernels (0: not used)
@@ -838,7 +838,7 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
         const cuuint32_t boxh = (cuuint32_t)(ops->H / ((ops->H + 255) / 256));
         const cuuint32_t estr[2] = {1, 1};
-        // G: complex chunk [chunk_tiles*H][WP] as floats; spec: u32 phase codes [nlocal*H][WP]
+        // G: complex chunk [chunk_tiles*H][WP] as floats; spec: u32 Q15 phasors [nlocal*H][WP]
         auto encode_pair = [&](CUtensorMap* mg, CUtensorMap* ms, int colp) {
             const cuuint64_t gd[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
             const cuuint64_t gs[1] = {(cuuint64_t)ops->WP * 8};
@@ -997,6 +997,13 @@ stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid,
 
 // Row kernels: warp-per-line (K1w/K4w) where the plan allows, else persistent CTA rows
 // (K1p/K4p), else one CTA per row block (K1/K4).
+// K6's divisor of the argmax value: max|c| / (W H) (C5); the fp32 path's NCPS carries the
+// Q15 phasor scale 32767^2 (pciam_kernels.cuh, phasor_q15).
+static double k6_peak_div(const stitch_ctx* ctx) {
+    const double wh = (double)ctx->W * (double)ctx->H;
+    return ctx->prec ? wh : wh * NCPS_Q15_SCALE;
+}
+
 static void launch_k1_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
     const PlanOps* o = ctx->ops;
     if (ctx->grid_k1w > 0)
@@ -1112,7 +1119,8 @@ static stitch_status pairs_impl(stitch_ctx* ctx) {
             ctx->launches += 1;
         }
         k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, s>>>(ctx->keys, ctx->mom, ctx->res,
-                                                                 ctx->H, ctx->W, (int)np);
+                                                                 ctx->H, ctx->W, (int)np,
+                                                                 k6_peak_div(ctx));
         CK(mark(ctx, 5), "event");
         ctx->launches += 1;
         CK(cudaGetLastError(), "ccf launch");
@@ -1219,7 +1227,7 @@ static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_sr
     if (np > 0) {
         CK(tl_wrap(ctx, sk, 2, 5, [&] {
                k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
-                   ctx->keys, ctx->mom, ctx->res, ctx->H, ctx->W, (int)np);
+                   ctx->keys, ctx->mom, ctx->res, ctx->H, ctx->W, (int)np, k6_peak_div(ctx));
            }), "timeline");
         ctx->launches += 1;
     }
@@ -1428,7 +1436,7 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
     if (ctx->prec) return fail(ctx, STITCH_ERR_STATE, "fp64 context: use stitch_debug_spectrum_f64");
-    // The resident store keeps phase codes; recompute the complex spectrum of this tile
+    // The resident store keeps Q15 unit phasors; recompute the complex spectrum of this tile
     // with the same K1 + K2 kernels into the chunk buffer G (slot 0) and copy it out.
     const int lt = tile - ctx->L.h_begin;
     const PlanOps* o = ctx->ops;

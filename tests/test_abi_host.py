@@ -166,35 +166,65 @@ def test_generated_fp64_codelets_are_dfts():
         assert np.abs(got - ref).max() <= 1e-13 * np.abs(ref).max(), (n, tag)
 
 
-def test_phase_code_polynomial_matches_atan2():
-    """The K2 phase encoder's atan2 (octant reduction + fitted polynomial, pciam_kernels.cuh)
-    re-evaluated in float32 on the host: within 3e-7 rad of the exact angle, and the
-    NCPS decoder's wrap-around difference of two codes recovers phase differences."""
+def _q15_encode(z):
+    """Host emulation of pciam_kernels.cuh phasor_q15 (fp32 rsqrt floored at 1e-36, scale
+    32767, magic-number rounding fmaf(x, r, 1.5*2^23), low 16 bits of each field)."""
+    x, y = z.real.astype(np.float32), z.imag.astype(np.float32)
+    s2 = (x.astype(np.float64) ** 2 + y.astype(np.float64) ** 2).astype(np.float32)
+    r = (np.float32(1.0) / np.sqrt(np.maximum(s2, np.float32(1e-36)))).astype(np.float32)
+    r = (r * np.float32(32767.0)).astype(np.float32)
+    fx = (x.astype(np.float64) * r + 12582912.0).astype(np.float32)   # one rounding (ulp 1)
+    fy = (y.astype(np.float64) * r + 12582912.0).astype(np.float32)
+    lo = fx.view(np.uint32) & np.uint32(0xFFFF)
+    hi = fy.view(np.uint32) & np.uint32(0xFFFF)
+    return lo | (hi << np.uint32(16))
+
+
+def _q15_decode(w):
+    lo = (w & np.uint32(0xFFFF)).astype(np.uint16).view(np.int16).astype(np.int64)
+    hi = (w >> np.uint32(16)).astype(np.uint16).view(np.int16).astype(np.int64)
+    return lo, hi
+
+
+def test_q15_phasor_encoder_and_ncps_decoder():
+    """The K2 resident-spectrum encoder (Q15 unit phasor, pciam_kernels.cuh phasor_q15) and
+    the K3 NCPS decoder (exact int32 U_A conj(U_B)) re-evaluated on the host: the code's
+    constants and byte selectors are read from the source; each decoded field is within
+    half a Q15 step (+ rsqrt rounding) of 32767 F/|F|; a zero F is the zero phasor (reading
+    C4); the integer NCPS equals 32767^2 F_A conj(F_B)/|F_A conj(F_B)| within 1e-4; the int32
+    products cannot overflow."""
     src = open(os.path.join(ROOT, "paper_conf_icpp_blattnerkcsbz14_b200", "csrc",
                             "pciam_kernels.cuh")).read()
-    body = src[src.index("__device__ __forceinline__ uint32_t phase_code"):]
+    body = src[src.index("__device__ __forceinline__ uint32_t phasor_q15"):]
     body = body[:body.index("\n}\n")]
-    coef = [float(c) for c in re.findall(r"fmaf\(p, s, (-?\d\.\d+)f\)", body)]
-    coef = [float(re.search(r"float p = (-?\d\.\d+)f;", body).group(1))] + coef
-    assert len(coef) == 9
+    assert "1e-36f" in body and "* 32767.0f" in body and body.count("12582912.0f") == 2
+    assert "0x5410" in body
+    dec = src[src.index("int32_t q15_lo"):src.index("NCPS_Q15_SCALE")]
+    assert "0x9910" in dec and "(int32_t)w >> 16" in dec
+    assert "32767.0 * 32767.0" in src
     rng = np.random.default_rng(5)
-    z = (rng.standard_normal(200000) + 1j * rng.standard_normal(200000)).astype(np.complex64)
-    x, y = z.real.astype(np.float32), z.imag.astype(np.float32)
-    ax, ay = np.abs(x), np.abs(y)
-    mx, mn = np.maximum(ax, ay), np.minimum(ax, ay)
-    t = (mn / mx).astype(np.float32)
-    s = (t * t).astype(np.float32)
-    p = np.float32(coef[0])
-    for c in coef[1:]:
-        p = (p * s + np.float32(c)).astype(np.float32)
-    r = (p * t).astype(np.float32)
-    r = np.where(ay > ax, np.float32(0.5) - r, r)
-    r = np.where(x < 0, np.float32(1.0) - r, r)
-    r = np.copysign(r, y)
-    err = np.abs(np.angle(np.exp(1j * (np.pi * r.astype(np.float64) - np.angle(z.astype(np.complex128))))))
-    assert err.max() <= 3e-7
-    q = np.clip(np.rint(r.astype(np.float64) * 2**31), -2**31, 2**31 - 1).astype(np.int64)
-    code = (q.astype(np.uint32) & np.uint32(0xFFFFFFFE)) | np.uint32(1)
-    d = (code[:-1] - code[1:]).astype(np.uint32).view(np.int32).astype(np.float64) * (2 * np.pi / 2**32)
-    ref = np.angle(z[:-1].astype(np.complex128) * np.conj(z[1:].astype(np.complex128)))
-    assert np.abs(np.angle(np.exp(1j * (d - ref)))).max() <= 1e-6
+    z = (rng.standard_normal(200000) * 10.0 ** rng.uniform(-3, 10, 200000)
+         + 1j * rng.standard_normal(200000) * 10.0 ** rng.uniform(-3, 10, 200000)).astype(np.complex64)
+    z[:4] = [0, 1e-30, -7e10 + 1e-3j, 1j]
+    w = _q15_encode(z)
+    ax, ay = _q15_decode(w)
+    assert ax[0] == 0 and ay[0] == 0                       # zero F -> zero phasor
+    # |F| < 1e-18 (|F|^2 under the 1e-36 floor: rounding noise of a vanishing bin) encodes
+    # as a phasor shorter than unit, here exactly zero; every larger F as its unit phasor
+    assert ax[1] == 0 and ay[1] == 0
+    assert np.abs(ax).max() <= 32767 and np.abs(ay).max() <= 32767
+    keep = np.abs(z) >= 1e-17
+    keep[:2] = False
+    ax, ay, z = ax[keep], ay[keep], z[keep]
+    zz = z.astype(np.complex128)
+    u = zz / np.abs(zz) * 32767.0
+    assert np.abs(ax - u.real).max() <= 0.5 + 0.02
+    assert np.abs(ay - u.imag).max() <= 0.5 + 0.02
+    bx, by = ax[1:], ay[1:]
+    ax, ay = ax[:-1], ay[:-1]
+    re, im = ax * bx + ay * by, ay * bx - ax * by           # the K3 int32 products
+    assert max(np.abs(re).max(), np.abs(im).max()) < 2 ** 31
+    za, zb = zz[:-1], zz[1:]
+    p = za * np.conj(zb)
+    ref = p / np.abs(p) * 32767.0 ** 2
+    assert np.abs((re + 1j * im) - ref).max() <= 1e-4 * 32767.0 ** 2
