@@ -743,15 +743,18 @@ namespace stitch {
 // region a = A[dy:H, dx:W], b = B[0:H-dy, 0:W-dx].  c1 = (x, y) and c2 = (W-x, y) share
 // their rows (dy = y: A rows y.., B rows 0..H-y-1), and so do c3 = (x, H-y) and
 // c4 = (W-x, H-y) (dy = H-y).  Row group g (0: c1/c2, 1: c3/c4) is cut into blocks of
-// CCF_ROWS rows; a CTA stages CCF_BATCH rows of A and B at a time in shared memory
-// (aligned 16-byte loads: each tile row is read once for both candidates) and every
-// B pixel b = B[i][j] is paired with both of its partners
+// CCF_ROWS rows; a CTA stages CCF_BATCH rows of A and B at a time in shared memory (TMA bulk
+// copies, double-buffered: each tile row is read once for both candidates) and one warp
+// takes one staged row, pairing every B pixel b = B[i][j] with both of its partners
 //   candidate dx = x   : a = A[dy+i][x + j],      j <  W - x
 //   candidate dx = W-x : a = A[dy+i][W - x + j],  j <  x
-// accumulating the exact integer moments Sa, Sb, Saa, Sbb, Sab (u32 / u64 wide MADs).
+// two pixels per 32-bit shared load (an odd offset dx is realigned with one funnel shift),
+// accumulating the exact integer moments Sa, Sb, Saa, Sbb, Sab (u32 sums, u64 wide MADs).
 constexpr int CCF_ROWS = 64;   // rows of one group per CTA
-constexpr int CCF_BATCH = 4;   // rows staged in shared memory at a time (two warps per row)
-constexpr int CCF_T = 256;
+constexpr int CCF_BATCH = 8;   // rows staged in shared memory at a time (one warp per row)
+constexpr int CCF_T = 32 * CCF_BATCH;
+constexpr int CCF_PAD = 16;    // bytes after each staging buffer (the realigned loads of an
+                               // odd dx read one pixel past the row's end, never used)
 
 __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v) {
 #pragma unroll
@@ -759,9 +762,8 @@ __device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v)
     return v;
 }
 
-struct Moments {
-    uint32_t sa = 0, sb = 0;  // <= CCF_ROWS/CCF_BATCH * ceil(W/64) * 65535 < 2^32 per lane
-    unsigned long long saa = 0, sbb = 0, sab = 0;
+struct Moments {  // exact per-lane totals
+    unsigned long long sa = 0, sb = 0, saa = 0, sbb = 0, sab = 0;
     __device__ __forceinline__ void add(uint32_t a, uint32_t b) {
         sa += a;
         sb += b;
@@ -771,24 +773,60 @@ struct Moments {
     }
 };
 
-// Moments of one candidate over one staged row: a = ar[off + j], b = br[j], j < w.
-// The two warps of a row interleave: lane l of half h takes j = 32h + l + 64k
-// (conflict-free 2-byte shared loads), alternating two accumulator sets so the wide
-// multiply-add chains overlap.  (A single pass pairing each B pixel with both candidates
-// was measured 2x slower: the compiler predicates both candidates' bodies everywhere.)
-__device__ __forceinline__ void row_moments(Moments& m, Moments& m2, const uint16_t* ar,
-                                            const uint16_t* br, int off, int w, int j0) {
-    const uint16_t* a = ar + off + j0;
-    const uint16_t* b = br + j0;
-    const int n = w - j0;                    // this lane touches j' = 64k < n
-    int k = 0;
-    for (; k + 192 < n; k += 256) {
-        m.add(a[k], b[k]);
-        m2.add(a[k + 64], b[k + 64]);
-        m.add(a[k + 128], b[k + 128]);
-        m2.add(a[k + 192], b[k + 192]);
+// Packed-pixel moments with 16x8-bit integer dot products (IDP.2A): for words wa = (a0, a1),
+// wb = (b0, b1) of two 16-bit pixels each, one byte permute gives wb' = (b0 lo byte, b1 lo
+// byte, b0 hi byte, b1 hi byte), and dp2a_lo(wa, wb') + 256 dp2a_hi(wa, wb') = a0 b0 + a1 b1
+// exactly, so Saa, Sbb, Sab take two dot products each per pixel pair of words and Sa, Sb one
+// (against the byte vector (1, 1)), with no unpacking: 2 PRMT + 8 IDP per two pixel pairs
+// instead of 4 unpacks, 6 wide multiplies and 8 adds (the u64 accumulation made the ALU pipe
+// K5's bottleneck, ncu).  Each u32 sum grows by < 2 * 65535 * 256 = 2^25 per call, so it is
+// flushed into the exact u64 totals at most every 127 calls (flush_rows()).
+struct MomentsPk {
+    uint32_t sa = 0, sb = 0, saa_l = 0, saa_h = 0, sbb_l = 0, sbb_h = 0, sab_l = 0, sab_h = 0;
+    __device__ __forceinline__ void add2(uint32_t wa, uint32_t wb) {
+        const uint32_t pa = __byte_perm(wa, 0, 0x3120), pb = __byte_perm(wb, 0, 0x3120);
+        sa = __dp2a_lo(wa, 0x0101u, sa);
+        sb = __dp2a_lo(wb, 0x0101u, sb);
+        saa_l = __dp2a_lo(wa, pa, saa_l);
+        saa_h = __dp2a_hi(wa, pa, saa_h);
+        sbb_l = __dp2a_lo(wb, pb, sbb_l);
+        sbb_h = __dp2a_hi(wb, pb, sbb_h);
+        sab_l = __dp2a_lo(wa, pb, sab_l);
+        sab_h = __dp2a_hi(wa, pb, sab_h);
     }
-    for (; k < n; k += 64) m.add(a[k], b[k]);
+    __device__ __forceinline__ void flush(Moments& m) {
+        m.sa += sa;
+        m.sb += sb;
+        m.saa += saa_l + ((unsigned long long)saa_h << 8);
+        m.sbb += sbb_l + ((unsigned long long)sbb_h << 8);
+        m.sab += sab_l + ((unsigned long long)sab_h << 8);
+        *this = MomentsPk();
+    }
+};
+// rows a warp may accumulate between flushes: a row gives one candidate set at most
+// ceil(W/2 / 32) + 1 calls (the +1: the odd-width tail is added to the u64 totals directly)
+template <int W>
+struct CcfFlush {
+    static constexpr int CALLS = (W / 2 + 31) / 32;
+    static constexpr int ROWS = 127 / CALLS > 0 ? 127 / CALLS : 1;
+};
+
+// Moments of one candidate over one staged row: a = ar[off + j], b = br[j], j < w; lane l
+// takes the pixel pairs (2q, 2q+1), q = l + 32k; an odd w leaves pixel w-1 to lane 0.
+template <bool ODD>
+__device__ __forceinline__ void row_moments_pk(MomentsPk& m, Moments& mt, const uint16_t* ar,
+                                               const uint16_t* br, int off, int w, int lane) {
+    const uint32_t* b32 = reinterpret_cast<const uint32_t*>(br);
+    const uint32_t* a32 = reinterpret_cast<const uint32_t*>(ar + off - (ODD ? 1 : 0));
+    const int npk = w >> 1;
+#pragma unroll 2
+    for (int q = lane; q < npk; q += 32) {
+        uint32_t wa;
+        if constexpr (ODD) wa = __funnelshift_r(a32[q], a32[q + 1], 16);
+        else wa = a32[q];
+        m.add2(wa, b32[q]);
+    }
+    if ((w & 1) && lane == 0) mt.add(ar[off + w - 1], br[w - 1]);
 }
 
 template <int W, int H>
@@ -797,8 +835,10 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
                                                         const unsigned long long* __restrict__ keys,
                                                         unsigned long long* __restrict__ mom,
                                                         int pair0) {
+    static_assert(W % 2 == 0, "packed pixel pairs need an even row length");
     constexpr bool BULK = (W * 2) % 16 == 0;   // rows 16-byte aligned: TMA bulk copies
     constexpr int BUFS = BULK ? 2 : 1;
+    constexpr int BUFB = (2 * CCF_BATCH * W * 2 + CCF_PAD + 15) / 16 * 16;   // bytes per buffer
     extern __shared__ __align__(16) unsigned char ccf_smem[];
     __shared__ unsigned long long red[10][CCF_T / 32];
     __shared__ uint64_t bar[2];
@@ -816,7 +856,7 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
     const int nbatch = (rows_total + CCF_BATCH - 1) / CCF_BATCH;
     const uint16_t* A = raw + (size_t)pr.a * H * W + (size_t)(dy + i0) * W;
     const uint16_t* B = raw + (size_t)pr.b * H * W + (size_t)i0 * W;
-    auto bufA = [&](int buf) { return reinterpret_cast<uint16_t*>(ccf_smem) + buf * 2 * CCF_BATCH * W; };
+    auto bufA = [&](int buf) { return reinterpret_cast<uint16_t*>(ccf_smem + buf * BUFB); };
     auto bufB = [&](int buf) { return bufA(buf) + CCF_BATCH * W; };
     auto issue = [&](int bi) {  // TMA bulk copy of batch bi (A rows and B rows) into buffer bi&1
         const int rows = min(CCF_BATCH, rows_total - bi * CCF_BATCH);
@@ -835,9 +875,11 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
         __syncthreads();
         if (threadIdx.x == 0) issue(0);
     }
-    const int w0 = W - x, lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-    const int rrow = warp >> 1, j0 = 32 * (warp & 1) + lane;   // two warps per staged row
-    Moments m0, m1, m0b, m1b;
+    const int w0 = W - x, lane = threadIdx.x & 31, rrow = threadIdx.x >> 5;
+    const bool odd = x & 1;                    // dx = x and dx = W - x have the same parity
+    Moments m0, m1;                            // exact totals, candidates dx = x and W - x
+    MomentsPk p0, p1;                          // running packed sums
+    constexpr int FLUSH = CcfFlush<W>::ROWS;
     for (int bi = 0; bi < nbatch; ++bi) {
         const int rows = min(CCF_BATCH, rows_total - bi * CCF_BATCH);
         const int buf = bi % BUFS;
@@ -857,19 +899,28 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
             }
             __syncthreads();
         }
-        if (rrow < rows) {
+        if (rrow < rows) {                     // warp-uniform
             const uint16_t* ar = bufA(buf) + rrow * W;
             const uint16_t* br = bufB(buf) + rrow * W;
-            row_moments(m0, m0b, ar, br, x, w0, j0);   // candidate dx = x
-            row_moments(m1, m1b, ar, br, w0, x, j0);   // candidate dx = W - x
+            if (odd) {
+                row_moments_pk<true>(p0, m0, ar, br, x, w0, lane);    // candidate dx = x
+                row_moments_pk<true>(p1, m1, ar, br, w0, x, lane);    // candidate dx = W - x
+            } else {
+                row_moments_pk<false>(p0, m0, ar, br, x, w0, lane);
+                row_moments_pk<false>(p1, m1, ar, br, w0, x, lane);
+            }
+            if (bi % FLUSH == FLUSH - 1) {
+                p0.flush(m0);
+                p1.flush(m1);
+            }
         }
         __syncthreads();                       // buffer free for batch bi+2
     }
-    unsigned long long v[10] = {
-        (unsigned long long)m0.sa + m0b.sa, (unsigned long long)m0.sb + m0b.sb, m0.saa + m0b.saa,
-        m0.sbb + m0b.sbb, m0.sab + m0b.sab,
-        (unsigned long long)m1.sa + m1b.sa, (unsigned long long)m1.sb + m1b.sb, m1.saa + m1b.saa,
-        m1.sbb + m1b.sbb, m1.sab + m1b.sab};
+    p0.flush(m0);
+    p1.flush(m1);
+    unsigned long long v[10] = {m0.sa, m0.sb, m0.saa, m0.sbb, m0.sab,
+                                m1.sa, m1.sb, m1.saa, m1.sbb, m1.sab};
+    const int warp = threadIdx.x >> 5;
 #pragma unroll
     for (int q = 0; q < 10; ++q) {
         v[q] = warp_sum_u64(v[q]);
@@ -886,7 +937,8 @@ __global__ void __launch_bounds__(CCF_T) k5_ccf_moments(const uint16_t* __restri
 }
 
 inline size_t k5_smem_bytes(int W) {
-    return (size_t)((W * 2) % 16 == 0 ? 2 : 1) * 2 * CCF_BATCH * W * sizeof(uint16_t);
+    const size_t bufb = ((size_t)2 * CCF_BATCH * W * 2 + CCF_PAD + 15) / 16 * 16;
+    return (size_t)((W * 2) % 16 == 0 ? 2 : 1) * bufb;
 }
 inline int k5_grid_x(int H) { return H / CCF_ROWS + 2; }
 
