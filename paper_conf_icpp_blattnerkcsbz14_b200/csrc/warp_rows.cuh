@@ -210,7 +210,8 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
     float2* twWs = reinterpret_cast<float2*>(smem_w + RW::OFF_TWW);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     unsigned char* mine = smem_w + RW::OFF_WARP + warp * RW::WARP_K4;
-    const float2* land = reinterpret_cast<const float2*>(mine);
+    float2* landw = reinterpret_cast<float2*>(mine);
+    const float2* land = landw;
     typename RW::IFft::Xc xc{reinterpret_cast<float2*>(mine + RW::QROW)};
     uint64_t* bar = &bars[warp];
     if (lane == 0) {
@@ -247,17 +248,24 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
         }
         acc.row_base = y;
         mbar_wait(bar, k & 1);
+        // C2R pre-processing in place, one mirror pair (q, M-q) per lane and iteration (all 32
+        // lanes; the radix-R0 stage below keeps only R1 of them busy):
+        //   d = X[q] - conj X[M-q],  o = d conj(w_W^q),  Z[q] = X[q] + conj X[M-q] + i o,
+        //   Z[M-q] = conj(X[q] + conj X[M-q]) + i conj(o)      (w_W^{M-q} = -conj w_W^q)
+        // so Z (the length-M complex sequence whose inverse FFT interleaves the real row)
+        // replaces the landed Hermitian row; Z[0] pairs X[0] with X[M].
+        for (int q = lane; 2 * q <= M; q += 32) {
+            const float2 xn = landw[q], xm = landw[M - q];
+            const float2 o = cmulc(make_float2(xn.x - xm.x, xn.y + xm.y), twWs[q]);
+            const float sx = xn.x + xm.x, dy = xn.y - xm.y;
+            landw[q] = make_float2(sx - o.y, dy + o.x);
+            if (q != 0 && 2 * q != M) landw[M - q] = make_float2(sx + o.y, o.x - dy);
+        }
+        __syncwarp();
         struct Src {
-            const float2* x;
-            const float2* w;
-            __device__ __forceinline__ float2 load(int, int n) const {
-                const float2 xn = x[n];
-                const float2 xm = x[M - n];
-                const float2 d = make_float2(xn.x - xm.x, xn.y + xm.y);
-                const float2 o = cmulc(d, w[n]);
-                return make_float2(xn.x + xm.x - o.y, xn.y - xm.y + o.x);
-            }
-        } src{land, twWs};
+            const float2* z;
+            __device__ __forceinline__ float2 load(int, int n) const { return z[n]; }
+        } src{land};
         auto prefetch = [&]() {
             if (lane == 0 && r + 1 < r1) {
                 fence_proxy_async();
