@@ -8,7 +8,8 @@ import json
 import subprocess
 import sys
 
-NAMES = {"k1p_fwd": "k1_fwd_rows", "k2t_fwd": "k2_fwd_cols", "k3t_pair": "k3_pair_cols",
+NAMES = {"k1p_fwd": "k1_fwd_rows", "k1w_fwd": "k1_fwd_rows", "k2t_fwd": "k2_fwd_cols",
+         "k3t_pair": "k3_pair_cols", "k4w_pair": "k4_pair_rows",
          "k4p_pair": "k4_pair_rows", "k5_ccf": "k5_ccf_moments"}
 MUL = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-9, "usecond": 1e-6,
        "msecond": 1e-3, "ns": 1e-9, "us": 1e-6, "ms": 1e-3}
