@@ -751,7 +751,7 @@ namespace stitch {
 // two pixels per 32-bit shared load (an odd offset dx is realigned with one funnel shift),
 // accumulating the exact integer moments Sa, Sb, Saa, Sbb, Sab (u32 sums, u64 wide MADs).
 constexpr int CCF_ROWS = 64;   // rows of one group per CTA
-constexpr int CCF_BATCH = 8;   // rows staged in shared memory at a time (one warp per row)
+constexpr int CCF_BATCH = 4;   // rows staged in shared memory at a time (one warp per row)
 constexpr int CCF_T = 32 * CCF_BATCH;
 constexpr int CCF_PAD = 16;    // bytes after each staging buffer (the realigned loads of an
                                // odd dx read one pixel past the row's end, never used)
