@@ -80,7 +80,7 @@ def test_workspace_size_matches_layout(lib):
     ws = pkg.workspace_size(cfg)
     H, W, WP = 1040, 1392, 704
     raw = 2478 * H * W * 2
-    spec = 2478 * H * WP * 4          # resident phase codes (u32)
+    spec = 2478 * H * WP * 4          # resident Q15 unit phasors (u32)
     chunks = 2 * 8 * H * WP * 8       # G (forward chunk) + Q (pair chunk), complex (8 each)
     assert raw + spec + chunks < ws < raw + spec + chunks + 5 * 2**20
 
