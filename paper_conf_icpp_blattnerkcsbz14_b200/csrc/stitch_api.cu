@@ -995,8 +995,6 @@ stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid,
     return load_common(ctx, dev_grid, n_bytes, cudaMemcpyDeviceToDevice);
 }
 
-// Row kernels: warp-per-line (K1w/K4w) where the plan allows, else persistent CTA rows
-// (K1p/K4p), else one CTA per row block (K1/K4).
 // K6's divisor of the argmax value: max|c| / (W H) (C5); the fp32 path's NCPS carries the
 // Q15 phasor scale 32767^2 (pciam_kernels.cuh, phasor_q15).
 static double k6_peak_div(const stitch_ctx* ctx) {
@@ -1004,6 +1002,8 @@ static double k6_peak_div(const stitch_ctx* ctx) {
     return ctx->prec ? wh : wh * NCPS_Q15_SCALE;
 }
 
+// Row kernels: warp-per-line (K1w/K4w) where the plan allows, else
+// persistent CTA rows (K1p/K4p), else one CTA per row block (K1/K4).
 static void launch_k1_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
     const PlanOps* o = ctx->ops;
     if (ctx->grid_k1w > 0)
