@@ -4,7 +4,8 @@
 Each codelet computes, in registers, an unnormalised length-R DFT
     X[k] = sum_j x[j] exp(SIGN * 2 pi i j k / R),   SIGN = -1 (forward) or +1 (inverse)
 in place on a float2[R] array.  Primes use the symmetric (x_j +- x_{R-j}) form,
-composites a Cooley-Tukey split R = R1*R2 with constant twiddles (trivial ones --
+composites a split R = R1*R2: prime-factor (Good-Thomas, index maps only, no twiddles)
+when R1 and R2 are coprime, else Cooley-Tukey with constant twiddles (trivial ones --
 multiples of pi/4 -- special-cased).  Constants are computed in double here and
 rounded once to float literals (fp32) or kept as double literals (fp64 path, f2: the same
 straight-line program with every float replaced by double).
@@ -98,8 +99,9 @@ _FORCE = {}
 
 
 def split(n):
-    """Cooley-Tukey split n = n1 * n2 of a composite radix, chosen (recursively, memoised)
-    to minimise the straight-line instruction count; None for a prime."""
+    """Split n = n1 * n2 of a composite radix (prime-factor / Good-Thomas when the factors
+    are coprime, Cooley-Tukey with twiddles otherwise), chosen (recursively, memoised) to
+    minimise the straight-line instruction count; None for a prime."""
     if n in _FORCE:
         return _FORCE[n]
     divs = [d for d in range(2, n) if n % d == 0]
@@ -222,6 +224,19 @@ def gen(e, xs, sign):
                 out[n - k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
         return out
     n1, n2 = sp
+    if math.gcd(n1, n2) == 1:
+        # Good-Thomas prime-factor split: no twiddles.  Input map (Ruritanian)
+        # j = (n2*a + n1*b) mod n, output map (CRT) k = (n2*u*k1 + n1*w*k2) mod n with
+        # u = n2^-1 mod n1, w = n1^-1 mod n2, so that exp(2 pi i j k / n) =
+        # exp(2 pi i a k1 / n1) exp(2 pi i b k2 / n2): a 2-D DFT with no cross term.
+        u, w = pow(n2, -1, n1), pow(n1, -1, n2)
+        Y = [gen(e, [xs[(n2 * a + n1 * b) % n] for a in range(n1)], sign) for b in range(n2)]
+        out = [None] * n
+        for k1 in range(n1):
+            X = gen(e, [Y[b][k1] for b in range(n2)], sign)
+            for k2 in range(n2):
+                out[(n2 * u * k1 + n1 * w * k2) % n] = X[k2]
+        return out
     # x index j = n2*a + b ; X index k = k1 + n1*k2
     Z = []
     for b in range(n2):
