@@ -158,17 +158,35 @@ def prime_rader(e, xs, sign):
                     e.let(f"fmaf({um[a]}, {flit(c)}, {nn})")
             A[b][comp] = e.let(f"{pp} + {nn}")
             A[b + q][comp] = e.let(f"{pp} - {nn}")
+    # Sine half: B = T d with T[b][a] = S(a - b), S(m) = sin(2 pi g^m / p), S(m + h) = -S(m).
+    # In q x q blocks T = [[A, C], [-C, A]] (A = S(a0 - b0), C = S(a0 - b0 + q)), i.e. the
+    # product (A - iC)(u + iv) of the halves u, v of d; three block products, two of them
+    # started from the previous result so the block sums cost no separate adds:
+    #   t1 = A u,  y0 = C v + t1,  y1 = (A - C)(u + v) + (y0 - 2 t1)  [= A v - C u].
+    def S(m):
+        return math.sin(2.0 * math.pi * pow(g, m % (n - 1), n) / n)
+    Bv = [[None, None] for _ in range(h)]
+    for comp in (0, 1):
+        u = [d[a][comp] for a in range(q)]
+        v = [d[a + q][comp] for a in range(q)]
+        uv = [e.let(f"{u[a]} + {v[a]}") for a in range(q)]
+        for b in range(q):
+            t1 = None
+            for a in range(q):
+                c = S(a - b)
+                t1 = e.let(f"{u[a]} * {flit(c)}") if t1 is None else \
+                    e.let(f"fmaf({u[a]}, {flit(c)}, {t1})")
+            y0 = t1
+            for a in range(q):
+                y0 = e.let(f"fmaf({v[a]}, {flit(S(a - b + q))}, {y0})")
+            y1 = e.let(f"fmaf({t1}, {flit(-2.0)}, {y0})")
+            for a in range(q):
+                y1 = e.let(f"fmaf({uv[a]}, {flit(S(a - b) - S(a - b + q))}, {y1})")
+            Bv[b][comp] = y0
+            Bv[b + q][comp] = y1
     for b in range(h):
         k = kb[b]
-        br = bi = None
-        for a in range(h):
-            sn = math.sin(2.0 * math.pi * ((ja[a] * k) % n) / n)
-            if br is None:
-                br = e.let(f"{d[a][0]} * {flit(sn)}")
-                bi = e.let(f"{d[a][1]} * {flit(sn)}")
-            else:
-                br = e.let(f"fmaf({d[a][0]}, {flit(sn)}, {br})")
-                bi = e.let(f"fmaf({d[a][1]}, {flit(sn)}, {bi})")
+        br, bi = Bv[b]
         ar, ai = A[b]
         if sign < 0:
             out[k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
@@ -203,6 +221,18 @@ def gen(e, xs, sign):
         for k in range(1, h + 1):
             ar, ai = xs[0]
             br, bi = None, None
+            if h == 1:                 # n = 3: the single sine product fused into the outputs
+                m = k % n
+                c = math.cos(2.0 * math.pi * m / n)
+                sn = math.sin(2.0 * math.pi * m / n) * (1 if sign < 0 else -1)
+                ar = e.let(f"fmaf({s[1][0]}, {flit(c)}, {ar})")
+                ai = e.let(f"fmaf({s[1][1]}, {flit(c)}, {ai})")
+                # X_k = A + sign i B, B = sn d:  (ar + sn d.im, ai - sn d.re) for sign < 0
+                out[k] = (e.let(f"fmaf({d[1][1]}, {flit(sn)}, {ar})"),
+                          e.let(f"fmaf({d[1][0]}, {flit(-sn)}, {ai})"))
+                out[n - k] = (e.let(f"fmaf({d[1][1]}, {flit(-sn)}, {ar})"),
+                              e.let(f"fmaf({d[1][0]}, {flit(sn)}, {ai})"))
+                continue
             for j in range(1, h + 1):
                 m = (j * k) % n
                 c = math.cos(2.0 * math.pi * m / n)
