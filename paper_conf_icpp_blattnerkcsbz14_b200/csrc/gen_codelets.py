@@ -133,31 +133,30 @@ def prime_rader(e, xs, sign):
     kb = [pow(g, (n - 1 - b) % (n - 1), n) for b in range(h)]  # g^-b
     s = [cadd(e, xs[j], xs[n - j]) for j in ja]
     d = [csub(e, xs[j], xs[n - j]) for j in ja]
-    acc = xs[0]
-    for a in range(h):
-        acc = cadd(e, acc, s[a])
-    out = [None] * n
-    out[0] = acc
     q = h // 2
+    up = [[e.let(f"{s[a][c]} + {s[a + q][c]}") for a in range(q)] for c in (0, 1)]
+    um = [[e.let(f"{s[a][c]} - {s[a + q][c]}") for a in range(q)] for c in (0, 1)]
+    out = [None] * n
+    acc = xs[0]                        # X_0 = x_0 + sum of the q pair sums up_a
+    for a in range(q):
+        acc = (e.let(f"{acc[0]} + {up[0][a]}"), e.let(f"{acc[1]} + {up[1][a]}"))
+    out[0] = acc
     C = [math.cos(2.0 * math.pi * pow(g, m, n) / n) for m in range(h)]
     P = [0.5 * (C[m] + C[(m + q) % h]) for m in range(q)]    # period q
     Nm = [0.5 * (C[m] - C[(m + q) % h]) for m in range(h)]   # anti-periodic (q), index mod h
     A = [[None, None] for _ in range(h)]
     for comp in (0, 1):
-        up = [e.let(f"{s[a][comp]} + {s[a + q][comp]}") for a in range(q)]
-        um = [e.let(f"{s[a][comp]} - {s[a + q][comp]}") for a in range(q)]
         for b in range(q):
             pp = xs[0][comp]
             for a in range(q):
-                pp = e.let(f"fmaf({up[a]}, {flit(P[(a - b) % q])}, {pp})")
-            nn = None
+                pp = e.let(f"fmaf({up[comp][a]}, {flit(P[(a - b) % q])}, {pp})")
+            ap = pp                            # A_b = pp + nn, the nn chain started from pp
             for a in range(q):
                 m = a - b                      # N_{a-b}: N_{m+q} = -N_m
                 c = Nm[m] if m >= 0 else -Nm[m + q]
-                nn = e.let(f"{um[a]} * {flit(c)}") if nn is None else \
-                    e.let(f"fmaf({um[a]}, {flit(c)}, {nn})")
-            A[b][comp] = e.let(f"{pp} + {nn}")
-            A[b + q][comp] = e.let(f"{pp} - {nn}")
+                ap = e.let(f"fmaf({um[comp][a]}, {flit(c)}, {ap})")
+            A[b][comp] = ap
+            A[b + q][comp] = e.let(f"fmaf({pp}, {flit(2.0)}, -{ap})")   # pp - nn
     # Sine half: B = T d with T[b][a] = S(a - b), S(m) = sin(2 pi g^m / p), S(m + h) = -S(m).
     # In q x q blocks T = [[A, C], [-C, A]] (A = S(a0 - b0), C = S(a0 - b0 + q)), i.e. the
     # product (A - iC)(u + iv) of the halves u, v of d; three block products, two of them
