@@ -91,7 +91,9 @@ def _cost(n, sp):
         gen(e, xs, -1)
     finally:
         del _FORCE[n]
-    return sum(1 + l.count(" * ") * ("fmaf(" in l) for l in e.lines
+    # one instruction per line; a product inside an fmaf argument and a scaled sum
+    # "h * (a +- b)" (an add and a multiply) count one more
+    return sum(1 + l.count(" * ") * ("fmaf(" in l) + (" * (" in l) for l in e.lines
                if not (l.count("= -t") and l.count("t") == 2))
 
 
@@ -233,24 +235,24 @@ def gen(e, xs, sign):
                               e.let(f"fmaf({d[1][0]}, {flit(sn)}, {ai})"))
                 continue
             for j in range(1, h + 1):
-                m = (j * k) % n
-                c = math.cos(2.0 * math.pi * m / n)
-                sn = math.sin(2.0 * math.pi * m / n)
+                c = math.cos(2.0 * math.pi * ((j * k) % n) / n)
                 ar = e.let(f"fmaf({s[j][0]}, {flit(c)}, {ar})")
                 ai = e.let(f"fmaf({s[j][1]}, {flit(c)}, {ai})")
-                if br is None:
-                    br = e.let(f"{d[j][0]} * {flit(sn)}")
-                    bi = e.let(f"{d[j][1]} * {flit(sn)}")
-                else:
-                    br = e.let(f"fmaf({d[j][0]}, {flit(sn)}, {br})")
-                    bi = e.let(f"fmaf({d[j][1]}, {flit(sn)}, {bi})")
-            # X_k = A + sign*i*B ; X_{n-k} = A - sign*i*B ; i*B = (-bi, br)
-            if sign < 0:
-                out[k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
-                out[n - k] = (e.let(f"{ar} - {bi}"), e.let(f"{ai} + {br}"))
-            else:
-                out[k] = (e.let(f"{ar} - {bi}"), e.let(f"{ai} + {br}"))
-                out[n - k] = (e.let(f"{ar} + {bi}"), e.let(f"{ai} - {br}"))
+            # B = sum_j sn_j d_j = sn_0 * (d_j0 + sum_{j != j0} (sn_j / sn_j0) d_j), j0 the
+            # largest |sn_j|: the inner sum starts from d_j0 and the common factor goes into
+            # the two output FMAs (X_k = A + sign i B, X_{n-k} = A - sign i B, i B = (-B.im, B.re))
+            sn = [None] + [math.sin(2.0 * math.pi * ((j * k) % n) / n) for j in range(1, h + 1)]
+            j0 = max(range(1, h + 1), key=lambda j: abs(sn[j]))
+            ir, ii = d[j0]
+            for j in range(1, h + 1):
+                if j != j0:
+                    r = sn[j] / sn[j0]
+                    ir = e.let(f"fmaf({d[j][0]}, {flit(r)}, {ir})")
+                    ii = e.let(f"fmaf({d[j][1]}, {flit(r)}, {ii})")
+            f = sn[j0] if sign < 0 else -sn[j0]
+            out[k] = (e.let(f"fmaf({ii}, {flit(f)}, {ar})"), e.let(f"fmaf({ir}, {flit(-f)}, {ai})"))
+            out[n - k] = (e.let(f"fmaf({ii}, {flit(-f)}, {ar})"),
+                          e.let(f"fmaf({ir}, {flit(f)}, {ai})"))
         return out
     n1, n2 = sp
     if math.gcd(n1, n2) == 1:
@@ -267,16 +269,35 @@ def gen(e, xs, sign):
                 out[(n2 * u * k1 + n1 * w * k2) % n] = X[k2]
         return out
     # x index j = n2*a + b ; X index k = k1 + n1*k2
-    Z = []
-    for b in range(n2):
-        Y = gen(e, [xs[n2 * a + b] for a in range(n1)], sign)
-        Z.append([twiddle(e, Y[k1], b * k1, n, sign) for k1 in range(n1)])
+    Y = [gen(e, [xs[n2 * a + b] for a in range(n1)], sign) for b in range(n2)]
     out = [None] * n
     for k1 in range(n1):
-        X = gen(e, [Z[b][k1] for b in range(n2)], sign)
+        if n2 == 2 and pi4_twiddle(k1, n):
+            # outer radix 2 after a (+-1 +- i)/sqrt2 twiddle: X = Y0 +- h t with t the
+            # unscaled rotation of Y1 (two adds), the scale h folded into the output FMAs
+            y0, y1 = Y[0][k1], Y[1][k1]
+            ang = sign * 2.0 * math.pi * k1 / n
+            cs, ss = (1 if math.cos(ang) > 0 else -1), (1 if math.sin(ang) > 0 else -1)
+            tr = e.let(f"{'' if cs > 0 else '-'}{y1[0]} {'-' if ss > 0 else '+'} {y1[1]}")
+            ti = e.let(f"{'' if ss > 0 else '-'}{y1[0]} {'+' if cs > 0 else '-'} {y1[1]}")
+            h = flit(math.sqrt(0.5))
+            hm = flit(-math.sqrt(0.5))
+            out[k1] = (e.let(f"fmaf({tr}, {h}, {y0[0]})"), e.let(f"fmaf({ti}, {h}, {y0[1]})"))
+            out[k1 + n1] = (e.let(f"fmaf({tr}, {hm}, {y0[0]})"), e.let(f"fmaf({ti}, {hm}, {y0[1]})"))
+            continue
+        X = gen(e, [twiddle(e, Y[b][k1], b * k1, n, sign) for b in range(n2)], sign)
         for k2 in range(n2):
             out[k1 + n1 * k2] = X[k2]
     return out
+
+
+def pi4_twiddle(num, den):
+    """exp(+-2 pi i num/den) is an odd multiple of pi/4."""
+    num %= den
+    if num == 0:
+        return False
+    g = math.gcd(num, den)
+    return den // g == 8
 
 
 def codelet(n, sign):
