@@ -102,6 +102,16 @@ cudaError_t max_smem(K* kernel, size_t bytes) {
                                 (int)cudaSharedmemCarveoutMaxShared);
 }
 
+// K4w runs the prime-factor row transform where the radices are coprime, unless STITCH_PFA=0
+inline bool pfa_enabled() {   // read per launch (launch sequences are captured once per ctx)
+    const char* env = std::getenv("STITCH_PFA");
+    return !(env && env[0] == '0');
+}
+template <class PL>
+constexpr bool k4_pfa_ok() {
+    if constexpr (RowWarp<PL>::OK) return RowWarp<PL>::RI::STAGES == 2 && WarpFftPfa<typename PL::Row, 1>::OK && RowWarp<PL>::PAD == 0;
+    else return false;
+}
 template <class PL>
 cudaError_t plan_setup(int* grid_k1p, int* grid_k4p, int* grid_k1w, int* grid_k4w) {
     cudaError_t e;
@@ -132,6 +142,8 @@ cudaError_t plan_setup(int* grid_k1p, int* grid_k4p, int* grid_k1w, int* grid_k4
         using RW = RowWarp<PL>;
         if ((e = max_smem(k1w_fwd_rows<PL>, RW::SMEM_K1)) != cudaSuccess) return e;
         if ((e = max_smem(k4w_pair_rows<PL>, RW::SMEM_K4)) != cudaSuccess) return e;
+        if constexpr (k4_pfa_ok<PL>())
+            if ((e = max_smem(k4w_pair_rows<PL, true>, RW::SMEM_K4)) != cudaSuccess) return e;
         if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1w_fwd_rows<PL>,
                                                                 32 * ROWW_WARPS, RW::SMEM_K1)) !=
             cudaSuccess)
@@ -224,6 +236,14 @@ void launch_k1w(const uint16_t* raw, float2* G, int t0, int nt, const float2* tw
 template <class PL>
 void launch_k4w(const float2* Q, unsigned long long* keys, int p0, int np, const float2* tw2,
                 const float2* twW, int grid, cudaStream_t s) {
+    if constexpr (k4_pfa_ok<PL>()) {
+        if (pfa_enabled()) {
+            const int need = (np * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
+            k4w_pair_rows<PL, true><<<grid < need ? grid : need, 32 * ROWW_WARPS,
+                                      RowWarp<PL>::SMEM_K4, s>>>(Q, keys, p0, np, tw2, twW);
+            return;
+        }
+    }
     if constexpr (RowWarp<PL>::OK) {
         const int need = (np * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
         k4w_pair_rows<PL><<<grid < need ? grid : need, 32 * ROWW_WARPS, RowWarp<PL>::SMEM_K4, s>>>(

@@ -11,6 +11,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 #include "async_copy.cuh"
 #include "fft_engine.cuh"
 
@@ -61,6 +63,55 @@ struct WarpFft2<Radix<N, R0, R1>, SIGN, PAD> {
             for (int j = 1; j < R1; ++j) v[j] = SIGN < 0 ? cmul(v[j], tw[j - 1]) : cmulc(v[j], tw[j - 1]);
             Dft<R1, SIGN>::run(v);
             store_butterfly<R1, R0>(dst, 0, lane, v);
+        }
+    }
+};
+
+// Prime-factor (Good-Thomas) variant for coprime radices (696 = 29 x 24): no twiddles between
+// the stages, only index maps --
+//   stage-1 input  n = (R1 a + R0 b) mod M   (a < R0: element of butterfly b < R1)
+//   stage-2 output k = (C1 k1 + C2 k2) mod M, C1 = R1 (R1^-1 mod R0), C2 = R0 (R0^-1 mod R1)
+// (k1 < R0: the stage-2 butterfly, k2 < R1: its output).  The input map wraps once per
+// butterfly, at a lane-dependent a, so each load picks one of two base pointers; the
+// destination receives whole butterflies (store_pfa) and maps indices itself.
+__host__ __device__ constexpr int modinv(int a, int m) {
+    int r = 1;
+    for (int x = 1; x < m; ++x)
+        if ((a * x) % m == 1) r = x;
+    return r;
+}
+__host__ __device__ constexpr int gcd_c(int a, int b) { return b == 0 ? a : gcd_c(b, a % b); }
+
+template <class RX, int SIGN>
+struct WarpFftPfa;
+
+template <int N, int R0, int R1, int SIGN>
+struct WarpFftPfa<Radix<N, R0, R1>, SIGN> {
+    static constexpr bool OK = gcd_c(R0, R1) == 1 && R0 <= 32 && R1 <= 32;
+    static constexpr int C1 = (R1 * modinv(R1 % R0, R0)) % N;
+    static constexpr int C2 = (R0 * modinv(R0 % R1, R1)) % N;
+    template <class Xc, class Dst, class Mid>
+    static __device__ __forceinline__ void run(const float2* z, const Xc& xc, Dst& dst, int lane,
+                                               const Mid& mid) {
+        if (lane < R1) {                       // stage 1: radix R0, butterfly b = lane
+            const float2* p1 = z + R0 * lane;  // n = R0 b + R1 a, minus N once it passes N
+            const float2* p2 = p1 - N;
+            const int aw = (N - R0 * lane + R1 - 1) / R1;
+            float2 v[R0];
+#pragma unroll
+            for (int a = 0; a < R0; ++a) v[a] = (a < aw ? p1 : p2)[a * R1];
+            Dft<R0, SIGN>::run(v);
+#pragma unroll
+            for (int a = 0; a < R0; ++a) xc.at(a, lane) = v[a];
+        }
+        __syncwarp();
+        mid();
+        if (lane < R0) {                       // stage 2: radix R1, butterfly k1 = lane
+            float2 v[R1];
+#pragma unroll
+            for (int j = 0; j < R1; ++j) v[j] = xc.at(lane, j);
+            Dft<R1, SIGN>::run(v);
+            dst.store_pfa(lane, v);
         }
     }
 };
@@ -198,7 +249,41 @@ struct WarpArgmaxDst {
     }
 };
 
-template <class PL>
+// K4w's argmax for the prime-factor transform: as WarpArgmaxDst, with the output index of
+// element k2 of butterfly k1 given by the CRT map (looked up only when a row beats the best).
+template <int NLANES, int R1, int C1, int C2, int N>
+struct WarpArgmaxPfa {
+    float best_v;
+    uint32_t best_i;
+    int row_base, W;
+    static constexpr unsigned MASK = NLANES >= 32 ? 0xFFFFFFFFu : ((1u << NLANES) - 1u);
+    __device__ __forceinline__ void store_pfa(int k1, const float2 (&v)[R1]) {
+        float m = fmaxf(fabsf(v[0].x), fabsf(v[0].y));
+#pragma unroll
+        for (int j = 1; j < R1; ++j) m = fmaxf(m, fmaxf(fabsf(v[j].x), fabsf(v[j].y)));
+        const float M = __uint_as_float(__reduce_max_sync(MASK, __float_as_uint(m)));
+        if (M > best_v) {                      // warp-uniform
+            uint32_t idx = 0xFFFFFFFFu;
+            if (m == M) {
+                const uint32_t base = (uint32_t)row_base * W;
+                uint32_t n = (uint32_t)((C1 * k1) % N);
+#pragma unroll
+                for (int j = 0; j < R1; ++j) {
+                    if (fabsf(v[j].x) == M) idx = min(idx, base + 2 * n);
+                    if (fabsf(v[j].y) == M) idx = min(idx, base + 2 * n + 1);
+                    n += C2;
+                    if (n >= (uint32_t)N) n -= N;
+                }
+            }
+            best_i = __reduce_min_sync(MASK, idx);
+            best_v = M;
+        }
+    }
+};
+
+// PFA: the prime-factor row transform (WarpFftPfa + WarpArgmaxPfa) where the radices are
+// coprime; otherwise Stockham with stage-2 twiddles (WarpFft2 + WarpArgmaxDst).
+template <class PL, bool PFA = false>
 __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
     k4w_pair_rows(const float2* __restrict__ Q, unsigned long long* __restrict__ keys, int pair0,
                   int npairs, const float2* __restrict__ tw2, const float2* __restrict__ twW) {
@@ -235,7 +320,11 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
         if (lane == 0) atomicMax(&keys[pair0 + pair], key);
     };
     if (lane == 0 && r0 < r1) issue(r0);
-    WarpArgmaxDst<RW::RI::R0> acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
+    using Pfa = WarpFftPfa<typename PL::Row, +1>;
+    using Acc = std::conditional_t<PFA,
+                                   WarpArgmaxPfa<RW::RI::R0, RW::RI::R1, Pfa::C1, Pfa::C2, PL::M>,
+                                   WarpArgmaxDst<RW::RI::R0>>;
+    Acc acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
     int cur = r0 < r1 ? r0 / H : -1;
     int k = 0;
     for (int r = r0; r < r1; ++r, ++k) {
@@ -272,7 +361,10 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
                 issue(r + 1);
             }
         };
-        RW::IFft::run(src, xc, acc, tw2s, lane, prefetch);
+        if constexpr (PFA)
+            Pfa::run(land, xc, acc, lane, prefetch);
+        else
+            RW::IFft::run(src, xc, acc, tw2s, lane, prefetch);
         __syncwarp();                          // exchange free for the next row
     }
     if (cur >= 0) flush(cur, acc.best_v, acc.best_i);

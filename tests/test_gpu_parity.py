@@ -330,6 +330,7 @@ def test_compute_from_host_pipelined_matches_load_then_compute():
 
 @pytest.mark.parametrize("env", [
     {"STITCH_ROWWARP": "0"},                         # CTA row kernels (K1p/K4p)
+    {"STITCH_PFA": "0"},                             # K4w Stockham + twiddles (not prime-factor)
     {"STITCH_COL_PERSIST": "1"},                     # persistent column kernels (K2p/K3p)
     {"STITCH_COLQ": "1"},                            # quad column plans (4-column panels)
     {"STITCH_GRAPH": "0"},                           # direct launches
@@ -341,7 +342,11 @@ def test_compute_from_host_pipelined_matches_load_then_compute():
 def test_launch_variants_bit_identical(env, monkeypatch):
     """Every measured kernel / schedule variant (selected by environment at
     stitch_init) gives bit-identical results to the default path, on the 256x192 plan and on
-    the headline 1392x1040 plan."""
+    the headline 1392x1040 plan -- except the peak height where a variant evaluates the inverse
+    row transform with another factorisation (the default K4w prime-factor transform at
+    1392x1040 against Stockham + twiddles: STITCH_ROWWARP=0, STITCH_PFA=0): the correlation
+    surface then differs by rounding, so the peak height agrees to 1e-5 and everything else
+    (location, translation, candidate, CCF) is bit-identical."""
     for n, m, H, W, seed in [(3, 4, 192, 256, 61), (2, 3, 1040, 1392, 62)]:
         g = synthgrid.make_grid(n, m, H, W, seed=seed)
         ref = run_gpu(g.tiles, chunk_pairs=4, chunk_tiles=3)
@@ -350,4 +355,12 @@ def test_launch_variants_bit_identical(env, monkeypatch):
         got = run_gpu(g.tiles, chunk_pairs=4, chunk_tiles=3)
         for k in env:
             monkeypatch.delenv(k)
-        assert got[0].tobytes() == ref[0].tobytes() and got[1].tobytes() == ref[1].tobytes()
+        if W == 1392 and ("STITCH_ROWWARP" in env or "STITCH_PFA" in env):
+            for a, b in ((got[0], ref[0]), (got[1], ref[1])):
+                np.testing.assert_allclose(a["peak"], b["peak"], rtol=1e-5)
+                a, b = a.copy(), b.copy()
+                a["peak"] = 0
+                b["peak"] = 0
+                assert a.tobytes() == b.tobytes()
+        else:
+            assert got[0].tobytes() == ref[0].tobytes() and got[1].tobytes() == ref[1].tobytes()
