@@ -177,13 +177,13 @@ struct LandSrc {  // a landed complex panel [H][COL_P] in shared memory
 // product with it is exactly 0 without a flag.  Quantisation error <= 1.6e-5 per component
 // (|U_q| = 1 +- 5e-5, angle +- 3e-5 rad): the correlation surface changes by a relative
 // ~1e-5/sqrt(HW) at the peak, far inside the 1e-4 peak-height contract.
-// Encoder (8 instructions, no atan2): r = 32767 / |v| (rsqrt, floored argument so v = 0
+// Encoder (7 instructions, no atan2): r = 32767 / |v| (rsqrt, argument + 1e-36 so v = 0
 // gives r finite and both fields 0); each field is rounded by the fp32 magic-number trick --
 // fmaf(x, r, 1.5*2^23) holds round(x r) in two's complement in its low 16 mantissa bits --
 // and the two low halves are packed with one byte permute.
 __device__ __forceinline__ uint32_t phasor_q15(float2 v) {
-    const float s2 = fmaf(v.x, v.x, v.y * v.y);
-    const float r = rsqrtf(fmaxf(s2, 1e-36f)) * 32767.0f;
+    const float s2 = fmaf(v.x, v.x, fmaf(v.y, v.y, 1e-36f));   // floored: v = 0 -> finite r
+    const float r = rsqrtf(s2) * 32767.0f;
     const float fx = fmaf(v.x, r, 12582912.0f);     // 1.5 * 2^23: ulp 1, round to nearest
     const float fy = fmaf(v.y, r, 12582912.0f);
     return __byte_perm(__float_as_uint(fx), __float_as_uint(fy), 0x5410);

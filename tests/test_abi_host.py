@@ -167,11 +167,11 @@ def test_generated_fp64_codelets_are_dfts():
 
 
 def _q15_encode(z):
-    """Host emulation of pciam_kernels.cuh phasor_q15 (fp32 rsqrt floored at 1e-36, scale
+    """Host emulation of pciam_kernels.cuh phasor_q15 (fp32 rsqrt of |v|^2 + 1e-36, scale
     32767, magic-number rounding fmaf(x, r, 1.5*2^23), low 16 bits of each field)."""
     x, y = z.real.astype(np.float32), z.imag.astype(np.float32)
-    s2 = (x.astype(np.float64) ** 2 + y.astype(np.float64) ** 2).astype(np.float32)
-    r = (np.float32(1.0) / np.sqrt(np.maximum(s2, np.float32(1e-36)))).astype(np.float32)
+    s2 = (x.astype(np.float64) ** 2 + y.astype(np.float64) ** 2 + 1e-36).astype(np.float32)
+    r = (np.float32(1.0) / np.sqrt(s2)).astype(np.float32)
     r = (r * np.float32(32767.0)).astype(np.float32)
     fx = (x.astype(np.float64) * r + 12582912.0).astype(np.float32)   # one rounding (ulp 1)
     fy = (y.astype(np.float64) * r + 12582912.0).astype(np.float32)
@@ -197,7 +197,7 @@ def test_q15_phasor_encoder_and_ncps_decoder():
                             "pciam_kernels.cuh")).read()
     body = src[src.index("__device__ __forceinline__ uint32_t phasor_q15"):]
     body = body[:body.index("\n}\n")]
-    assert "1e-36f" in body and "* 32767.0f" in body and body.count("12582912.0f") == 2
+    assert "1e-36f)" in body and "* 32767.0f" in body and body.count("12582912.0f") == 2
     assert "0x5410" in body
     dec = src[src.index("int32_t q15_lo"):src.index("NCPS_Q15_SCALE")]
     assert "0x9910" in dec and "(int32_t)w >> 16" in dec
