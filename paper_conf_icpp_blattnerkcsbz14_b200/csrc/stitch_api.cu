@@ -900,12 +900,17 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     // Processing order (results do not depend on it): tiles in bands of PAIR_BAND tile
     // rows, column-major inside a band, so a tile's spectrum and raw pixels are reused by
     // its <= 4 pairs while still in L2 (the paper's traversal-order idea).
-    constexpr int PAIR_BAND = 8;
+    // 4 rows: a tile's west-pair reuse 8 pairs (~90 MB of panels and Q) after its first use
+    // stays in the 126 MB L2 (bands of 1-8 measured: 3-4 best, K3 10.81 -> 10.63 ms), and the
+    // first pair chunk waits for 4 tile rows of forward transforms instead of 8.
+    // STITCH_PAIR_BAND overrides (experiments).
+    int PAIR_BAND = 4;
+    if (const char* benv = std::getenv("STITCH_PAIR_BAND")) PAIR_BAND = std::max(1, std::atoi(benv));
     std::vector<int> order;
     order.reserve((size_t)(L.t_end - L.t_begin));
     for (int t = L.t_begin; t < L.t_end; ++t) order.push_back(t);
     const int mm = ctx->m;
-    std::stable_sort(order.begin(), order.end(), [mm](int a, int b) {
+    std::stable_sort(order.begin(), order.end(), [mm, PAIR_BAND](int a, int b) {
         const int ra = a / mm, rb = b / mm, ba = ra / PAIR_BAND, bb = rb / PAIR_BAND;
         if (ba != bb) return ba < bb;
         if (a % mm != b % mm) return a % mm < b % mm;
