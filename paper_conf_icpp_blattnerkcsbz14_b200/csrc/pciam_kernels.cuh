@@ -256,8 +256,13 @@ struct ColTw {
 // K2: column FFT of a chunk of row-transformed tiles (G, complex, L2-resident), panel of
 // COL_P columns landed by TMA; writes the resident phase spectrum (or, for the test hook,
 // the complex spectrum back into G).
+#ifdef STITCH_K2_MAXREG   // experiment hook: register cap for K2 (80 fits three CTAs per SM)
+#define K2_MAXREG(PL) (PL::COL_MAXREG * 0 + STITCH_K2_MAXREG)
+#else
+#define K2_MAXREG(PL) PL::COL_MAXREG
+#endif
 template <class PL, bool PHASE_OUT>
-__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
+__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(K2_MAXREG(PL))
     k2t_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
                  uint32_t* __restrict__ spec, int tile0, const float2* __restrict__ tw2,
                  int ahead = 0) {
