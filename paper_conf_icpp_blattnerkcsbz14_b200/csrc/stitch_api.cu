@@ -456,8 +456,8 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     if (c->precision != 0 && c->precision != 1) return STITCH_ERR_INVALID_ARG;
     L->prec = c->precision;
     // fp64 chunks of 8 keep the 94 MB intermediate (8 x H x WP x 16 B at 1392x1040) in L2
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : (L->prec ? 8 : 96);
-    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : (L->prec ? 8 : 48);
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : (L->prec ? 8 : 160);
+    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : (L->prec ? 8 : 64);
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     // resident spectrum: u32 Q15 unit phasor (fp32) or double2 unit phasor (fp64)
