@@ -116,32 +116,52 @@ def band(rank: int, world: int, n: int, m: int):
     return b, e, halo
 
 
-def cpu_baseline(cfg: dict, sub_rows: int = 3, sub_cols: int = 4):
-    """The oracle as it stands, on a bounded sample (a sub_rows x sub_cols corner of the
-    workload's grid: same tiles, same pair kinds), all host cores."""
-    import oracle
-    g = synthgrid.make_grid(sub_rows, sub_cols, cfg["H"], cfg["W"], overlap=cfg["overlap"],
+# The oracle's bounded sample (cpu_baseline and the reference arm time the same one): the
+# top-left SUB corner of the workload's grid -- the same tiles and pair kinds as the GPU
+# step -- through oracle.grid (fp64, Fig. 4 over Fig. 2) on every host core.
+SUB = (4, 5)
+
+
+def metric_name(cfg: dict) -> str:
+    """One metric string for both arms (the driver pairs them by it)."""
+    return f"tile-pair translations/sec ({cfg['name']} grid)"
+
+
+def workload_config(cfg: dict, config_index: int) -> dict:
+    n, m, H, W = cfg["n"], cfg["m"], cfg["H"], cfg["W"]
+    return {"workload": f"{cfg['name']} (BASELINE.json configs[{config_index - 1}])",
+            "grid": f"{n}x{m}", "tile": f"{W}x{H} uint16", "pairs": 2 * n * m - n - m,
+            "tiles": n * m, "overlap": cfg["overlap"], "seed": synthgrid.SEED}
+
+
+def oracle_sample(cfg: dict):
+    g = synthgrid.make_grid(SUB[0], SUB[1], cfg["H"], cfg["W"], overlap=cfg["overlap"],
                             delta=cfg["delta"])
+    pairs = 2 * SUB[0] * SUB[1] - SUB[0] - SUB[1]
+    desc = (f"{SUB[0]}x{SUB[1]} corner of the {cfg['name']} grid ({pairs} pairs, "
+            f"{SUB[0] * SUB[1]} forward transforms) per sample, oracle.grid fp64")
+    return g, pairs, desc
+
+
+def cpu_baseline(cfg: dict):
+    """The oracle as it stands, on the bounded sample, all host cores (one sample)."""
+    import oracle
+    g, pairs, desc = oracle_sample(cfg)
     cores = os.cpu_count() or 1
     t = time.perf_counter()
     oracle.grid(g.tiles, threads=cores)
     dt = time.perf_counter() - t
-    pairs = 2 * sub_rows * sub_cols - sub_rows - sub_cols
     return {"value": pairs / dt, "unit": "pairs/s", "cores": cores, "kind": "oracle",
-            "sample": f"{sub_rows}x{sub_cols} corner of the {cfg['name']} grid ({pairs} pairs, "
-                      f"{sub_rows * sub_cols} tiles), oracle.grid fp64, {dt:.1f} s wall"}
+            "sample": f"{desc}, {dt:.1f} s wall"}
 
 
 def run_reference(args, cfg):
-    """Reference arm: the oracle timed on the host cores, bounded sample per step."""
+    """Reference arm: the oracle timed on the host cores, the same bounded sample per step."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
     import oracle
-    sub = (2, 3)
-    g = synthgrid.make_grid(sub[0], sub[1], cfg["H"], cfg["W"], overlap=cfg["overlap"],
-                            delta=cfg["delta"])
-    pairs = 2 * sub[0] * sub[1] - sub[0] - sub[1]
+    g, pairs, desc = oracle_sample(cfg)
     cores = os.cpu_count() or 1
     for _ in range(args.warmup):
         oracle.grid(g.tiles, threads=cores)
@@ -150,15 +170,16 @@ def run_reference(args, cfg):
         oracle.grid(g.tiles, threads=cores)
     dt = time.perf_counter() - t
     value = pairs * args.steps / dt
+    conf = workload_config(cfg, args.config)
+    conf["sample"] = desc
     line = {
-        "impl": "reference", "metric": f"tile-pair translations/sec ({cfg['name']} grid)",
+        "impl": "reference", "metric": metric_name(cfg),
         "value": value, "unit": "pairs/s", "n_gpus": args.gpus, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": 1e3 * dt / args.steps, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
-        "config": {"workload": cfg["name"], "sample": f"{sub[0]}x{sub[1]} sub-grid per step"},
+        "config": conf,
         "cpu_baseline": {"value": value, "unit": "pairs/s", "cores": cores, "kind": "oracle",
-                         "sample": f"{sub[0]}x{sub[1]} corner of the {cfg['name']} grid "
-                                   f"({pairs} pairs) per step"},
+                         "sample": desc},
         "e2e": {"value": value, "unit": "pairs/s", "h2d_bytes_per_step": 0,
                 "d2h_bytes_per_step": 0},
     }
@@ -256,8 +277,9 @@ def main():
     ap.add_argument("--dist-backend", default="nccl", choices=["nccl", "gloo"],
                     help="gloo: logic check of the N > 1 path with ranks sharing GPUs (not a "
                          "bench number; the halo goes through host memory)")
-    ap.add_argument("--no-exchange", action="store_true",
-                    help="N > 1: recompute the halo row's spectra instead of receiving them")
+    ap.add_argument("--transport", default=None, choices=["library", "torch", "recompute"],
+                    help="N > 1 halo: the library's NCCL send/recv (default with nccl), "
+                         "torch.distributed on a side stream (default with gloo), or recompute")
     args = ap.parse_args()
     cfg = dict(synthgrid.CONFIGS[args.config])
     if args.impl == "reference":
@@ -298,7 +320,8 @@ def main():
                         out=host.numpy().view(np.uint16), rows=(r0, r1))
     first = r0 * m
 
-    bp = BandPciam(n, m, H, W, rank, world, device=local, exchange=not args.no_exchange,
+    transport = args.transport or ("library" if args.dist_backend == "nccl" else "torch")
+    bp = BandPciam(n, m, H, W, rank, world, device=local, transport=transport,
                    chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles,
                    precision=1 if args.precision == "f64" else 0)
     pg = bp.grid
@@ -386,15 +409,22 @@ def main():
     avg_launch_ms = kd["ms"] / kd["launches"]
     pk, pk_kind = peaks()
     achieved = bytes_per_launch / (avg_launch_ms / 1e3) / 1e9
+    kms = {k: v["ms"] / nsteps_k for k, v in kt_sum.items()}
+    klaunch = {k: v["launches"] / nsteps_k for k, v in kt_sum.items()}
     roofline = {"bound": "hbm", "kernel": dom, "achieved": achieved, "peak": pk["hbm_gbs"],
                 "unit": "GB/s", "frac": achieved / pk["hbm_gbs"], "traffic": None,
                 "peak_source": pk_kind, "avg_launch_ms": avg_launch_ms,
                 "alg_bytes_per_launch": bytes_per_launch,
+                "byte_model": ("design: bytes each kernel must move with the resident spectrum "
+                               "as a Q15 unit phasor (S/2 per tile) and complex64 G/Q chunks "
+                               "(S); DESIGN.md section 6"),
                 "share_of_step": kd["ms"] / step_kernel_ms,
-                "kernels_ms_per_step": {k: v["ms"] / nsteps_k for k, v in kt_sum.items()},
-                "kernels_frac": {k: (alg_bytes_per_unit[k] * units_total[k] / (v["ms"] / nsteps_k
-                                                                              / 1e3) / 1e9)
-                                 / pk["hbm_gbs"] for k, v in kt_sum.items() if v["ms"] > 0}}
+                "kernels_ms_per_step": kms,
+                "kernels_launches_per_step": klaunch,
+                # algorithmic GB/s per kernel (K5's 2T per pair re-reads tiles K1 left in L2,
+                # so it is not an HBM fraction: see kernels_dram_frac)
+                "kernels_alg_GBps": {k: alg_bytes_per_unit[k] * units_total[k] / (ms / 1e3) / 1e9
+                                     for k, ms in kms.items() if ms > 0}}
     design_bytes = sum(alg_bytes_per_unit[k] * units_total[k] for k in alg_bytes_per_unit)
     survey_2pass = fwd_tiles * (T + 3 * S) + pairs_local * (4 * S + 2 * T)
     roofline["step_alg_GBps"] = design_bytes / (dev_ms / 1e3) / 1e9
@@ -415,16 +445,32 @@ def main():
     if args.precision == "f64":   # B200 FP64 vector rate: half the FP32 rate
         fft["peak_tflops"] = fp_peak / 2
     fft["frac"] = fft["achieved_tflops"] / fft["peak_tflops"]
+    # Measured DRAM traffic: dram__bytes_read.sum + dram__bytes_write.sum of one launch of each
+    # kernel (ncu --set full, caches flushed before the launch: an upper bound for a step
+    # whose kernels share L2) at the default chunks, scaled by the launches per step; the
+    # HBM fraction of each kernel and of the step on those bytes.
     traffic_path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(traffic_path) and args.precision == "f32":   # captured on the fp32 kernels
+    default_chunks = args.chunk_pairs == 0 and args.chunk_tiles == 0
+    if os.path.exists(traffic_path) and args.precision == "f32" and default_chunks:
         with open(traffic_path) as f:
-            tr = json.load(f).get(dom)
+            tj = json.load(f)
+        tr = tj.get(dom)
         if tr:
             roofline["traffic"] = tr.get("bytes_per_launch")
+        dram = {k: tj[k]["bytes_per_launch"] * klaunch[k] for k in kms
+                if k in tj and kms[k] > 0}
+        roofline["dram_source"] = tj.get("_source", "profiles/ncu_traffic.json")
+        roofline["kernels_dram_GB_per_step"] = {k: v / 1e9 for k, v in dram.items()}
+        roofline["kernels_dram_frac"] = {k: v / (kms[k] / 1e3) / 1e9 / pk["hbm_gbs"]
+                                         for k, v in dram.items()}
+        roofline["dram_frac"] = (dram[dom] / (kms[dom] / 1e3) / 1e9 / pk["hbm_gbs"]
+                                 if dom in dram else None)
+        roofline["step_dram_GB"] = sum(dram.values()) / 1e9
+        roofline["step_dram_frac"] = sum(dram.values()) / (dev_ms / 1e3) / 1e9 / pk["hbm_gbs"]
 
     # ---- e2e: through the C ABI from pinned host buffers ------------------------------
     e2e_steps = max(1, args.e2e_steps)
-    pipelined = not bp.use_exchange           # whole-band contexts: H2D pipelined under compute
+    pipelined = bp.transport != "torch"       # one library call per step: H2D pipelined
     if pipelined:
         pg.compute_from_host_async(host, first)     # warm: captures this buffer's graph
         pg.get_translations()
@@ -469,21 +515,26 @@ def main():
         cpu = cpu_baseline(cfg)
 
     if rank == 0:
+        conf = workload_config(cfg, args.config)
+        conf.update({"pairs": int(total_pairs), "grid_wall_ms": ms,
+                     "parallelism": f"row-bands x{world}",
+                     "halo": ({"library": "nccl-exchange (in library)",
+                               "torch": "exchange (torch.distributed)"}.get(bp.transport,
+                                                                            "recompute")
+                              if world > 1 else "none"),
+                     "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)"})
         line = {
-            "metric": f"tile-pair translations/sec ({cfg['name']} grid; grid wall time in config)",
+            "metric": metric_name(cfg),
             "value": value, "unit": "pairs/s", "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": value / PAPER_PAIRS_PER_S,
-            "vs_baseline_ref": "paper Pipelined-GPU 1xC2070, 42x59 in 49.7 s (Table II, P:L1208)"
-                               " = 97.7 pairs/s; other hardware, end-to-end incl. TIFF reads",
-            "dtype": args.precision, "data": "synthetic",
-            "config": {"workload": f"{cfg['name']} (BASELINE.json configs[{args.config - 1}])",
-                       "grid": f"{n}x{m}", "tile": f"{W}x{H} uint16", "pairs": int(total_pairs),
-                       "tiles": n * m, "grid_wall_ms": ms, "parallelism": f"row-bands x{world}",
-                       "halo": ("nccl-exchange" if bp.use_exchange else
-                                ("recompute" if world > 1 else "none")),
-                       "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)",
-                       "overlap": cfg["overlap"], "seed": synthgrid.SEED},
+            "scaling": "strong",
+            "vs_baseline": value / PAPER_PAIRS_PER_S if args.config == 3 else None,
+            "vs_baseline_ref": "BASELINE.md: paper Pipelined-GPU 1x C2070, 42x59 in 49.7 s "
+                               "(Table II, P:L1208) = 97.7 pairs/s; other hardware, end to end "
+                               "incl. TIFF reads",
+            "dtype": ("f64" if args.precision == "f64" else "f32 (Q15 resident phasor)"),
+            "data": "synthetic",
+            "config": conf,
             "roofline": roofline,
             "fft_flops": fft,
             "cpu_baseline": cpu,

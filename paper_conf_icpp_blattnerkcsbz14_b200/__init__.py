@@ -23,7 +23,10 @@ _PKG = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_PKG, "libstitch_b200.so")
 
 STATUS = {0: "STITCH_OK", 1: "STITCH_ERR_INVALID_ARG", 2: "STITCH_ERR_UNSUPPORTED",
-          3: "STITCH_ERR_OUT_OF_MEMORY", 4: "STITCH_ERR_CUDA", 6: "STITCH_ERR_STATE"}
+          3: "STITCH_ERR_OUT_OF_MEMORY", 4: "STITCH_ERR_CUDA", 5: "STITCH_ERR_NCCL",
+          6: "STITCH_ERR_STATE"}
+FLAG_NO_GRAPH = 1   # STITCH_FLAG_NO_GRAPH: direct launches instead of a replayed CUDA graph
+FLAG_SERIAL = 2     # STITCH_FLAG_SERIAL: one stream for every kernel
 
 # stitch_pair (include/stitch.h), 64 bytes
 PAIR_DTYPE = np.dtype([
@@ -49,7 +52,9 @@ class Config(ctypes.Structure):
                 ("tile_end", ctypes.c_int32), ("chunk_pairs", ctypes.c_int32),
                 ("chunk_tiles", ctypes.c_int32), ("precision", ctypes.c_int32),
                 ("stream", ctypes.c_void_p), ("workspace", ctypes.c_void_p),
-                ("workspace_bytes", ctypes.c_size_t)]
+                ("workspace_bytes", ctypes.c_size_t), ("pool_tiles", ctypes.c_int32),
+                ("rank", ctypes.c_int32), ("world_size", ctypes.c_int32),
+                ("nccl_id", ctypes.c_void_p), ("flags", ctypes.c_uint32)]
 
 
 EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count", "stitch_init",
@@ -60,7 +65,8 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_load_tiles", "stitch_resident_range", "stitch_kernel_timings",
            "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async",
            "stitch_global_positions", "stitch_compose_overlay", "stitch_debug_spectrum_f64",
-           "stitch_compute_translations_from_host_async", "stitch_timeline"]
+           "stitch_compute_translations_from_host_async", "stitch_timeline",
+           "stitch_nccl_unique_id", "stitch_pairs_part_async", "stitch_debug_surface"]
 
 _lib = None
 
@@ -78,6 +84,9 @@ def load_library():
     C = P(Config)
     sig = {
         "stitch_status_string": (ctypes.c_char_p, [ctypes.c_int]),
+        "stitch_nccl_unique_id": (ctypes.c_int, [vp]),
+        "stitch_pairs_part_async": (ctypes.c_int, [vp, i32]),
+        "stitch_debug_surface": (ctypes.c_int, [vp, i32, i32, vp]),
         "stitch_workspace_size": (ctypes.c_int, [C, P(ctypes.c_size_t)]),
         "stitch_pair_count": (ctypes.c_int, [C, P(i64)]),
         "stitch_init": (ctypes.c_int, [C, P(vp)]),
@@ -115,10 +124,21 @@ def load_library():
 
 
 def make_config(n, m, H, W, device=0, tile_begin=0, tile_end=0, chunk_pairs=0, chunk_tiles=0,
-                stream=None, workspace=None, workspace_bytes=0, precision=0) -> Config:
-    """precision: 0 = fp32 transforms (default), 1 = fp64."""
+                stream=None, workspace=None, workspace_bytes=0, precision=0, pool_tiles=0,
+                rank=0, world_size=1, nccl_id=None, flags=0) -> Config:
+    """precision: 0 = fp32 transforms (default), 1 = fp64; pool_tiles > 0: the
+    bounded mode (row f1); nccl_id: 128 bytes from nccl_unique_id() (in-library halo exchange)."""
     return Config(W, H, n, m, device, tile_begin, tile_end, chunk_pairs, chunk_tiles, precision,
-                  stream, workspace, workspace_bytes)
+                  stream, workspace, workspace_bytes, pool_tiles, rank, world_size, nccl_id, flags)
+
+
+def nccl_unique_id() -> bytes:
+    """A fresh 128-byte NCCL unique id (rank 0; broadcast it to the other ranks)."""
+    buf = ctypes.create_string_buffer(128)
+    st = load_library().stitch_nccl_unique_id(buf)
+    if st:
+        raise StitchError(st, "stitch_nccl_unique_id")
+    return buf.raw
 
 
 def workspace_size(cfg: Config) -> int:
@@ -172,19 +192,29 @@ def compose_overlay(tiles, pos_xy: np.ndarray, canvas=None):
 
 class PciamGrid:
     """One context over an n x m grid of H x W uint16 tiles (or the row band
-    [tile_begin, tile_end) of it, for multi-GPU row-band partitioning)."""
+    [tile_begin, tile_end) of it, for multi-GPU row-band partitioning).
+
+    pool_tiles > 0 selects the bounded mode: a fixed pool of tile slots recycled
+    by reference count; tiles then arrive through compute_from_host_async.  rank / world_size /
+    nccl_id: the in-library NCCL halo exchange (the library derives the rank's band)."""
 
     def __init__(self, n: int, m: int, H: int, W: int, device: int = 0, tile_begin: int = 0,
                  tile_end: int = 0, chunk_pairs: int = 0, chunk_tiles: int = 0,
-                 use_torch: bool = True, precision: int = 0):
+                 use_torch: bool = True, precision: int = 0, pool_tiles: int = 0,
+                 rank: int = 0, world_size: int = 1, nccl_id: bytes | None = None,
+                 flags: int = 0):
         self.lib = load_library()
         self.n, self.m, self.H, self.W = n, m, H, W
         self.device = device
         self._ctx = ctypes.c_void_p(None)
         self._ws = None
         self.precision = precision
+        self._nccl_id = ctypes.create_string_buffer(nccl_id, 128) if nccl_id is not None else None
         cfg = make_config(n, m, H, W, device, tile_begin, tile_end, chunk_pairs, chunk_tiles,
-                          precision=precision)
+                          precision=precision, pool_tiles=pool_tiles, rank=rank,
+                          world_size=world_size,
+                          nccl_id=ctypes.cast(self._nccl_id, ctypes.c_void_p) if nccl_id else None,
+                          flags=flags)
         self.stream = None
         if use_torch:
             import torch
@@ -199,16 +229,28 @@ class PciamGrid:
             cfg.stream = self.stream.cuda_stream
             cfg.workspace = self._ws.data_ptr()
             cfg.workspace_bytes = nbytes
+            # the workspace was allocated on the current stream: order the context after it
+            self._after_torch()
         self.cfg = cfg
         self.npairs = pair_count(cfg)
-        self.tile_begin = tile_begin
-        self.tile_end = tile_end if tile_end else n * m
         self._check(self.lib.stitch_init(ctypes.byref(cfg), ctypes.byref(self._ctx)), "init")
+        hb, tb, te = self.resident_range()
+        self.halo_begin, self.tile_begin, self.tile_end = hb, tb, te
 
     def _check(self, st: int, what: str):
         if st:
             msg = self.lib.stitch_last_error(self._ctx).decode() if self._ctx else ""
             raise StitchError(st, f"{what}: {msg}")
+
+    def _after_torch(self, tensor=None) -> None:
+        """Order the context stream after torch's current stream (where `tensor` was written)
+        and tell torch's allocator the context stream uses `tensor`."""
+        import torch
+        cur = torch.cuda.current_stream(torch.device("cuda", self.device))
+        if self.stream is not None and cur.cuda_stream != self.stream.cuda_stream:
+            self.stream.wait_stream(cur)
+        if tensor is not None and tensor.is_cuda and self.stream is not None:
+            tensor.record_stream(self.stream)
 
     # -- step 1: load --------------------------------------------------------
     def load_grid(self, tiles) -> None:
@@ -217,15 +259,15 @@ class PciamGrid:
         if isinstance(tiles, np.ndarray):
             if tiles.dtype != np.uint16 or not tiles.flags.c_contiguous or tiles.nbytes != nbytes:
                 raise ValueError("tiles must be a C-contiguous uint16 [n, m, H, W] array")
-            self._keep = tiles
             self._check(self.lib.stitch_load_grid(self._ctx, tiles.ctypes.data, nbytes), "load")
             return
         import torch
         if tiles.dtype != torch.uint16 or not tiles.is_contiguous() or \
                 tiles.numel() * 2 != nbytes:
             raise ValueError("tiles must be a contiguous torch.uint16 [n, m, H, W] tensor")
-        self._keep = tiles
         if tiles.is_cuda:
+            self._after_torch(tiles)
+            self._keep = tiles
             self._check(self.lib.stitch_load_grid_device(self._ctx, tiles.data_ptr(), nbytes),
                         "load")
         else:
@@ -242,7 +284,6 @@ class PciamGrid:
         """Load a run of consecutive tiles starting at `first_tile` (numpy or torch, [k, H, W]
         or [rows, m, H, W]) covering resident_range()."""
         count = (tiles.size if isinstance(tiles, np.ndarray) else tiles.numel()) // (self.H * self.W)
-        self._keep = tiles
         if isinstance(tiles, np.ndarray):
             if tiles.dtype != np.uint16 or not tiles.flags.c_contiguous:
                 raise ValueError("tiles must be C-contiguous uint16")
@@ -252,6 +293,9 @@ class PciamGrid:
             if tiles.dtype != torch.uint16 or not tiles.is_contiguous():
                 raise ValueError("tiles must be a contiguous torch.uint16 tensor")
             ptr, dev = tiles.data_ptr(), int(tiles.is_cuda)
+            if dev:
+                self._after_torch(tiles)
+                self._keep = tiles
         self._check(self.lib.stitch_load_tiles(self._ctx, ptr, first_tile, count, dev), "load")
 
     def compute_from_host_async(self, tiles, first_tile: int = 0) -> None:
@@ -283,9 +327,10 @@ class PciamGrid:
         """Step 2 for resident tiles [first_tile, first_tile + count) (global indices)."""
         self._check(self.lib.stitch_forward_range_async(self._ctx, first_tile, count), "forward")
 
-    def pairs_async(self) -> None:
-        """Steps 3-7 for every pair of the context (spectra already resident)."""
-        self._check(self.lib.stitch_pairs_async(self._ctx), "pairs")
+    def pairs_async(self, part: int = 0) -> None:
+        """Steps 3-7 (spectra already resident) for part 0 = every pair of the context,
+        1 = the interior pairs (tile A owned), 2 = the boundary pairs (tile A in the halo)."""
+        self._check(self.lib.stitch_pairs_part_async(self._ctx, int(part)), "pairs")
 
     def spectra_range(self, first_tile: int, count: int) -> tuple[int, int]:
         """(device address, bytes) of the resident spectra of tiles [first_tile, +count)."""
@@ -304,10 +349,19 @@ class PciamGrid:
         return self._ws[off: off + nbytes]
 
     def get_translations(self, west: np.ndarray | None = None, north: np.ndarray | None = None):
+        """Copy the last compute's results out: (west, north) PAIR_DTYPE arrays [n, m].  Caller
+        arrays (to merge several band contexts) must be C-contiguous PAIR_DTYPE of n*m entries;
+        only the owned tiles' entries are written."""
+        nt = self.n * self.m
         if west is None:
-            west = np.zeros(self.n * self.m, PAIR_DTYPE)
+            west = np.zeros(nt, PAIR_DTYPE)
         if north is None:
-            north = np.zeros(self.n * self.m, PAIR_DTYPE)
+            north = np.zeros(nt, PAIR_DTYPE)
+        for a in (west, north):
+            if not isinstance(a, np.ndarray) or a.dtype != PAIR_DTYPE or a.size != nt or \
+                    not a.flags.c_contiguous or not a.flags.writeable:
+                raise ValueError(f"result arrays must be writeable C-contiguous PAIR_DTYPE "
+                                 f"arrays of n*m = {nt} entries")
         self._check(self.lib.stitch_get_translations(self._ctx, west.ctypes.data,
                                                      north.ctypes.data), "get")
         return west.reshape(self.n, self.m), north.reshape(self.n, self.m)
@@ -330,6 +384,15 @@ class PciamGrid:
             return out
         out = np.empty((self.H, self.W // 2 + 1), np.complex64)
         self._check(self.lib.stitch_debug_spectrum(self._ctx, tile, out.ctypes.data), "spectrum")
+        return out
+
+    def surface(self, tile: int, kind: int) -> np.ndarray:
+        """Test hook (reading C11): the normalised correlation surface |iFFT2(NCC)|/(HW),
+        float32 [H, W], of the (kind 0 west / 1 north) pair of `tile`, computed by the step's
+        K3 + K4 transforms from the last computed spectra."""
+        out = np.empty((self.H, self.W), np.float32)
+        self._check(self.lib.stitch_debug_surface(self._ctx, int(tile), int(kind),
+                                                  out.ctypes.data), "surface")
         return out
 
     def synchronize(self) -> None:

@@ -13,10 +13,23 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libstitch_b200.so")
 SOURCES = ["stitch_api.cu", "phase23.cu"]
-HEADERS = ["fft_engine.cuh", "pciam_kernels.cuh", "pciam_fp64.cuh", "warp_rows.cuh", "col_groups.cuh",
+HEADERS = ["fft_engine.cuh", "pciam_kernels.cuh", "pciam_fp64.cuh", "warp_rows.cuh",
            "async_copy.cuh", "codelets.cuh", "gen_codelets.py"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
+
+
+def nccl_include() -> str:
+    """nccl.h for the types of the run-time-loaded NCCL (the copy torch ships, else the system's)."""
+    try:
+        import nvidia.nccl
+        for d in nvidia.nccl.__path__:
+            inc = os.path.join(d, "include")
+            if os.path.exists(os.path.join(inc, "nccl.h")):
+                return inc
+    except ImportError:
+        pass
+    return "/usr/include"
 
 
 def _stale(target: str, deps: list[str]) -> bool:
@@ -43,10 +56,11 @@ def build(force: bool = False, ptxas_verbose: bool = False) -> str:
     if not force and not _stale(LIB, deps):
         return LIB
     cmd = [NVCC, "-O3", "-std=c++17", *ARCH, "-lineinfo", "-Xcompiler", "-fPIC", "-shared",
-           "-I" + os.path.join(ROOT, "include"), "-o", LIB]
+           "-I" + os.path.join(ROOT, "include"), "-I" + nccl_include(), "-o", LIB]
     if ptxas_verbose:
         cmd += ["-Xptxas", "-v"]
     cmd += [os.path.join(CSRC, s) for s in SOURCES]
+    cmd += ["-ldl"]
     subprocess.check_call(cmd)
     return LIB
 

@@ -2,11 +2,17 @@
 //
 // Data layout in HBM:
 //   raw   uint16 [tiles][H][W]           W contiguous (the caller's tile layout)
-//   G     float2 [chunk][H][WP]          row-transformed tiles of a forward chunk (L2-sized)
-//   spec  u32    [tiles][H][WP]          resident half spectrum kx in [0, W/2] (WP = pad16(W/2+1))
+//   raw   uint16 [slots][H][W]           tile pixels by slot (slot = tile in the resident mode;
+//                                        a recycled pool slot in the bounded mode, row f1)
+//   G     float2 [chunk][H][WP]          row-transformed tiles of a forward chunk
+//   spec  u32    [slots][H][WP]          half spectrum kx in [0, W/2] (WP = pad16(W/2+1))
 //                                        stored as its Q15 unit phasor F/|F| (2 x int16),
 //                                        reused by <= 4 pairs
-//   Q     float2 [chunk][H][WP]          per-pair column-inverse intermediate (L2-sized chunk)
+//   Q     float2 [chunk][H][WP]          per-pair column-inverse intermediate
+//   fslot i32    [local tiles]           slot of each local tile (K1/K2 write there)
+//   pairs {a, b} [pairs]                 slots of the pair's tiles (K3/K5 read there)
+// (G and Q chunks are 0.38 / 0.94 GB at the default 64 / 160 chunks: they round-trip HBM,
+// DESIGN.md section 6.)
 //   keys  u64    [pairs]                 packed (|c| bits << 32 | ~index) argmax per pair
 //   mom   u64    [pairs][4][5]           exact integer CCF moments per candidate
 //
@@ -73,10 +79,6 @@ struct Plan {
         CI::STAGES == 1 ? 0 : sizeof(float2) * COL_P * CI::R1 * (CI::R0 + COL_PAD);
     static constexpr size_t COL_BUF = ((COL_LAND > COL_XCH ? COL_LAND : COL_XCH) + 15) / 16 * 16;
     static constexpr int COL_TW2N = CI::R0 * (CI::R1 - 1);      // stage-2 twiddles in smem
-    // persistent column kernels: separate landing and exchange buffers (prefetch overlap)
-    static constexpr size_t COLP_XOFF = (COL_LAND + 127) / 128 * 128;
-    static constexpr size_t COLP_TOFF = COLP_XOFF + (COL_XCH + 15) / 16 * 16;
-    static constexpr size_t COLP_SMEM = COLP_TOFF + sizeof(float2) * (COL_TW2N > 0 ? COL_TW2N : 1);
     static constexpr size_t COL_SMEM = COL_BUF + sizeof(float2) * (COL_TW2N > 0 ? COL_TW2N : 1);
     static constexpr int BOXH = H / ((H + 255) / 256);   // TMA box rows (<= 256)
     static_assert(H % BOXH == 0, "H must split into equal TMA boxes of <= 256 rows");
@@ -100,7 +102,7 @@ struct Plan {
 };
 
 struct PairIdx {
-    int32_t a, b;  // local tile indices: A = west/north neighbour, B = tile
+    int32_t a, b;  // slots of A = west/north neighbour and B = tile
 };
 
 // ------------------------------------------------------------------ K1 ----
@@ -138,11 +140,12 @@ __device__ __forceinline__ void r2c_post_line(const Xc& xc, int line, float2* __
 template <class PL>
 __global__ void __launch_bounds__(PL::ROW_T) k1_fwd_rows(const uint16_t* __restrict__ raw,
                                                          float2* __restrict__ G, int tile0,
+                                                         const int32_t* __restrict__ fslot,
                                                          const float2* __restrict__ tw2,
                                                          const float2* __restrict__ twW) {
     extern __shared__ float2 smem[];
     constexpr int L = PL::ROW_L, T = PL::ROW_T;
-    const size_t t = (size_t)tile0 + blockIdx.y;
+    const size_t t = (size_t)fslot[tile0 + blockIdx.y];
     const int y0 = blockIdx.x * L;
     U16RowSrc<PL> src{reinterpret_cast<const uint32_t*>(raw + (t * PL::H + y0) * PL::W)};
     typename PL::RowX xc{smem};
@@ -253,19 +256,15 @@ struct ColTw {
     }
 };
 
-// K2: column FFT of a chunk of row-transformed tiles (G, complex, L2-resident), panel of
-// COL_P columns landed by TMA; writes the resident phase spectrum (or, for the test hook,
-// the complex spectrum back into G).
-#ifdef STITCH_K2_MAXREG   // experiment hook: register cap for K2 (80 fits three CTAs per SM)
-#define K2_MAXREG(PL) (PL::COL_MAXREG * 0 + STITCH_K2_MAXREG)
-#else
-#define K2_MAXREG(PL) PL::COL_MAXREG
-#endif
+// K2: column FFT of a chunk of row-transformed tiles (G, complex), panel of COL_P columns
+// landed by TMA; writes the phase spectrum of each tile's slot (or, for the test hook, the
+// complex spectrum back into G).  `ahead`: L2 prefetch of the panel of the CTA that many
+// launch slots later (one wave of resident CTAs: K2 7.25 -> 6.86 ms).
 template <class PL, bool PHASE_OUT>
-__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(K2_MAXREG(PL))
+__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     k2t_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
-                 uint32_t* __restrict__ spec, int tile0, const float2* __restrict__ tw2,
-                 int ahead = 0) {
+                 uint32_t* __restrict__ spec, int tile0, const int32_t* __restrict__ fslot,
+                 const float2* __restrict__ tw2, int ahead) {
     extern __shared__ __align__(128) unsigned char csmem[];
     __shared__ uint64_t bar;
     const int tl = blockIdx.y, c0 = blockIdx.x * PL::COL_P;
@@ -290,7 +289,7 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(K2_MAXREG(PL))
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
     using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, true>;
     if constexpr (PHASE_OUT) {
-        PhaseDst<PL> dst{spec + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
+        PhaseDst<PL> dst{spec + (size_t)fslot[tile0 + tl] * PL::H * PL::WP + c0};
         Run::template run<true>(src, xc, dst, tws);
     } else {
         PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
@@ -313,8 +312,7 @@ struct NcpsPhaseSrc {  // step 3 from two landed phasor panels: U_A conj(U_B) (x
 template <class PL>
 __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     k3t_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
-                  const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2,
-                  int ahead = 0) {
+                  const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2) {
     extern __shared__ __align__(128) unsigned char csmem[];
     __shared__ uint64_t bar;
     const PairIdx pr = pairs[pair0 + blockIdx.y];
@@ -333,13 +331,6 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
         tma_panel<PL>(la, &tmS, c0, pr.a * PL::H, 4, &bar);
         tma_panel<PL>(lb, &tmS, c0, pr.b * PL::H, 4, &bar);
         ColTw<PL>::issue(tws, tw2, &bar);
-        int pn, it;
-        ahead_cta(ahead, pn, it);
-        if (it >= 0) {
-            const PairIdx nx = pairs[pair0 + it];
-            l2_prefetch_panel<PL>(&tmS, pn * PL::COL_P, nx.a * PL::H);
-            l2_prefetch_panel<PL>(&tmS, pn * PL::COL_P, nx.b * PL::H);
-        }
     }
     ColTw<PL>::fallback(tws, tw2);
     mbar_wait(&bar, 0);
@@ -348,111 +339,6 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
     FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, true>::template run<true>(src, xc,
                                                                                          dst, tws);
-}
-
-// ------------------------------------------ persistent column kernels ----
-// K2p / K3p: one CTA per SM walks (tile|pair, panel) items in static round robin.  Each
-// item's panel lands by TMA in its own buffer; stage 1 reads it into registers, and right
-// after that barrier the TMA for the next item is issued, so the fetch overlaps stage 1's
-// butterflies, the exchange and stage 2 of the current item.
-// MINB: CTAs per SM the kernel is register-budgeted for.  TWG: stage-2 twiddles read through
-// L1 from global memory instead of a shared copy (the narrow-panel "quad" plans, 4 columns
-// per panel, fit three CTAs per SM only without it: landing + exchange = 67 KB per CTA).
-template <class PL, bool PHASE_OUT, int MINB = 1, bool TWG = false>
-__global__ void __launch_bounds__(PL::COL_T, MINB)
-    k2p_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
-                 uint32_t* __restrict__ spec, int tile0, int ntiles,
-                 const float2* __restrict__ tw2) {
-    extern __shared__ __align__(128) unsigned char csmem[];
-    __shared__ uint64_t bar;
-    constexpr int NP = PL::WP / PL::COL_P;
-    const int nitems = ntiles * NP;
-    typename PL::ColX xc{reinterpret_cast<float2*>(csmem + PL::COLP_XOFF)};
-    float2* tws = reinterpret_cast<float2*>(csmem + PL::COLP_TOFF);
-    auto issue = [&](int item) {
-        const int tl = item / NP, panel = item - tl * NP;
-        mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C);
-        tma_panel<PL>(csmem, &tmG, 2 * panel * PL::COL_P, tl * PL::H, 8, &bar);
-    };
-    if (threadIdx.x == 0) {
-        prefetch_tensormap(&tmG);
-        mbar_init(&bar, 1);
-        fence_mbar_init();
-    }
-    if constexpr (!TWG)
-        for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
-    const float2* twp = TWG ? tw2 : tws;
-    __syncthreads();
-    if (threadIdx.x == 0 && (int)blockIdx.x < nitems) issue(blockIdx.x);
-    using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, !TWG>;
-    int k = 0;
-    for (int item = blockIdx.x; item < nitems; item += gridDim.x, ++k) {
-        mbar_wait(&bar, k & 1);
-        const int tl = item / NP, c0 = (item - tl * NP) * PL::COL_P;
-        const int nxt = item + gridDim.x;
-        auto after_loads = [&]() {
-            if (threadIdx.x == 0 && nxt < nitems) {
-                fence_proxy_async();
-                issue(nxt);
-            }
-        };
-        LandSrc<PL> src{reinterpret_cast<const float2*>(csmem)};
-        if constexpr (PHASE_OUT) {
-            PhaseDst<PL> dst{spec + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
-            Run::template run<true>(src, xc, dst, twp, NoMid(), after_loads);
-        } else {
-            PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
-            Run::template run<true>(src, xc, dst, twp, NoMid(), after_loads);
-        }
-    }
-}
-
-template <class PL, int MINB = 1, bool TWG = false>
-__global__ void __launch_bounds__(PL::COL_T, MINB)
-    k3p_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
-                  const PairIdx* __restrict__ pairs, int pair0, int npairs,
-                  const float2* __restrict__ tw2) {
-    extern __shared__ __align__(128) unsigned char csmem[];
-    __shared__ uint64_t bar;
-    constexpr int NP = PL::WP / PL::COL_P;
-    const int nitems = npairs * NP;
-    uint32_t* la = reinterpret_cast<uint32_t*>(csmem);
-    uint32_t* lb = reinterpret_cast<uint32_t*>(csmem + PL::COL_PHASE_B);
-    typename PL::ColX xc{reinterpret_cast<float2*>(csmem + PL::COLP_XOFF)};
-    float2* tws = reinterpret_cast<float2*>(csmem + PL::COLP_TOFF);
-    auto issue = [&](int item) {
-        const int pl = item / NP, panel = item - pl * NP;
-        const PairIdx pr = pairs[pair0 + pl];
-        mbar_arrive_expect_tx(&bar, (uint32_t)(2 * PL::H * PL::COL_P * 4));
-        tma_panel<PL>(la, &tmS, panel * PL::COL_P, pr.a * PL::H, 4, &bar);
-        tma_panel<PL>(lb, &tmS, panel * PL::COL_P, pr.b * PL::H, 4, &bar);
-    };
-    if (threadIdx.x == 0) {
-        prefetch_tensormap(&tmS);
-        mbar_init(&bar, 1);
-        fence_mbar_init();
-    }
-    if constexpr (!TWG)
-        for (int i = threadIdx.x; i < PL::COL_TW2N; i += PL::COL_T) tws[i] = __ldg(tw2 + i);
-    const float2* twp = TWG ? tw2 : tws;
-    __syncthreads();
-    if (threadIdx.x == 0 && (int)blockIdx.x < nitems) issue(blockIdx.x);
-    using Run = FftRun<typename PL::Col, +1, PL::COL_P, PL::COL_T, ColMap, !TWG>;
-    int k = 0;
-    for (int item = blockIdx.x; item < nitems; item += gridDim.x, ++k) {
-        mbar_wait(&bar, k & 1);
-        const int pl = item / NP, c0 = (item - pl * NP) * PL::COL_P;
-        const int nxt = item + gridDim.x;
-        auto after_loads = [&]() {
-            if (threadIdx.x == 0 && nxt < nitems) {
-                fence_proxy_async();
-                issue(nxt);
-            }
-        };
-        NcpsPhaseSrc<PL> src{la, lb};
-        PanelIO<PL> dst{Q + (size_t)pl * PL::H * PL::WP + c0};
-        Run::template run<true>(src, xc, dst, twp, NoMid(), after_loads);
-    }
 }
 
 // ------------------------------------------------------------------ K4 ----
@@ -536,206 +422,42 @@ __device__ __forceinline__ unsigned long long block_max_u64(unsigned long long v
     return v;
 }
 
-template <class PL>
+// Test hook (stitch_debug_surface): the correlation surface |x| * scale stored row-major
+// [H][W] instead of reduced (the same transform, so the same values the argmax sees).
+struct SurfaceDst {
+    float* out;
+    int row_base, W;
+    float scale;
+    __device__ __forceinline__ void store(int line, int n, float2 v) const {
+        float* o = out + (size_t)(row_base + line) * W + 2 * n;
+        o[0] = fabsf(v.x) * scale;
+        o[1] = fabsf(v.y) * scale;
+    }
+};
+
+// CTA row kernel (plans whose row transform is not a two-stage warp FFT: 48x40, 58x26).
+// SURF: the test hook's surface output instead of the argmax.
+template <class PL, bool SURF = false>
 __global__ void __launch_bounds__(PL::ROW_T) k4_pair_rows(const float2* __restrict__ Q,
                                                           unsigned long long* __restrict__ keys,
                                                           int pair0,
                                                           const float2* __restrict__ tw2,
-                                                          const float2* __restrict__ twW) {
+                                                          const float2* __restrict__ twW,
+                                                          float* __restrict__ surf = nullptr,
+                                                          float scale = 0.f) {
     extern __shared__ float2 smem[];
     constexpr int L = PL::ROW_L, T = PL::ROW_T;
     const int y0 = blockIdx.x * L;
     C2RSrc<PL> src{Q + ((size_t)blockIdx.y * PL::H + y0) * PL::WP, twW};
-    ArgmaxDst dst{-1.f, 0xFFFFFFFFu, y0, PL::W};
     typename PL::RowX xc{smem};
-    FftRun<typename PL::Row, +1, L, T, RowMap>::run(src, xc, dst, tw2);
-    const unsigned long long best = block_max_u64<T>(dst.key());
-    if (threadIdx.x == 0) atomicMax(&keys[pair0 + blockIdx.y], best);
-}
-
-// ------------------------------------------------ persistent row kernels ----
-// K1p / K4p: persistent CTAs walk the row blocks of a chunk (static round robin).  A
-// block's input rows land in shared memory by TMA bulk copy (cp.async.bulk + mbarrier);
-// the copy for block k+1 is issued as soon as stage 1 of block k has consumed the
-// landing buffer, so it overlaps stage 2 / the epilogue of block k and the other CTAs
-// on the SM.  Stage-2 twiddle tables live in shared memory.
-template <class PL>
-struct RowPersist {
-    static constexpr int L = PL::ROW_L;
-    static constexpr int LP = PL::WP + 8;            // padded landing pitch (float2), 16-B rows
-    static constexpr int RAWB = L * PL::W * 2;       // raw landing bytes per block (K1)
-    static constexpr int QB = L * PL::WP * 8;        // Q landing bytes per block (K4, copied row by row)
-    static constexpr int XCH = L * PL::RowX::LSTRIDE;  // exchange float2
-    static constexpr int TW2 = PL::ROW_TW2 > 0 ? PL::ROW_TW2 : 1;
-    static constexpr int TWW = PL::M + 1;
-    // byte offsets in dynamic shared memory
-    static constexpr size_t OFF_BAR = 0;                              // 2 x u64
-    static constexpr size_t OFF_TW2 = 16;
-    static constexpr size_t OFF_TWW = OFF_TW2 + (size_t)TW2 * 8;
-    static constexpr size_t OFF_XCH = (OFF_TWW + (size_t)TWW * 8 + 15) / 16 * 16;
-    static constexpr size_t OFF_LAND = OFF_XCH + (size_t)XCH * 8;
-    static constexpr size_t LAND_K1 = ((size_t)RAWB + 15) / 16 * 16;
-    static constexpr size_t LAND_K4 = (size_t)L * LP * 8;
-    static constexpr size_t SMEM_K1 = OFF_LAND + LAND_K1;
-    // K4 keeps w_W in global memory (L1) so three CTAs fit an SM
-    static constexpr size_t OFF_XCH4 = (OFF_TW2 + (size_t)TW2 * 8 + 15) / 16 * 16;
-    static constexpr size_t OFF_LAND4 = OFF_XCH4 + (size_t)XCH * 8;
-    static constexpr size_t SMEM_K4 = OFF_LAND4 + LAND_K4;
-    static constexpr bool K1_BULK = (PL::W * 2) % 16 == 0;   // raw rows 16-byte aligned
-};
-
-template <class PL>
-__device__ __forceinline__ void load_row_tables(float2* tw2s, float2* twWs, const float2* tw2,
-                                                const float2* twW) {
-    for (int i = threadIdx.x; i < PL::ROW_TW2; i += PL::ROW_T) tw2s[i] = __ldg(tw2 + i);
-    for (int i = threadIdx.x; i <= PL::M; i += PL::ROW_T) twWs[i] = __ldg(twW + i);
-}
-
-template <class PL>
-struct U16SmemSrc {  // z[n] = x[2n] + i x[2n+1] from a landed raw row block
-    const uint32_t* p;
-    __device__ __forceinline__ float2 load(int line, int n) const {
-        const uint32_t u = p[line * (PL::W / 2) + n];
-        return make_float2((float)(u & 0xFFFFu), (float)(u >> 16));
-    }
-};
-
-template <class PL>
-__global__ void __launch_bounds__(PL::ROW_T) k1p_fwd_rows(const uint16_t* __restrict__ raw,
-                                                          float2* __restrict__ G, int tile0,
-                                                          int ntiles,
-                                                          const float2* __restrict__ tw2,
-                                                          const float2* __restrict__ twW) {
-    using RP = RowPersist<PL>;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    constexpr int L = PL::ROW_L, T = PL::ROW_T, BPT = PL::H / L;
-    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + RP::OFF_BAR);
-    float2* tw2s = reinterpret_cast<float2*>(smem_raw + RP::OFF_TW2);
-    float2* twWs = reinterpret_cast<float2*>(smem_raw + RP::OFF_TWW);
-    typename PL::RowX xc{reinterpret_cast<float2*>(smem_raw + RP::OFF_XCH)};
-    unsigned char* land = smem_raw + RP::OFF_LAND;
-    const int nblk = ntiles * BPT;
-    auto issue = [&](int blk, int buf) {
-        const int tl = blk / BPT, y0 = (blk - tl * BPT) * L;
-        const uint16_t* src = raw + ((size_t)(tile0 + tl) * PL::H + y0) * PL::W;
-        mbar_arrive_expect_tx(&bar[buf], RP::RAWB);
-        bulk_g2s(land, src, RP::RAWB, &bar[buf]);
-    };
-    if (threadIdx.x == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
-        fence_mbar_init();
-    }
-    load_row_tables<PL>(tw2s, twWs, tw2, twW);
-    __syncthreads();
-    // One landing buffer: block k+1's rows are fetched (TMA bulk copy) as soon as stage 1
-    // of block k has consumed them, overlapping stage 2 + post-processing of block k.
-    // Round robin over row blocks: neighbouring CTAs read neighbouring raw rows
-    // (measured faster than contiguous per-CTA ranges here).
-    if (threadIdx.x == 0 && (int)blockIdx.x < nblk) issue(blockIdx.x, 0);
-    int k = 0;
-    for (int blk = blockIdx.x; blk < nblk; blk += gridDim.x, ++k) {
-        mbar_wait(&bar[0], k & 1);
-        const int tl = blk / BPT, y0 = (blk - tl * BPT) * L;
-        const int nxt = blk + gridDim.x;
-        U16SmemSrc<PL> src{reinterpret_cast<const uint32_t*>(land)};
-        auto prefetch = [&]() {
-            if (threadIdx.x == 0 && nxt < nblk) {
-                fence_proxy_async();
-                issue(nxt, 0);
-            }
-        };
-        FftRun<typename PL::Row, -1, L, T, RowMap, true>::run(src, xc, xc, tw2s, prefetch);
-        __syncthreads();
-        float2* out0 = G + ((size_t)tl * PL::H + y0) * PL::WP;
-#pragma unroll 1
-        for (int line = 0; line < L; ++line)
-            r2c_post_line<PL>(xc, line, out0 + (size_t)line * PL::WP,
-                              [&](int q) { return twWs[q]; });
-        __syncthreads();   // exchange free
-    }
-}
-
-template <class PL>
-struct C2RSmemSrc {  // C2R pre-processing from a landed Q row block (pitch LP)
-    const float2* rows;
-    const float2* twW;
-    __device__ __forceinline__ float2 load(int line, int n) const {
-        const float2* r = rows + line * RowPersist<PL>::LP;
-        const float2 xn = r[n];
-        const float2 xm = r[PL::M - n];
-        const float2 d = make_float2(xn.x - xm.x, xn.y + xm.y);
-        const float2 o = cmulc(d, __ldg(twW + n));   // global table (L1-resident)
-        return make_float2(xn.x + xm.x - o.y, xn.y - xm.y + o.x);
-    }
-};
-
-template <class PL>
-__global__ void __launch_bounds__(PL::ROW_T, 4) k4p_pair_rows(const float2* __restrict__ Q,
-                                                           unsigned long long* __restrict__ keys,
-                                                           int pair0, int npairs,
-                                                           const float2* __restrict__ tw2,
-                                                           const float2* __restrict__ twW) {
-    using RP = RowPersist<PL>;
-    extern __shared__ __align__(16) unsigned char smem_raw[];
-    constexpr int L = PL::ROW_L, T = PL::ROW_T, BPP = PL::H / L;
-    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + RP::OFF_BAR);
-    float2* tw2s = reinterpret_cast<float2*>(smem_raw + RP::OFF_TW2);
-    typename PL::RowX xc{reinterpret_cast<float2*>(smem_raw + RP::OFF_XCH4)};
-    float2* land = reinterpret_cast<float2*>(smem_raw + RP::OFF_LAND4);
-    const int nblk = npairs * BPP;
-    auto issue = [&](int blk, int buf) {
-        const int pl = blk / BPP, y0 = (blk - pl * BPP) * L;
-        const float2* src = Q + ((size_t)pl * PL::H + y0) * PL::WP;
-        mbar_arrive_expect_tx(&bar[buf], RP::QB);
-#pragma unroll
-        for (int line = 0; line < L; ++line)
-            bulk_g2s(land + line * RP::LP, src + (size_t)line * PL::WP, PL::WP * 8, &bar[buf]);
-    };
-    if (threadIdx.x == 0) {
-        mbar_init(&bar[0], 1);
-        mbar_init(&bar[1], 1);
-        fence_mbar_init();
-    }
-    for (int i = threadIdx.x; i < PL::ROW_TW2; i += T) tw2s[i] = __ldg(tw2 + i);
-    __syncthreads();
-    // Each CTA walks a contiguous range of row blocks (consecutive rows of mostly one pair):
-    // one landing buffer, refilled (TMA bulk copies) as soon as stage 1 consumed it; the
-    // running (max, index) of every thread carries across the blocks of a pair and is
-    // reduced (block reduction + one atomicMax) only when the pair changes.
-    const int b0 = (int)((long long)nblk * blockIdx.x / gridDim.x);
-    const int b1 = (int)((long long)nblk * (blockIdx.x + 1) / gridDim.x);
-    if (threadIdx.x == 0 && b0 < b1) issue(b0, 0);
-    ArgmaxDst acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
-    int cur = -1;
-    int k = 0;
-    for (int blk = b0; blk < b1; ++blk, ++k) {
-        const int pl = blk / BPP, y0 = (blk - pl * BPP) * L;
-        if (pl != cur) {                                   // block-uniform
-            if (cur >= 0) {
-                const unsigned long long best = block_max_u64<T>(acc.key());
-                if (threadIdx.x == 0) atomicMax(&keys[pair0 + cur], best);
-            }
-            cur = pl;
-            acc.best_v = -1.f;
-            acc.best_i = 0xFFFFFFFFu;
-        }
-        acc.row_base = y0;
-        mbar_wait(&bar[0], k & 1);
-        const int nxt = blk + 1;
-        C2RSmemSrc<PL> src{land, twW};
-        auto prefetch = [&]() {
-            if (threadIdx.x == 0 && nxt < b1) {
-                fence_proxy_async();
-                issue(nxt, 0);
-            }
-        };
-        FftRun<typename PL::Row, +1, L, T, RowMap, true>::run(src, xc, acc, tw2s, prefetch);
-        __syncthreads();   // exchange free for the next block
-    }
-    if (cur >= 0) {
-        const unsigned long long best = block_max_u64<T>(acc.key());
-        if (threadIdx.x == 0) atomicMax(&keys[pair0 + cur], best);
+    if constexpr (SURF) {
+        SurfaceDst dst{surf, y0, PL::W, scale};
+        FftRun<typename PL::Row, +1, L, T, RowMap>::run(src, xc, dst, tw2);
+    } else {
+        ArgmaxDst dst{-1.f, 0xFFFFFFFFu, y0, PL::W};
+        FftRun<typename PL::Row, +1, L, T, RowMap>::run(src, xc, dst, tw2);
+        const unsigned long long best = block_max_u64<T>(dst.key());
+        if (threadIdx.x == 0) atomicMax(&keys[pair0 + blockIdx.y], best);
     }
 }
 

@@ -1,20 +1,33 @@
 // stitch_api.cu — host side of the C ABI declared in include/stitch.h.
 //
-// Owns the device memory plan, the pair list (Fig. 4 order), the
-// launch schedule of K1..K6 (pciam_kernels.cuh) and the copy-in / copy-out.
-// The runtime is deliberately small: one stream, chunked launches sized so the
-// per-chunk intermediates (K1->K2 spectra, K3->K4 Q) stay in the 126 MB L2.
+// Owns the device memory plan, the step schedule and the copy-in / copy-out:
+//   * plan table: the compiled FFT plans per tile size (radices, CTA shapes);
+//   * layout: raw pixels and Q15 phasor spectra by SLOT (slot = local tile in the resident
+//     mode; a recycled pool slot in the bounded mode), the forward-chunk G
+//     and pair-chunk Q intermediates (0.38 / 0.94 GB at the default 64 / 160 chunks: they
+//     round-trip HBM), the pair list (Fig. 4), argmax keys, CCF moments, results;
+//   * schedule: a static list of forward chunks (K1 + K2, an H2D copy first when the tiles come
+//     from the host) and pair chunks (K3 + K4, then K5), decided at stitch_init and enqueued on
+//     internal streams (forward, pairs, CCF, H2D) joined by events, captured once into a CUDA
+//     graph and replayed on the caller's stream.  In the bounded mode the list interleaves the
+//     two kinds so that slots are recycled by reference count (the paper's pool);
+//   * multi-rank: an optional in-library NCCL halo exchange (libnccl.so.2 loaded at run time) on
+//     its own stream, overlapped with the interior pairs.
 #include <cuda.h>
 #include <cuda_runtime.h>
 #include <cudaTypedefs.h>
+#include <dlfcn.h>
+#include <nccl.h>   // types only: the functions are resolved with dlsym (no link-time NCCL)
 
 #include <algorithm>
 #include <cmath>
-#include <cstdlib>
 #include <cstdio>
 #include <cstring>
+#include <deque>
 #include <map>
+#include <mutex>
 #include <new>
+#include <set>
 #include <string>
 #include <type_traits>
 #include <vector>
@@ -22,69 +35,39 @@
 #include "../../include/stitch.h"
 #include "pciam_kernels.cuh"
 #include "pciam_fp64.cuh"
-#include "col_groups.cuh"
 
 using namespace stitch;
 
 namespace {
 
 // ------------------------------------------------------------ plan table ---
-// Compiled tile-size plans (Radix lists: the row transform is W/2 complex).
+// Compiled tile-size plans (the row transform is the W/2-point complex FFT of a real row).
 //            W     H     row radices          column radices      rowL rowT colP colT rowPad colPad
 using P1392 = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 8, 208, 0, 1>;
 using P256 = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 8, 128, 1, 1>;
 using P48 = Plan<48, 40, Radix<24, 24>, Radix<40, 40>, 8, 32, 8, 32, 0, 0>;
 using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 32, 8, 32, 0, 0>;
 
-// "Quad" column plans: the same transforms on 4-column panels, run by the persistent column
-// kernels with three CTAs per SM, each prefetching its next panel by TMA while it computes
-// (the one-panel-per-CTA kernels spend ~30 % of their stall samples waiting for their panel,
-// ncu r01c).  void: no quad variant for that plan.
-template <class PL> struct QuadOf { using type = void; };
-template <> struct QuadOf<P1392> {
-    using type = Plan<1392, 1040, Radix<696, 29, 24>, Radix<1040, 40, 26>, 4, 128, 4, 160, 0, 1>;
-};
-template <> struct QuadOf<P256> {
-    using type = Plan<256, 192, Radix<128, 16, 8>, Radix<192, 16, 12>, 8, 128, 4, 64, 1, 1>;
-};
-constexpr int QUAD_MINB = 3;
+// Tile rows per band of the resident pair order (a tile's spectrum and
+// pixels are reused by its <= 4 pairs while still in L2; bands of 1-8 measured, 3-4 best).
+constexpr int PAIR_BAND = 4;
 
 struct PlanOps {
-    int W, H, M, WC, WP, row_l, col_p;
-    int row_r0, row_r1, col_r0, col_r1;  // stage radices (r1 = 1: single stage)
-    cudaError_t (*setup)(int* grid_k1p, int* grid_k4p, int* grid_k1w, int* grid_k4w);
-    void (*k1p)(const uint16_t*, float2*, int, int, const float2*, const float2*, int, cudaStream_t);
-    void (*k4p)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
-                cudaStream_t);
+    int W, H, M, WC, WP, col_p;
+    int row_r0, row_r1, col_r0, col_r1;   // stage radices (r1 = 1: single stage)
+    cudaError_t (*setup)(int* grid_k1, int* grid_k4);
+    void (*k1)(const uint16_t*, float2*, int, int, const int32_t*, const float2*, const float2*,
+               int, cudaStream_t);
+    void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const int32_t*, const float2*,
+               bool, int, cudaStream_t);
+    void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
+    void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
+               cudaStream_t);
+    void (*k4s)(const float2*, float*, float, const float2*, const float2*, int, cudaStream_t);
     void (*k5)(const uint16_t*, const PairIdx*, const unsigned long long*, unsigned long long*, int,
                int, cudaStream_t);
-    void (*k2p)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, int,
-                cudaStream_t);
-    void (*k3p)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
-                cudaStream_t);
-    void (*k1w)(const uint16_t*, float2*, int, int, const float2*, const float2*, int, cudaStream_t);
-    void (*k4w)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
-                cudaStream_t);
-    void (*k1)(const uint16_t*, float2*, int, int, const float2*, const float2*, cudaStream_t);
-    void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, bool, int,
-               cudaStream_t);
-    void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
-               cudaStream_t);
-    void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*,
-               cudaStream_t);
-    // two-group column kernels (K2g/K3g); setup_g returns the grid (0: none for this plan)
-    cudaError_t (*setup_g)(int* grid);
-    void (*k2g)(const CUtensorMap&, uint32_t*, int, int, const float2*, int, cudaStream_t);
-    void (*k3g)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
-                cudaStream_t);
-    // quad column plans (col_p_q = 0: none); setup returns the persistent grid
-    int col_p_q;
-    cudaError_t (*setup_q)(int* grid);
-    void (*k2q)(const CUtensorMap&, float2*, uint32_t*, int, int, const float2*, int, cudaStream_t);
-    void (*k3q)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, int,
-                cudaStream_t);
     // fp64 path (f2, pciam_fp64.cuh)
-    int nblk64, colp64;
+    int nblk64;
     cudaError_t (*d_setup)();
     void (*d1)(const uint16_t*, double2*, int, int, const double2*, const double2*, cudaStream_t);
     void (*d2)(double2*, double2*, int, int, const double2*, bool, cudaStream_t);
@@ -102,155 +85,109 @@ cudaError_t max_smem(K* kernel, size_t bytes) {
                                 (int)cudaSharedmemCarveoutMaxShared);
 }
 
-// K4w runs the prime-factor row transform where the radices are coprime, unless STITCH_PFA=0
-inline bool pfa_enabled() {   // read per launch (launch sequences are captured once per ctx)
-    const char* env = std::getenv("STITCH_PFA");
-    return !(env && env[0] == '0');
-}
+// K4w runs the prime-factor (Good-Thomas) row transform where the two radices are coprime
+// (696 = 29 x 24), Stockham with stage-2 twiddles otherwise (128 = 16 x 8).
 template <class PL>
 constexpr bool k4_pfa_ok() {
-    if constexpr (RowWarp<PL>::OK) return RowWarp<PL>::RI::STAGES == 2 && WarpFftPfa<typename PL::Row, 1>::OK && RowWarp<PL>::PAD == 0;
-    else return false;
-}
-template <class PL>
-cudaError_t plan_setup(int* grid_k1p, int* grid_k4p, int* grid_k1w, int* grid_k4w) {
-    cudaError_t e;
-    *grid_k1w = *grid_k4w = 0;
-    using RP = RowPersist<PL>;
-    int dev = 0, sms = 0, nb = 0;
-    if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
-    if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
-        return e;
-    *grid_k1p = 0;
-    if (RP::K1_BULK) {
-        if ((e = max_smem(k1p_fwd_rows<PL>, RP::SMEM_K1)) != cudaSuccess) return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1p_fwd_rows<PL>, PL::ROW_T,
-                                                                RP::SMEM_K1)) != cudaSuccess)
-            return e;
-        *grid_k1p = nb * sms;
-    }
-    if ((e = max_smem(k4p_pair_rows<PL>, RP::SMEM_K4)) != cudaSuccess) return e;
-    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k4p_pair_rows<PL>, PL::ROW_T,
-                                                            RP::SMEM_K4)) != cudaSuccess)
-        return e;
-    *grid_k4p = nb * sms;
-    if ((e = max_smem(k5_ccf_moments<PL::W, PL::H>, k5_smem_bytes(PL::W))) != cudaSuccess) return e;
-    if ((e = max_smem(k2p_fwd_cols<PL, true>, PL::COLP_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(k2p_fwd_cols<PL, false>, PL::COLP_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(k3p_pair_cols<PL>, PL::COLP_SMEM)) != cudaSuccess) return e;
-    if constexpr (RowWarp<PL>::OK) {
-        using RW = RowWarp<PL>;
-        if ((e = max_smem(k1w_fwd_rows<PL>, RW::SMEM_K1)) != cudaSuccess) return e;
-        if ((e = max_smem(k4w_pair_rows<PL>, RW::SMEM_K4)) != cudaSuccess) return e;
-        if constexpr (k4_pfa_ok<PL>())
-            if ((e = max_smem(k4w_pair_rows<PL, true>, RW::SMEM_K4)) != cudaSuccess) return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1w_fwd_rows<PL>,
-                                                                32 * ROWW_WARPS, RW::SMEM_K1)) !=
-            cudaSuccess)
-            return e;
-        *grid_k1w = nb * sms;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k4w_pair_rows<PL>,
-                                                                32 * ROWW_WARPS, RW::SMEM_K4)) !=
-            cudaSuccess)
-            return e;
-        *grid_k4w = nb * sms;
-    }
-    if ((e = max_smem(k1_fwd_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(k4_pair_rows<PL>, PL::ROW_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(k2t_fwd_cols<PL, false>, PL::COL_SMEM)) != cudaSuccess) return e;
-    return max_smem(k3t_pair_cols<PL>, PL::COL_SMEM);
+    if constexpr (RowWarp<PL>::OK)
+        return RowWarp<PL>::RI::STAGES == 2 && WarpFftPfa<typename PL::Row, 1>::OK &&
+               RowWarp<PL>::PAD == 0;
+    else
+        return false;
 }
 
+#define CKE(x)                                     \
+    do {                                           \
+        cudaError_t e_ = (x);                      \
+        if (e_ != cudaSuccess) return e_;          \
+    } while (0)
+
 template <class PL>
-void launch_k1(const uint16_t* raw, float2* G, int t0, int nt, const float2* twM,
-               const float2* twW, cudaStream_t s) {
-    k1_fwd_rows<PL><<<dim3(PL::H / PL::ROW_L, nt), PL::ROW_T, PL::ROW_SMEM, s>>>(raw, G, t0,
-                                                                                 twM, twW);
+cudaError_t plan_setup(int* grid_k1, int* grid_k4) {
+    *grid_k1 = *grid_k4 = 0;
+    int dev = 0, sms = 0, nb = 0;
+    CKE(cudaGetDevice(&dev));
+    CKE(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    CKE(max_smem(k5_ccf_moments<PL::W, PL::H>, k5_smem_bytes(PL::W)));
+    CKE(max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM));
+    CKE(max_smem(k2t_fwd_cols<PL, false>, PL::COL_SMEM));
+    CKE(max_smem(k3t_pair_cols<PL>, PL::COL_SMEM));
+    if constexpr (RowWarp<PL>::OK) {
+        using RW = RowWarp<PL>;
+        constexpr bool PFA = k4_pfa_ok<PL>();
+        CKE(max_smem(k1w_fwd_rows<PL>, RW::SMEM_K1));
+        CKE(max_smem(k4w_pair_rows<PL, PFA>, RW::SMEM_K4));
+        CKE(max_smem(k4w_pair_rows<PL, PFA, true>, RW::SMEM_K4));
+        CKE(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1w_fwd_rows<PL>, 32 * ROWW_WARPS,
+                                                          RW::SMEM_K1));
+        *grid_k1 = nb * sms;
+        CKE(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k4w_pair_rows<PL, PFA>,
+                                                          32 * ROWW_WARPS, RW::SMEM_K4));
+        *grid_k4 = nb * sms;
+    } else {
+        CKE(max_smem(k1_fwd_rows<PL>, PL::ROW_SMEM));
+        CKE(max_smem(k4_pair_rows<PL>, PL::ROW_SMEM));
+        CKE(max_smem(k4_pair_rows<PL, true>, PL::ROW_SMEM));
+    }
+    return cudaSuccess;
+}
+
+// K1: warp-per-row persistent kernel (K1w) where the plan's row transform is a two-stage warp
+// FFT; one CTA per row block otherwise (the small test plans).
+template <class PL>
+void launch_k1(const uint16_t* raw, float2* G, int t0, int nt, const int32_t* fslot,
+               const float2* tw2, const float2* twW, int grid, cudaStream_t s) {
+    if constexpr (RowWarp<PL>::OK) {
+        const int need = (nt * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
+        k1w_fwd_rows<PL><<<grid < need ? grid : need, 32 * ROWW_WARPS, RowWarp<PL>::SMEM_K1, s>>>(
+            raw, G, t0, nt, fslot, tw2, twW);
+    } else {
+        k1_fwd_rows<PL><<<dim3(PL::H / PL::ROW_L, nt), PL::ROW_T, PL::ROW_SMEM, s>>>(
+            raw, G, t0, fslot, tw2, twW);
+    }
 }
 template <class PL>
-void launch_k2(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt, const float2* tw2,
-               bool phase_out, int ahead, cudaStream_t s) {
+void launch_k2(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt,
+               const int32_t* fslot, const float2* tw2, bool phase_out, int ahead, cudaStream_t s) {
     const dim3 grid(PL::WP / PL::COL_P, nt);
     if (phase_out)
-        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2, ahead);
+        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, fslot, tw2,
+                                                                     ahead);
     else
-        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, tw2, 0);
+        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, fslot, tw2,
+                                                                      0);
 }
 template <class PL>
 void launch_k3(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
-               const float2* tw2, int ahead, cudaStream_t s) {
-    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(
-        tmS, Q, pairs, p0, tw2, ahead);
+               const float2* tw2, cudaStream_t s) {
+    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(tmS, Q, pairs,
+                                                                                   p0, tw2);
 }
 template <class PL>
-void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const float2* twM,
-               const float2* twW, cudaStream_t s) {
-    k4_pair_rows<PL><<<dim3(PL::H / PL::ROW_L, np), PL::ROW_T, PL::ROW_SMEM, s>>>(Q, keys, p0,
-                                                                                  twM, twW);
-}
-
-template <class PL>
-void launch_k1p(const uint16_t* raw, float2* G, int t0, int nt, const float2* tw2,
-                const float2* twW, int grid, cudaStream_t s) {
-    const int nblk = nt * (PL::H / PL::ROW_L);
-    k1p_fwd_rows<PL><<<grid < nblk ? grid : nblk, PL::ROW_T, RowPersist<PL>::SMEM_K1, s>>>(
-        raw, G, t0, nt, tw2, twW);
-}
-template <class PL>
-void launch_k4p(const float2* Q, unsigned long long* keys, int p0, int np, const float2* tw2,
-                const float2* twW, int grid, cudaStream_t s) {
-    const int nblk = np * (PL::H / PL::ROW_L);
-    k4p_pair_rows<PL><<<grid < nblk ? grid : nblk, PL::ROW_T, RowPersist<PL>::SMEM_K4, s>>>(
-        Q, keys, p0, np, tw2, twW);
-}
-
-template <class PL>
-void launch_k2p(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt,
-                const float2* tw2, bool phase_out, int grid, cudaStream_t s) {
-    const int items = nt * (PL::WP / PL::COL_P);
-    const int gx = grid < items ? grid : items;
-    if (phase_out)
-        k2p_fwd_cols<PL, true><<<gx, PL::COL_T, PL::COLP_SMEM, s>>>(tmG, G, spec, t0, nt, tw2);
-    else
-        k2p_fwd_cols<PL, false><<<gx, PL::COL_T, PL::COLP_SMEM, s>>>(tmG, G, spec, t0, nt, tw2);
-}
-template <class PL>
-void launch_k3p(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
-                const float2* tw2, int grid, cudaStream_t s) {
-    const int items = np * (PL::WP / PL::COL_P);
-    const int gx = grid < items ? grid : items;
-    k3p_pair_cols<PL><<<gx, PL::COL_T, PL::COLP_SMEM, s>>>(tmS, Q, pairs, p0, np, tw2);
-}
-
-template <class PL>
-void launch_k1w(const uint16_t* raw, float2* G, int t0, int nt, const float2* tw2,
-                const float2* twW, int grid, cudaStream_t s) {
-    if constexpr (RowWarp<PL>::OK) {
-        const int warps = (nt * PL::H + 0) / 1;
-        const int need = (warps + ROWW_WARPS - 1) / ROWW_WARPS;
-        k1w_fwd_rows<PL><<<grid < need ? grid : need, 32 * ROWW_WARPS, RowWarp<PL>::SMEM_K1, s>>>(
-            raw, G, t0, nt, tw2, twW);
-    }
-}
-template <class PL>
-void launch_k4w(const float2* Q, unsigned long long* keys, int p0, int np, const float2* tw2,
-                const float2* twW, int grid, cudaStream_t s) {
-    if constexpr (k4_pfa_ok<PL>()) {
-        if (pfa_enabled()) {
-            const int need = (np * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
-            k4w_pair_rows<PL, true><<<grid < need ? grid : need, 32 * ROWW_WARPS,
-                                      RowWarp<PL>::SMEM_K4, s>>>(Q, keys, p0, np, tw2, twW);
-            return;
-        }
-    }
+void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const float2* tw2,
+               const float2* twW, int grid, cudaStream_t s) {
     if constexpr (RowWarp<PL>::OK) {
         const int need = (np * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
-        k4w_pair_rows<PL><<<grid < need ? grid : need, 32 * ROWW_WARPS, RowWarp<PL>::SMEM_K4, s>>>(
-            Q, keys, p0, np, tw2, twW);
+        k4w_pair_rows<PL, k4_pfa_ok<PL>()><<<grid < need ? grid : need, 32 * ROWW_WARPS,
+                                             RowWarp<PL>::SMEM_K4, s>>>(Q, keys, p0, np, tw2, twW);
+    } else {
+        k4_pair_rows<PL><<<dim3(PL::H / PL::ROW_L, np), PL::ROW_T, PL::ROW_SMEM, s>>>(Q, keys, p0,
+                                                                                      tw2, twW);
     }
 }
-
+template <class PL>
+void launch_k4s(const float2* Q, float* surf, float scale, const float2* tw2, const float2* twW,
+                int grid, cudaStream_t s) {
+    if constexpr (RowWarp<PL>::OK) {
+        const int need = (PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
+        k4w_pair_rows<PL, k4_pfa_ok<PL>(), true><<<grid < need ? grid : need, 32 * ROWW_WARPS,
+                                                   RowWarp<PL>::SMEM_K4, s>>>(
+            Q, nullptr, 0, 1, tw2, twW, surf, scale);
+    } else {
+        k4_pair_rows<PL, true><<<dim3(PL::H / PL::ROW_L, 1), PL::ROW_T, PL::ROW_SMEM, s>>>(
+            Q, nullptr, 0, tw2, twW, surf, scale);
+    }
+}
 template <class PL>
 void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long long* keys,
                unsigned long long* mom, int p0, int np, cudaStream_t s) {
@@ -258,110 +195,14 @@ void launch_k5(const uint16_t* raw, const PairIdx* pairs, const unsigned long lo
         raw, pairs, keys, mom, p0);
 }
 
-// ---- two-group column kernels
-template <class PL>
-cudaError_t setup_g(int* grid) {
-    *grid = 0;
-    using CG = ColGroups<PL>;
-    if constexpr (CG::OK) {
-        cudaError_t e;
-        int dev = 0, sms = 0, nb2 = 0, nb3 = 0;
-        if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
-        if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
-            return e;
-        if ((e = max_smem(k2g_fwd_cols<PL>, CG::SMEM)) != cudaSuccess) return e;
-        if ((e = max_smem(k3g_pair_cols<PL>, CG::SMEM)) != cudaSuccess) return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb2, k2g_fwd_cols<PL>, CG::NT,
-                                                                CG::SMEM)) != cudaSuccess)
-            return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb3, k3g_pair_cols<PL>, CG::NT,
-                                                                CG::SMEM)) != cudaSuccess)
-            return e;
-        *grid = std::min(nb2, nb3) * sms;
-    }
-    return cudaSuccess;
-}
-template <class PL>
-void launch_k2g(const CUtensorMap& tmG, uint32_t* spec, int t0, int nt, const float2* tw2,
-                int grid, cudaStream_t s) {
-    using CG = ColGroups<PL>;
-    if constexpr (CG::OK) {
-        const int items = nt * (PL::WP / PL::COL_P);
-        k2g_fwd_cols<PL><<<grid < items ? grid : items, CG::NT, CG::SMEM, s>>>(tmG, spec, t0, nt,
-                                                                              tw2);
-    }
-}
-template <class PL>
-void launch_k3g(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
-                const float2* tw2, int grid, cudaStream_t s) {
-    using CG = ColGroups<PL>;
-    if constexpr (CG::OK) {
-        const int items = np * (PL::WP / PL::COL_P);
-        k3g_pair_cols<PL><<<grid < items ? grid : items, CG::NT, CG::SMEM, s>>>(tmS, Q, pairs, p0,
-                                                                               np, tw2);
-    }
-}
-
-// ---- quad column plans
-template <class PL>
-cudaError_t setup_q(int* grid) {
-    *grid = 0;
-    using Q = typename QuadOf<PL>::type;
-    if constexpr (!std::is_void<Q>::value) {
-        cudaError_t e;
-        int dev = 0, sms = 0, nb2 = 0, nb3 = 0;
-        if ((e = cudaGetDevice(&dev)) != cudaSuccess) return e;
-        if ((e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev)) != cudaSuccess)
-            return e;
-        auto k2 = k2p_fwd_cols<Q, true, QUAD_MINB, true>;
-        auto k3 = k3p_pair_cols<Q, QUAD_MINB, true>;
-        if ((e = max_smem(k2, Q::COLP_TOFF)) != cudaSuccess) return e;
-        if ((e = max_smem(k3, Q::COLP_TOFF)) != cudaSuccess) return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb2, k2, Q::COL_T, Q::COLP_TOFF)) !=
-            cudaSuccess)
-            return e;
-        if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb3, k3, Q::COL_T, Q::COLP_TOFF)) !=
-            cudaSuccess)
-            return e;
-        *grid = std::min(nb2, nb3) * sms;
-    }
-    return cudaSuccess;
-}
-template <class PL>
-void launch_k2q(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt,
-                const float2* tw2, int grid, cudaStream_t s) {
-    using Q = typename QuadOf<PL>::type;
-    if constexpr (!std::is_void<Q>::value) {
-        const int items = nt * (Q::WP / Q::COL_P);
-        k2p_fwd_cols<Q, true, QUAD_MINB, true><<<grid < items ? grid : items, Q::COL_T,
-                                                 Q::COLP_TOFF, s>>>(tmG, G, spec, t0, nt, tw2);
-    }
-}
-template <class PL>
-void launch_k3q(const CUtensorMap& tmS, float2* Q_, const PairIdx* pairs, int p0, int np,
-                const float2* tw2, int grid, cudaStream_t s) {
-    using Q = typename QuadOf<PL>::type;
-    if constexpr (!std::is_void<Q>::value) {
-        const int items = np * (Q::WP / Q::COL_P);
-        k3p_pair_cols<Q, QUAD_MINB, true><<<grid < items ? grid : items, Q::COL_T, Q::COLP_TOFF,
-                                            s>>>(tmS, Q_, pairs, p0, np, tw2);
-    }
-}
-template <class PL>
-constexpr int quad_col_p() {
-    using Q = typename QuadOf<PL>::type;
-    if constexpr (std::is_void<Q>::value) return 0; else return Q::COL_P;
-}
-
 // ---- fp64 path launchers (f2)
 template <class PL>
 cudaError_t d_setup() {
     using P64 = Plan64<PL>;
-    cudaError_t e;
-    if ((e = max_smem(d1_fwd_rows<PL>, P64::ROW_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(d4_pair_rows<PL>, P64::ROW_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(d2_fwd_cols<PL, true>, P64::COL_SMEM)) != cudaSuccess) return e;
-    if ((e = max_smem(d2_fwd_cols<PL, false>, P64::COL_SMEM)) != cudaSuccess) return e;
+    CKE(max_smem(d1_fwd_rows<PL>, P64::ROW_SMEM));
+    CKE(max_smem(d4_pair_rows<PL>, P64::ROW_SMEM));
+    CKE(max_smem(d2_fwd_cols<PL, true>, P64::COL_SMEM));
+    CKE(max_smem(d2_fwd_cols<PL, false>, P64::COL_SMEM));
     return max_smem(d3_pair_cols<PL>, P64::COL_SMEM);
 }
 template <class PL>
@@ -397,15 +238,16 @@ void launch_d4(const double2* Q, double* pv, uint32_t* pi, int p0, int np, const
 
 template <class PL>
 PlanOps make_ops() {
-    return PlanOps{PL::W,       PL::H,         PL::M,          PL::WC,        PL::WP,
-                   PL::ROW_L,   PL::COL_P,     PL::RI::R0,     PL::RI::R1,    PL::CI::R0,
-                   PL::CI::R1,  plan_setup<PL>, launch_k1p<PL>, launch_k4p<PL>, launch_k5<PL>,
-                   launch_k2p<PL>, launch_k3p<PL>, launch_k1w<PL>, launch_k4w<PL>, launch_k1<PL>,
-                   launch_k2<PL>, launch_k3<PL>, launch_k4<PL>, setup_g<PL>, launch_k2g<PL>,
-                   launch_k3g<PL>, quad_col_p<PL>(), setup_q<PL>,
-                   launch_k2q<PL>, launch_k3q<PL>, Plan64<PL>::NBLK,
-                   Plan64<PL>::COL_P, d_setup<PL>, launch_d1<PL>, launch_d2<PL>, launch_d3<PL>,
-                   launch_d4<PL>};
+    PlanOps o;
+    o.W = PL::W; o.H = PL::H; o.M = PL::M; o.WC = PL::WC; o.WP = PL::WP; o.col_p = PL::COL_P;
+    o.row_r0 = PL::RI::R0; o.row_r1 = PL::RI::R1; o.col_r0 = PL::CI::R0; o.col_r1 = PL::CI::R1;
+    o.setup = plan_setup<PL>;
+    o.k1 = launch_k1<PL>; o.k2 = launch_k2<PL>; o.k3 = launch_k3<PL>; o.k4 = launch_k4<PL>;
+    o.k4s = launch_k4s<PL>; o.k5 = launch_k5<PL>;
+    o.nblk64 = Plan64<PL>::NBLK;
+    o.d_setup = d_setup<PL>;
+    o.d1 = launch_d1<PL>; o.d2 = launch_d2<PL>; o.d3 = launch_d3<PL>; o.d4 = launch_d4<PL>;
+    return o;
 }
 
 const PlanOps* find_plan(int W, int H) {
@@ -418,36 +260,106 @@ const PlanOps* find_plan(int W, int H) {
 
 size_t align256(size_t x) { return (x + 255) / 256 * 256; }
 
-// Dual pair schedule (STITCH_DUAL=1): K3 and K4 on separate streams with two Q slots, and K4's
-// persistent grid limited to STITCH_DUAL_K4 CTAs per SM (default 1), so a K4 chunk and the next
-// chunk's K3 share every SM: the issue-bound row kernel fills the column kernel's TMA waits.
-int dual_pairs_env() {
-    const char* e = std::getenv("STITCH_DUAL");
-    return e && e[0] == '1';
-}
-
 // twiddle tables: row stage-2 [r0*(r1-1)], column stage-2 [c0*(c1-1)], R2C/C2R w_W [W]
 // (slot counts rounded up to even, so every table starts 16-byte aligned for bulk copies)
 size_t tw_row(const PlanOps* o) { return ((size_t)o->row_r0 * (o->row_r1 - 1) + 1) & ~(size_t)1; }
 size_t tw_col(const PlanOps* o) { return ((size_t)o->col_r0 * (o->col_r1 - 1) + 1) & ~(size_t)1; }
 size_t tw_count(const PlanOps* o) { return tw_row(o) + tw_col(o) + o->W + 2; }
 
+// ------------------------------------------------------------- NCCL ----
+// Loaded at run time (the one torch ships is already in the process when torch is; else the
+// system's), so the library has no link-time NCCL dependency and single-GPU use needs none.
+struct NcclApi {
+    bool ok = false;
+    std::string err;
+    ncclResult_t (*get_unique_id)(ncclUniqueId*) = nullptr;
+    ncclResult_t (*comm_init_rank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+    ncclResult_t (*comm_destroy)(ncclComm_t) = nullptr;
+    ncclResult_t (*send)(const void*, size_t, ncclDataType_t, int, ncclComm_t,
+                         cudaStream_t) = nullptr;
+    ncclResult_t (*recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+    ncclResult_t (*group_start)() = nullptr;
+    ncclResult_t (*group_end)() = nullptr;
+    const char* (*error_string)(ncclResult_t) = nullptr;
+};
+
+const NcclApi& nccl() {
+    static NcclApi api;
+    static std::once_flag once;
+    std::call_once(once, [] {
+        void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) h = dlopen("libnccl.so", RTLD_NOW | RTLD_GLOBAL);
+        if (!h) {
+            const char* d = dlerror();
+            api.err = std::string("cannot load libnccl.so.2: ") + (d ? d : "?");
+            return;
+        }
+        auto sym = [&](const char* n) { return dlsym(h, n); };
+        api.get_unique_id = reinterpret_cast<decltype(api.get_unique_id)>(sym("ncclGetUniqueId"));
+        api.comm_init_rank = reinterpret_cast<decltype(api.comm_init_rank)>(sym("ncclCommInitRank"));
+        api.comm_destroy = reinterpret_cast<decltype(api.comm_destroy)>(sym("ncclCommDestroy"));
+        api.send = reinterpret_cast<decltype(api.send)>(sym("ncclSend"));
+        api.recv = reinterpret_cast<decltype(api.recv)>(sym("ncclRecv"));
+        api.group_start = reinterpret_cast<decltype(api.group_start)>(sym("ncclGroupStart"));
+        api.group_end = reinterpret_cast<decltype(api.group_end)>(sym("ncclGroupEnd"));
+        api.error_string = reinterpret_cast<decltype(api.error_string)>(sym("ncclGetErrorString"));
+        api.ok = api.get_unique_id && api.comm_init_rank && api.comm_destroy && api.send &&
+                 api.recv && api.group_start && api.group_end && api.error_string;
+        if (!api.ok) api.err = "libnccl.so.2 lacks a required symbol";
+    });
+    return api;
+}
+
+// ------------------------------------------------------------- layout ----
 struct Layout {
     int h_begin, t_begin, t_end, nlocal;
+    int nslots;          // tile slots (raw + spectrum): nlocal, or the pool size (bounded mode)
     int64_t npairs;
     int chunk_pairs, chunk_tiles;
-    int prec;   // 0 fp32, 1 fp64 (f2)
-    int q_slots;  // pair-chunk intermediates: 2 = K3(c+1) may run beside K4(c) (dual schedule)
+    int prec;            // 0 fp32, 1 fp64 (f2)
+    int pool;            // bounded mode (row f1)
+    int world, rank;
+    bool exchange;       // in-library NCCL halo exchange
     size_t off_raw, off_spec, off_g, off_q, off_pairs, off_keys, off_mom, off_res, off_tw,
-        off_part, total;
+        off_part, off_fslot, total;
 };
+
+// Balanced row-band partition: rank k of R owns [k nt/R, (k+1) nt/R).
+void band_of(int64_t nt, int rank, int world, int* b, int* e) {
+    *b = (int)(nt * rank / world);
+    *e = (int)(nt * (rank + 1) / world);
+}
+
+// Every halo lies in the previous rank's band (all bands but the last hold >= one tile row).
+bool exchange_feasible(int64_t nt, int m, int world) {
+    if (world < 2) return false;
+    for (int k = 0; k + 1 < world; ++k) {
+        int b, e;
+        band_of(nt, k, world, &b, &e);
+        if (e - b < m) return false;
+    }
+    return true;
+}
 
 stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L) {
     const int n = c->grid_rows, m = c->grid_cols;
     const int64_t nt = (int64_t)n * m;
+    L->world = c->world_size > 1 ? c->world_size : 1;
+    L->rank = L->world > 1 ? c->rank : 0;
+    if (L->world > 1 && (c->rank < 0 || c->rank >= c->world_size || nt < c->world_size))
+        return STITCH_ERR_INVALID_ARG;
     L->t_begin = c->tile_begin;
     L->t_end = c->tile_end ? c->tile_end : (int)nt;
+    if (L->world > 1 && c->tile_begin == 0 && c->tile_end == 0)
+        band_of(nt, L->rank, L->world, &L->t_begin, &L->t_end);
     if (L->t_begin < 0 || L->t_end > nt || L->t_begin >= L->t_end) return STITCH_ERR_INVALID_ARG;
+    L->exchange = false;
+    if (c->nccl_id) {
+        // the library owns the partition when it owns the exchange
+        if (L->world < 2 || c->tile_begin != 0 || c->tile_end != 0) return STITCH_ERR_INVALID_ARG;
+        if (c->precision != 0) return STITCH_ERR_UNSUPPORTED;   // the exchange moves Q15 spectra
+        L->exchange = exchange_feasible(nt, m, L->world);
+    }
     L->h_begin = L->t_begin - m > 0 ? L->t_begin - m : 0;
     L->nlocal = L->t_end - L->h_begin;
     int64_t np = 0;
@@ -455,27 +367,34 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     L->npairs = np;
     if (c->precision != 0 && c->precision != 1) return STITCH_ERR_INVALID_ARG;
     L->prec = c->precision;
+    if (c->pool_tiles < 0) return STITCH_ERR_INVALID_ARG;
+    L->pool = c->pool_tiles > 0;
+    if (L->pool && (L->prec || c->nccl_id)) return STITCH_ERR_UNSUPPORTED;
+    L->nslots = L->pool ? std::min(c->pool_tiles, L->nlocal) : L->nlocal;
     // fp64 chunks of 8 keep the 94 MB intermediate (8 x H x WP x 16 B at 1392x1040) in L2
     L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : (L->prec ? 8 : 160);
-    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : (L->prec ? 8 : 64);
+    L->chunk_tiles = c->chunk_tiles > 0
+                         ? c->chunk_tiles
+                         : (L->prec ? 8 : (L->pool ? std::max(1, std::min(64, L->nslots / 4)) : 64));
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
-    // resident spectrum: u32 Q15 unit phasor (fp32) or double2 unit phasor (fp64)
+    // spectrum by slot: u32 Q15 unit phasor (fp32) or double2 unit phasor (fp64)
     const size_t spec_el = L->prec ? sizeof(double2) : sizeof(uint32_t);
     const size_t cplx = L->prec ? sizeof(double2) : sizeof(float2);
+    const size_t np1 = (size_t)(np > 0 ? np : 1);
     size_t o = 0;
-    L->off_raw = o;   o += align256((size_t)L->nlocal * H * W * sizeof(uint16_t));
-    L->off_spec = o;  o += align256((size_t)L->nlocal * H * WP * spec_el);
+    L->off_raw = o;   o += align256((size_t)L->nslots * H * W * sizeof(uint16_t));
+    L->off_spec = o;  o += align256((size_t)L->nslots * H * WP * spec_el);
     L->off_g = o;     o += align256((size_t)L->chunk_tiles * H * WP * cplx);
-    L->q_slots = (!L->prec && dual_pairs_env()) ? 2 : 1;
-    L->off_q = o;     o += align256((size_t)L->q_slots * L->chunk_pairs * H * WP * cplx);
-    L->off_pairs = o; o += align256((size_t)(np > 0 ? np : 1) * sizeof(PairIdx));
-    L->off_keys = o;  o += align256((size_t)(np > 0 ? np : 1) * sizeof(unsigned long long));
-    L->off_mom = o;   o += align256((size_t)(np > 0 ? np : 1) * 20 * sizeof(unsigned long long));
-    L->off_res = o;   o += align256((size_t)(np > 0 ? np : 1) * sizeof(stitch_pair));
+    L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * cplx);
+    L->off_pairs = o; o += align256(np1 * sizeof(PairIdx));
+    L->off_keys = o;  o += align256(np1 * sizeof(unsigned long long));
+    L->off_mom = o;   o += align256(np1 * 20 * sizeof(unsigned long long));
+    L->off_res = o;   o += align256(np1 * sizeof(stitch_pair));
     L->off_tw = o;    o += align256((size_t)(tw_count(ops)) * cplx);
+    L->off_fslot = o; o += align256((size_t)L->nlocal * sizeof(int32_t));
     L->off_part = o;  // fp64 argmax partials: double [pairs][nblk] then u32 [pairs][nblk]
-    if (L->prec) o += align256((size_t)(np > 0 ? np : 1) * ops->nblk64 * (8 + 4));
+    if (L->prec) o += align256(np1 * ops->nblk64 * (8 + 4));
     L->total = o;
     return STITCH_OK;
 }
@@ -485,11 +404,46 @@ stitch_status check_config(const stitch_config* c, const PlanOps** ops) {
     if (c->grid_rows < 1 || c->grid_cols < 1 || c->tile_width < 2 || c->tile_height < 1)
         return STITCH_ERR_INVALID_ARG;
     if ((int64_t)c->grid_rows * c->grid_cols > (1 << 30)) return STITCH_ERR_INVALID_ARG;
+    if (c->flags & ~(uint32_t)(STITCH_FLAG_NO_GRAPH | STITCH_FLAG_SERIAL))
+        return STITCH_ERR_INVALID_ARG;
     *ops = find_plan(c->tile_width, c->tile_height);
     if (!*ops) return STITCH_ERR_UNSUPPORTED;
-    if ((int64_t)c->tile_width * c->tile_height > 0x7FFFFFFF) return STITCH_ERR_UNSUPPORTED;
     return STITCH_OK;
 }
+
+// Makes `dev` current for the lifetime of the guard and restores the caller's device.
+struct DevGuard {
+    int old = -1;
+    bool changed = false;
+    cudaError_t err = cudaSuccess;
+    explicit DevGuard(int dev) {
+        if ((err = cudaGetDevice(&old)) != cudaSuccess) return;
+        if (old != dev) {
+            err = cudaSetDevice(dev);
+            changed = err == cudaSuccess;
+        }
+    }
+    ~DevGuard() {
+        if (changed) cudaSetDevice(old);
+    }
+};
+
+// ----------------------------------------------------------- schedule ----
+struct FwdChunk {
+    int t0, nt;          // local tiles [t0, t0 + nt)
+    int wait_pair = -1;  // bounded mode: pair chunk whose K5 frees the last slot this chunk takes
+    int wait_fwd = -1;   // bounded mode: forward chunk whose K1 last read a slot this chunk takes
+};
+struct PairChunk {
+    int64_t p0;
+    int np;
+    int need;            // forward chunk (index in the step list) completing its tiles; -1: none
+    bool boundary;       // reads a halo spectrum received from rank-1
+};
+struct Op {
+    enum Kind : int8_t { FWD, PAIR, EXCH } kind;
+    int idx;
+};
 
 }  // namespace
 
@@ -503,51 +457,52 @@ struct stitch_ctx {
     char* mem = nullptr;
     bool own_mem = false;
     uint16_t* raw;
-    uint32_t* spec;                   // resident Q15 phasor spectra [nlocal][H][WP]
+    uint32_t* spec;                   // Q15 phasor spectra by slot [nslots][H][WP]
     float2 *G, *Q, *twM, *twH, *twW;  // chunk intermediates, twiddles
-    float2* Q2 = nullptr;             // second pair-chunk slot (dual schedule)
-    int grid_k4w_dual = 0;            // K4w grid beside K3 (dual schedule)
-    cudaStream_t s_pair4 = nullptr;   // K4 stream (dual schedule)
-    std::vector<cudaEvent_t> ev_k3;   // per pair chunk: its Q is complete (dual schedule)
+    int32_t* fslot;                   // slot of each local tile
     int prec = 0;                     // 1: fp64 path (f2): the buffers below are used instead
     double2 *Gd = nullptr, *Qd = nullptr, *Ud = nullptr;   // Ud: resident unit phasors
     double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
     double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
     uint32_t* part_i = nullptr;
     CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (Q15 phasors)
-    CUtensorMap tmG4, tmS4;           // the same with the quad plans' 4-column boxes
-    int grid_colq = 0;                // quad persistent column kernels (0: not used)
-    int grid_colg = 0;                // two-group column kernels (0: not used)
-    int col_ahead = 0;                // K2 L2 prefetch distance in CTAs (0: off)
-    int col_ahead3 = 0;               // K3 L2 prefetch distance in CTAs (0: off)
+    int grid_k1 = 0, grid_k4 = 0;     // persistent grids of the warp row kernels (0: CTA kernels)
+    int col_ahead = 0;                // K2 L2 prefetch distance in CTAs (one wave)
     PairIdx* pairs;
     unsigned long long *keys, *mom;
     stitch_pair* res;
+    std::vector<PairIdx> pairs_h;
     std::vector<int32_t> pair_tile;   // global tile index (B) of each pair
     std::vector<int8_t> pair_kind;    // 0 west, 1 north
+    std::vector<int32_t> fslot_h;
     std::vector<stitch_pair> res_h;
+    // static schedule (stitch_init)
+    std::vector<FwdChunk> fwd;
+    std::vector<PairChunk> pch;
+    std::vector<Op> ops_step;         // the whole step in enqueue order
+    int64_t n_interior = 0;           // pairs [0, n_interior) need no halo spectrum
+    int c_boundary = 0;               // first pair chunk of the boundary pairs
+    // NCCL halo exchange (L.exchange)
+    ncclComm_t comm = nullptr;
+    int send_lt = 0, send_cnt = 0, recv_lt = 0, recv_cnt = 0;   // local tile ranges
     bool loaded = false, computed = false;
     int64_t launches = 0;
-    int grid_k1p = 0, grid_k4p = 0;   // persistent-kernel grids (0: use the non-persistent kernel)
-    int grid_colp = 0;                // persistent column kernels (K2p/K3p): one CTA per SM
-    int grid_k1w = 0, grid_k4w = 0;   // warp-per-line row kernels (0: not used)
-    // CUDA graphs of the launch sequences (captured on first use on an internal stream,
-    // replayed on the caller's stream): one graph launch per step instead of ~700 launches
-    bool use_graph = true;
+    bool use_graph = true, concurrent = true;
     cudaStream_t cap_stream = nullptr;
     struct GraphRec {
-        cudaGraphExec_t exec;
-        int64_t launches;
+        cudaGraphExec_t exec = nullptr;
+        cudaGraph_t graph = nullptr;
+        int64_t launches = 0;
+        const char* src = nullptr;    // host source baked into the H2D nodes (nullptr: none)
+        std::vector<cudaGraphNode_t> h2d;
+        std::vector<cudaMemcpy3DParms> h2d_p;
     };
     std::map<uint64_t, GraphRec> graphs;
-    // concurrent schedule (timing off): forward chunks, pair chunks and CCF chunks on three
-    // internal streams joined by events, so compute-bound and memory-bound kernels overlap
-    bool concurrent = true;
-    cudaStream_t s_fwd = nullptr, s_pair = nullptr, s_ccf = nullptr, s_h2d = nullptr;
-    std::vector<cudaEvent_t> ev_h2d;          // per forward chunk: its tiles have landed
-    std::vector<cudaEvent_t> ev_fwd, ev_k4;   // per forward chunk / per pair chunk
-    cudaEvent_t ev_fork = nullptr, ev_join[3] = {nullptr, nullptr, nullptr};
-    std::vector<int> pair_need;               // forward chunk completing each pair chunk's tiles
+    cudaStream_t s_fwd = nullptr, s_pair = nullptr, s_ccf = nullptr, s_h2d = nullptr,
+                 s_comm = nullptr;
+    std::vector<cudaEvent_t> ev_h2d, ev_fwd, ev_k4, ev_k5;
+    cudaEvent_t ev_halo = nullptr, ev_fork = nullptr;
+    cudaEvent_t ev_join[5] = {nullptr, nullptr, nullptr, nullptr, nullptr};
     int timing = 0;  // 0 off, 1 per-stage events, 2 per-stage + per-launch events,
                      // 3 timeline of the concurrent schedule (events around every launch)
     struct TlRec {
@@ -595,7 +550,7 @@ static cudaError_t tl_wrap(stitch_ctx* ctx, cudaStream_t s, int si, int kid, F l
     return cudaSuccess;
 }
 
-// Per-launch event (timing mode 2): kid 0..5 = K1..K6.
+// Per-launch event (timing mode 2): kid 0..5 = K1..K6 (-1: not a kernel).
 static cudaError_t mark(stitch_ctx* ctx, int kid) {
     if (ctx->timing < 2) return cudaSuccess;
     const size_t i = ctx->kkind.size();
@@ -621,11 +576,513 @@ static stitch_status cuda_fail(stitch_ctx* ctx, cudaError_t e, const char* where
                 std::string(where) + ": " + cudaGetErrorString(e));
 }
 
-#define CK(call, where)                                   \
-    do {                                                  \
-        cudaError_t e_ = (call);                          \
+static stitch_status nccl_fail(stitch_ctx* ctx, ncclResult_t r, const char* where) {
+    const NcclApi& api = nccl();
+    return fail(ctx, STITCH_ERR_NCCL,
+                std::string(where) + ": " + (api.error_string ? api.error_string(r) : "nccl error"));
+}
+
+#define CK(call, where)                                          \
+    do {                                                         \
+        cudaError_t e_ = (call);                                 \
         if (e_ != cudaSuccess) return cuda_fail(ctx, e_, where); \
     } while (0)
+
+#define GUARD(ctx)                                                          \
+    DevGuard guard_((ctx)->cfg.device);                                     \
+    if (guard_.err != cudaSuccess) return cuda_fail(ctx, guard_.err, "set device")
+
+// ------------------------------------------------ schedule construction ----
+// Resident mode: forward chunks in tile order; pairs in bands of PAIR_BAND tile rows
+// (column-major inside a band), interior pairs first, then the boundary pairs (tile A in the
+// halo, which an NCCL exchange may still be delivering); every pair chunk waits for the
+// forward chunk that completes its tiles.
+static void build_resident(stitch_ctx* ctx) {
+    const Layout& L = ctx->L;
+    const int m = ctx->m, hb = L.h_begin, tbl = L.t_begin - hb;
+    const int ct = L.chunk_tiles, cp = L.chunk_pairs;
+    ctx->fslot_h.resize(L.nlocal);
+    for (int i = 0; i < L.nlocal; ++i) ctx->fslot_h[i] = i;
+    // the step's forward chunks: every local tile, or only the owned ones when the halo's
+    // spectra arrive by NCCL
+    const int f0 = L.exchange ? tbl : 0;
+    std::vector<int> chunk_of(L.nlocal, -1);
+    for (int t0 = f0; t0 < L.nlocal; t0 += ct) {
+        const int nt = std::min(ct, L.nlocal - t0);
+        for (int i = 0; i < nt; ++i) chunk_of[t0 + i] = (int)ctx->fwd.size();
+        ctx->fwd.push_back(FwdChunk{t0, nt});
+    }
+    std::vector<int> order;
+    for (int t = L.t_begin; t < L.t_end; ++t) order.push_back(t);
+    std::stable_sort(order.begin(), order.end(), [m](int a, int b) {
+        const int ra = a / m, rb = b / m, ba = ra / PAIR_BAND, bb = rb / PAIR_BAND;
+        if (ba != bb) return ba < bb;
+        if (a % m != b % m) return a % m < b % m;
+        return ra < rb;
+    });
+    struct P { int a, b, t; int8_t kind; };
+    std::vector<P> inner, bound;
+    for (const int t : order) {
+        const int r = t / m, c = t % m;
+        if (c >= 1) (t - 1 >= L.t_begin ? inner : bound).push_back(P{t - 1 - hb, t - hb, t, 0});
+        if (r >= 1) (t - m >= L.t_begin ? inner : bound).push_back(P{t - m - hb, t - hb, t, 1});
+    }
+    ctx->n_interior = (int64_t)inner.size();
+    auto emit = [&](const std::vector<P>& v, bool boundary) {
+        for (size_t i = 0; i < v.size(); i += (size_t)cp) {
+            PairChunk pc{(int64_t)ctx->pairs_h.size(), (int)std::min(v.size() - i, (size_t)cp), -1,
+                         boundary};
+            for (size_t j = i; j < i + (size_t)pc.np; ++j) {
+                const P& q = v[j];
+                ctx->pairs_h.push_back(PairIdx{q.a, q.b});
+                ctx->pair_tile.push_back(q.t);
+                ctx->pair_kind.push_back(q.kind);
+                pc.need = std::max(pc.need, std::max(chunk_of[q.a], chunk_of[q.b]));
+            }
+            ctx->pch.push_back(pc);
+        }
+    };
+    emit(inner, false);
+    ctx->c_boundary = (int)ctx->pch.size();
+    emit(bound, true);
+    for (int f = 0; f < (int)ctx->fwd.size(); ++f) ctx->ops_step.push_back(Op{Op::FWD, f});
+    if (L.exchange) ctx->ops_step.push_back(Op{Op::EXCH, 0});
+    for (int c = 0; c < (int)ctx->pch.size(); ++c) ctx->ops_step.push_back(Op{Op::PAIR, c});
+}
+
+// Bounded mode (row f1; the paper's pool of reusable buffers with per-tile reference counts,
+// P:L1082-1110): tiles are transformed in row-major forward chunks into free slots of a
+// fixed pool; each tile's count starts at the number of pairs that read it (<= 4: west, east,
+// north, south, Fig. 4) and drops as pair chunks are scheduled; a slot whose count reaches 0
+// is free again once that pair chunk's K5 (the last reader of its pixels and, through the
+// K3 -> K4 -> K5 chain, of its spectrum) has finished -- the forward chunk that takes it
+// next waits for that event.  Pairs are scheduled as soon as both tiles are ready, in chunks
+// of up to chunk_pairs, earlier when the pool runs dry.  The simulation runs once, here, so
+// the step is a static interleaving of forward and pair chunks (graph-capturable).
+static bool build_pooled(stitch_ctx* ctx, std::string* why) {
+    const Layout& L = ctx->L;
+    const int m = ctx->m, hb = L.h_begin, nl = L.nlocal;
+    const int ct = L.chunk_tiles, cp = L.chunk_pairs;
+    std::vector<int> refs(nl, 0);
+    for (int t = L.t_begin; t < L.t_end; ++t) {
+        const int lt = t - hb;
+        if (t % m >= 1) { ++refs[lt]; ++refs[lt - 1]; }
+        if (t / m >= 1) { ++refs[lt]; ++refs[lt - m]; }
+    }
+    ctx->fslot_h.assign(nl, -1);
+    std::set<int> free_slots;
+    for (int s = 0; s < L.nslots; ++s) free_slots.insert(s);
+    std::vector<int> tag_pair(L.nslots, -1), tag_fwd(L.nslots, -1);
+    struct P { int a, b, t; int8_t kind; };   // local tiles
+    std::deque<P> pending;
+    int cur_f = -1;
+    auto release = [&](int lt, int tp, int tf) {
+        const int s = ctx->fslot_h[lt];
+        tag_pair[s] = tp;
+        tag_fwd[s] = tf;
+        free_slots.insert(s);
+    };
+    auto emit_pairs = [&](int k) {
+        const int c = (int)ctx->pch.size();
+        ctx->pch.push_back(PairChunk{(int64_t)ctx->pairs_h.size(), k, cur_f, false});
+        ctx->ops_step.push_back(Op{Op::PAIR, c});
+        for (int i = 0; i < k; ++i) {
+            const P q = pending.front();
+            pending.pop_front();
+            ctx->pairs_h.push_back(PairIdx{ctx->fslot_h[q.a], ctx->fslot_h[q.b]});
+            ctx->pair_tile.push_back(q.t);
+            ctx->pair_kind.push_back(q.kind);
+            for (const int lt : {q.a, q.b})
+                if (--refs[lt] == 0) release(lt, c, -1);
+        }
+    };
+    for (int t0 = 0; t0 < nl; t0 += ct) {
+        const int nt = std::min(ct, nl - t0);
+        while ((int)free_slots.size() < nt) {
+            if (pending.empty()) {
+                *why = "pool_tiles too small for the grid: every slot holds a tile still awaiting a "
+                       "pair (need about one tile row + one forward chunk of slots)";
+                return false;
+            }
+            emit_pairs(std::min((int)pending.size(), cp));
+        }
+        FwdChunk fc{t0, nt};
+        for (int i = 0; i < nt; ++i) {
+            const int s = *free_slots.begin();
+            free_slots.erase(free_slots.begin());
+            ctx->fslot_h[t0 + i] = s;
+            fc.wait_pair = std::max(fc.wait_pair, tag_pair[s]);
+            fc.wait_fwd = std::max(fc.wait_fwd, tag_fwd[s]);
+        }
+        cur_f = (int)ctx->fwd.size();
+        ctx->fwd.push_back(fc);
+        ctx->ops_step.push_back(Op{Op::FWD, cur_f});
+        for (int lt = t0; lt < t0 + nt; ++lt) {
+            const int t = lt + hb;
+            if (t >= L.t_begin) {   // pairs with tile B = t become ready (tile A < B is ready)
+                if (t % m >= 1) pending.push_back(P{lt - 1, lt, t, 0});
+                if (t / m >= 1) pending.push_back(P{lt - m, lt, t, 1});
+            }
+            if (refs[lt] == 0) release(lt, -1, cur_f);   // read by no pair (e.g. a 1x1 grid)
+        }
+        while ((int)pending.size() >= cp) emit_pairs(cp);
+    }
+    while (!pending.empty()) emit_pairs(std::min((int)pending.size(), cp));
+    ctx->n_interior = (int64_t)ctx->pairs_h.size();
+    ctx->c_boundary = (int)ctx->pch.size();
+    return true;
+}
+
+// ------------------------------------------------------------ enqueue ----
+static bool serial(const stitch_ctx* ctx) {
+    return !ctx->concurrent || ctx->timing == 1 || ctx->timing == 2;
+}
+
+// Host-to-device copy of a forward chunk's tiles into their slots (runs of consecutive slots
+// coalesced into one copy).  src: the caller's buffer, tile 0 = local tile 0.
+static stitch_status copy_chunk_in(stitch_ctx* ctx, const FwdChunk& fc, const uint16_t* src,
+                                   cudaStream_t s) {
+    const size_t tile_px = (size_t)ctx->H * ctx->W;
+    for (int i = 0; i < fc.nt;) {
+        int j = i + 1;
+        while (j < fc.nt && ctx->fslot_h[fc.t0 + j] == ctx->fslot_h[fc.t0 + i] + (j - i)) ++j;
+        CK(cudaMemcpyAsync(ctx->raw + (size_t)ctx->fslot_h[fc.t0 + i] * tile_px,
+                           src + (size_t)(fc.t0 + i) * tile_px, (size_t)(j - i) * tile_px * 2,
+                           cudaMemcpyHostToDevice, s),
+           "tile H2D");
+        i = j;
+    }
+    return STITCH_OK;
+}
+
+static void launch_fwd(stitch_ctx* ctx, int t0, int nt, cudaStream_t s, int si) {
+    const PlanOps* o = ctx->ops;
+    tl_wrap(ctx, s, si, 0, [&] {
+        o->k1(ctx->raw, ctx->G, t0, nt, ctx->fslot, ctx->twM, ctx->twW, ctx->grid_k1, s);
+    });
+    mark(ctx, 0);
+    tl_wrap(ctx, s, si, 1, [&] {
+        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->fslot, ctx->twH, true, ctx->col_ahead, s);
+    });
+    mark(ctx, 1);
+    ctx->launches += 2;
+}
+
+// The halo exchange (rank k: send the spectra of its last tile row to k+1, receive its halo
+// row from k-1), one NCCL group on stream s.
+static stitch_status exchange(stitch_ctx* ctx, cudaStream_t s) {
+    const NcclApi& api = nccl();
+    const size_t per = (size_t)ctx->H * ctx->ops->WP * sizeof(uint32_t);
+    ncclResult_t r;
+    if ((r = api.group_start()) != ncclSuccess) return nccl_fail(ctx, r, "ncclGroupStart");
+    if (ctx->send_cnt > 0 &&
+        (r = api.send(ctx->spec + (size_t)ctx->fslot_h[ctx->send_lt] * (per / 4),
+                      (size_t)ctx->send_cnt * per, ncclUint8, ctx->L.rank + 1, ctx->comm, s)) !=
+            ncclSuccess) {
+        api.group_end();
+        return nccl_fail(ctx, r, "ncclSend");
+    }
+    if (ctx->recv_cnt > 0 &&
+        (r = api.recv(ctx->spec + (size_t)ctx->fslot_h[ctx->recv_lt] * (per / 4),
+                      (size_t)ctx->recv_cnt * per, ncclUint8, ctx->L.rank - 1, ctx->comm, s)) !=
+            ncclSuccess) {
+        api.group_end();
+        return nccl_fail(ctx, r, "ncclRecv");
+    }
+    if ((r = api.group_end()) != ncclSuccess) return nccl_fail(ctx, r, "ncclGroupEnd");
+    return STITCH_OK;
+}
+
+// Enqueue a list of forward / exchange / pair ops (the whole step or a part of it) on the
+// context's streams.  Concurrent: forward chunks on s_fwd (their H2D on s_h2d), pair chunks'
+// K3 + K4 on s_pair and K5 on s_ccf, the exchange on s_comm, joined by events; serial (timing
+// modes 1-2, or STITCH_FLAG_SERIAL): everything on the context stream in list order.
+// src: host tiles (local tile 0 first) copied per forward chunk, or nullptr (resident).
+// [pa, pb): the pairs these ops cover (keys/moments cleared first, K6 over them last).
+static stitch_status enqueue_ops(stitch_ctx* ctx, const std::vector<Op>& ops, const uint16_t* src,
+                                 bool wait_fwd, int64_t pa, int64_t pb) {
+    const PlanOps* o = ctx->ops;
+    cudaStream_t m = ctx->stream;
+    const bool ser = serial(ctx);
+    cudaStream_t sf = ser ? m : ctx->s_fwd, sp = ser ? m : ctx->s_pair, sk = ser ? m : ctx->s_ccf;
+    cudaStream_t sh = ser ? m : ctx->s_h2d, sc = ser ? m : ctx->s_comm;
+    const int64_t np = pb - pa;
+    if (np > 0) {
+        CK(cudaMemsetAsync(ctx->keys + pa, 0, (size_t)np * sizeof(unsigned long long), m), "memset");
+        CK(cudaMemsetAsync(ctx->mom + pa * 20, 0, (size_t)np * 20 * sizeof(unsigned long long), m),
+           "memset");
+    }
+    if (ctx->timing == 3) {
+        ctx->tl.clear();
+        ctx->tl_used = 0;
+        CK(tl_event(ctx, &ctx->tl_origin), "event");
+        CK(cudaEventRecord(ctx->tl_origin, m), "event");
+    }
+    if (!ser) {
+        CK(cudaEventRecord(ctx->ev_fork, m), "fork");
+        for (cudaStream_t st : {sf, sp, sk, sh, sc})
+            if (st) CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
+    }
+    int waited = -1, last_fwd = -1;
+    bool halo_waited = false, any_k4 = false;
+    for (const Op& op : ops) {
+        if (op.kind == Op::FWD) {
+            const FwdChunk& fc = ctx->fwd[op.idx];
+            if (!ser) {   // bounded mode: the slots this chunk takes must be free
+                if (fc.wait_pair >= 0) {
+                    CK(cudaStreamWaitEvent(sf, ctx->ev_k5[fc.wait_pair], 0), "wait slot");
+                    if (src) CK(cudaStreamWaitEvent(sh, ctx->ev_k5[fc.wait_pair], 0), "wait slot");
+                }
+                if (fc.wait_fwd >= 0 && src)
+                    CK(cudaStreamWaitEvent(sh, ctx->ev_fwd[fc.wait_fwd], 0), "wait slot");
+            }
+            if (src) {
+                stitch_status st = copy_chunk_in(ctx, fc, src, sh);
+                if (st != STITCH_OK) return st;
+                if (!ser) {
+                    CK(cudaEventRecord(ctx->ev_h2d[op.idx], sh), "event");
+                    CK(cudaStreamWaitEvent(sf, ctx->ev_h2d[op.idx], 0), "wait H2D");
+                }
+            }
+            launch_fwd(ctx, fc.t0, fc.nt, sf, 0);
+            if (!ser) CK(cudaEventRecord(ctx->ev_fwd[op.idx], sf), "event");
+            last_fwd = op.idx;
+        } else if (op.kind == Op::EXCH) {
+            if (!ser && last_fwd >= 0) CK(cudaStreamWaitEvent(sc, ctx->ev_fwd[last_fwd], 0), "wait");
+            stitch_status st = exchange(ctx, sc);
+            if (st != STITCH_OK) return st;
+            if (!ser) CK(cudaEventRecord(ctx->ev_halo, sc), "event");
+        } else {
+            const PairChunk& pc = ctx->pch[op.idx];
+            if (!ser) {
+                if (wait_fwd && pc.need > waited) {
+                    CK(cudaStreamWaitEvent(sp, ctx->ev_fwd[pc.need], 0), "wait forward");
+                    waited = pc.need;
+                }
+                if (pc.boundary && ctx->L.exchange && !halo_waited) {
+                    CK(cudaStreamWaitEvent(sp, ctx->ev_halo, 0), "wait halo");
+                    halo_waited = true;
+                }
+            }
+            if (ctx->timing && !any_k4 && ser) CK(cudaEventRecord(ctx->ev[1], m), "event");
+            any_k4 = true;
+            tl_wrap(ctx, sp, 1, 2, [&] {
+                o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)pc.p0, pc.np, ctx->twH, sp);
+            });
+            mark(ctx, 2);
+            tl_wrap(ctx, sp, 1, 3, [&] {
+                o->k4(ctx->Q, ctx->keys, (int)pc.p0, pc.np, ctx->twM, ctx->twW, ctx->grid_k4, sp);
+            });
+            mark(ctx, 3);
+            if (!ser) {
+                CK(cudaEventRecord(ctx->ev_k4[op.idx], sp), "event");
+                CK(cudaStreamWaitEvent(sk, ctx->ev_k4[op.idx], 0), "wait k4");
+            }
+            tl_wrap(ctx, sk, 2, 4, [&] {
+                o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)pc.p0, pc.np, sk);
+            });
+            mark(ctx, 4);
+            if (!ser) CK(cudaEventRecord(ctx->ev_k5[op.idx], sk), "event");
+            ctx->launches += 3;
+        }
+    }
+    if (ctx->timing && ser) CK(cudaEventRecord(ctx->ev[2], m), "event");
+    if (np > 0) {
+        tl_wrap(ctx, sk, 2, 5, [&] {
+            k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
+                ctx->keys + pa, ctx->mom + pa * 20, ctx->res + pa, ctx->H, ctx->W, (int)np,
+                (double)ctx->W * ctx->H * NCPS_Q15_SCALE);
+        });
+        mark(ctx, 5);
+        ctx->launches += 1;
+    }
+    CK(cudaGetLastError(), "launch");
+    if (!ser) {
+        int j = 0;
+        for (cudaStream_t st : {sf, sp, sk, sh, sc}) {
+            if (!st) continue;
+            CK(cudaEventRecord(ctx->ev_join[j], st), "join");
+            CK(cudaStreamWaitEvent(m, ctx->ev_join[j], 0), "join wait");
+            ++j;
+        }
+    }
+    return STITCH_OK;
+}
+
+// fp64 path (f2): serial on the context stream -- D1 + D2 per forward chunk, D3 + D4 per pair
+// chunk (per-block argmax partials), D5 reducing them into the K5/K6 key, K5 per chunk, K6.
+static stitch_status enqueue_fp64(stitch_ctx* ctx, bool forward, bool pairs) {
+    const PlanOps* o = ctx->ops;
+    cudaStream_t s = ctx->stream;
+    if (forward) {
+        for (const FwdChunk& fc : ctx->fwd) {
+            o->d1(ctx->raw, ctx->Gd, fc.t0, fc.nt, ctx->twMd, ctx->twWd, s);
+            CK(mark(ctx, 0), "event");
+            o->d2(ctx->Gd, ctx->Ud, fc.t0, fc.nt, ctx->twHd, true, s);
+            CK(mark(ctx, 1), "event");
+            ctx->launches += 2;
+        }
+    }
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], s), "event");
+    const int64_t np = ctx->L.npairs;
+    if (pairs && np > 0) {
+        CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), s), "memset");
+        for (const PairChunk& pc : ctx->pch) {
+            o->d3(ctx->Ud, ctx->Qd, ctx->pairs, (int)pc.p0, pc.np, ctx->twHd, s);
+            CK(mark(ctx, 2), "event");
+            o->d4(ctx->Qd, ctx->part_v, ctx->part_i, (int)pc.p0, pc.np, ctx->twMd, ctx->twWd, s);
+            CK(mark(ctx, 3), "event");
+            ctx->launches += 2;
+        }
+        d5_argmax_keys<<<(unsigned)((np + 7) / 8), 256, 0, s>>>(ctx->part_v, ctx->part_i,
+                                                               ctx->keys, o->nblk64, (int)np);
+        CK(mark(ctx, 3), "event");
+        ctx->launches += 1;
+        if (ctx->timing) CK(cudaEventRecord(ctx->ev[2], s), "event");
+        for (const PairChunk& pc : ctx->pch) {
+            o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)pc.p0, pc.np, s);
+            CK(mark(ctx, 4), "event");
+            ctx->launches += 1;
+        }
+        k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, s>>>(
+            ctx->keys, ctx->mom, ctx->res, ctx->H, ctx->W, (int)np, (double)ctx->W * ctx->H);
+        CK(mark(ctx, 5), "event");
+        ctx->launches += 1;
+    }
+    CK(cudaGetLastError(), "fp64 launch");
+    return STITCH_OK;
+}
+
+// Start of a step: reset launch counters and (timing modes) record the start events.
+static stitch_status step_begin(stitch_ctx* ctx) {
+    cudaStream_t s = ctx->stream;
+    ctx->launches = 0;
+    ctx->kkind.clear();
+    ctx->computed = false;
+    if (ctx->timing >= 2) {
+        if (ctx->kev.empty()) {
+            ctx->kev.resize(1024, nullptr);
+            for (auto& e : ctx->kev) CK(cudaEventCreate(&e), "event create");
+        }
+        CK(cudaEventRecord(ctx->kev[0], s), "event");
+    }
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[0], s), "event");
+    return STITCH_OK;
+}
+
+static stitch_status step_end(stitch_ctx* ctx) {
+    if (ctx->timing) CK(cudaEventRecord(ctx->ev[3], ctx->stream), "event");
+    return STITCH_OK;
+}
+
+extern "C++" {
+// Enqueue `body` (which launches on ctx->stream) directly, or -- graph mode, no event
+// timing, no NCCL -- as a CUDA graph captured once per key on the internal capture stream
+// and replayed on the caller's stream.  Every launch parameter (pointers, tensor maps, the
+// schedule) is fixed per context, so a replay is exactly the captured sequence; only the
+// host source of the H2D copies may change between replays (`src`): the graph's memcpy nodes
+// are then re-pointed in place (cudaGraphExecMemcpyNodeSetParams), so one executable graph
+// serves any number of caller buffers.
+template <class F>
+static stitch_status run_graphed(stitch_ctx* ctx, uint64_t key, F body,
+                                 const uint16_t* src = nullptr) {
+    if (ctx->timing || !ctx->use_graph || ctx->comm) return body();
+    auto it = ctx->graphs.find(key);
+    if (it == ctx->graphs.end()) {
+        cudaStream_t user = ctx->stream;
+        const int64_t l0 = ctx->launches;
+        ctx->stream = ctx->cap_stream;
+        cudaError_t e = cudaStreamBeginCapture(ctx->cap_stream, cudaStreamCaptureModeThreadLocal);
+        if (e != cudaSuccess) {
+            ctx->stream = user;
+            return cuda_fail(ctx, e, "begin capture");
+        }
+        stitch_status st = body();
+        cudaGraph_t g = nullptr;
+        e = cudaStreamEndCapture(ctx->cap_stream, &g);
+        ctx->stream = user;
+        if (st != STITCH_OK) {
+            if (g) cudaGraphDestroy(g);
+            return st;
+        }
+        if (e != cudaSuccess) return cuda_fail(ctx, e, "end capture");
+        stitch_ctx::GraphRec rec;
+        rec.graph = g;
+        rec.launches = ctx->launches - l0;
+        rec.src = reinterpret_cast<const char*>(src);
+        if (src) {   // remember the H2D nodes (the only memcpy nodes of a step)
+            size_t nn = 0;
+            CK(cudaGraphGetNodes(g, nullptr, &nn), "graph nodes");
+            std::vector<cudaGraphNode_t> nodes(nn);
+            CK(cudaGraphGetNodes(g, nodes.data(), &nn), "graph nodes");
+            for (cudaGraphNode_t nd : nodes) {
+                cudaGraphNodeType ty;
+                CK(cudaGraphNodeGetType(nd, &ty), "node type");
+                if (ty != cudaGraphNodeTypeMemcpy) continue;
+                cudaMemcpy3DParms p;
+                CK(cudaGraphMemcpyNodeGetParams(nd, &p), "memcpy params");
+                rec.h2d.push_back(nd);
+                rec.h2d_p.push_back(p);
+            }
+        }
+        e = cudaGraphInstantiate(&rec.exec, g, 0);
+        if (e != cudaSuccess) {
+            cudaGraphDestroy(g);
+            return cuda_fail(ctx, e, "graph instantiate");
+        }
+        it = ctx->graphs.emplace(key, rec).first;
+        ctx->launches = l0;
+    }
+    stitch_ctx::GraphRec& rec = it->second;
+    if (src && reinterpret_cast<const char*>(src) != rec.src) {
+        const char* ns = reinterpret_cast<const char*>(src);
+        for (size_t i = 0; i < rec.h2d.size(); ++i) {
+            cudaMemcpy3DParms p = rec.h2d_p[i];
+            p.srcPtr.ptr = const_cast<char*>(ns + (static_cast<const char*>(p.srcPtr.ptr) - rec.src));
+            CK(cudaGraphExecMemcpyNodeSetParams(rec.exec, rec.h2d[i], &p), "re-point H2D node");
+            rec.h2d_p[i] = p;
+        }
+        rec.src = ns;
+    }
+    CK(cudaGraphLaunch(rec.exec, ctx->stream), "graph launch");
+    ctx->launches += rec.launches;
+    return STITCH_OK;
+}
+}  // extern "C++"
+
+static cudaError_t collect_timings(stitch_ctx* ctx) {
+    cudaError_t e = cudaSuccess;
+    if (ctx->timing == 3) {
+        ctx->tl_ms.assign(2 * ctx->tl.size(), 0.f);
+        for (size_t i = 0; i < ctx->tl.size(); ++i) {
+            if ((e = cudaEventElapsedTime(&ctx->tl_ms[2 * i], ctx->tl_origin, ctx->tl[i].a)) !=
+                    cudaSuccess ||
+                (e = cudaEventElapsedTime(&ctx->tl_ms[2 * i + 1], ctx->tl_origin, ctx->tl[i].b)) !=
+                    cudaSuccess)
+                return e;
+        }
+        return cudaSuccess;
+    }
+    if (ctx->timing) {   // stage events a split step did not record read as 0
+        for (int i = 0; i < 4; ++i) {
+            if (cudaEventElapsedTime(&ctx->ms[i], ctx->ev[i < 3 ? i : 0], ctx->ev[i < 3 ? i + 1 : 3]) !=
+                cudaSuccess) {
+                ctx->ms[i] = 0.f;
+                cudaGetLastError();
+            }
+        }
+    }
+    if (ctx->timing >= 2) {
+        for (int k = 0; k < 6; ++k) { ctx->kms[k] = 0.f; ctx->kcount[k] = 0; }
+        for (size_t i = 0; i < ctx->kkind.size(); ++i) {
+            float t = 0.f;
+            if ((e = cudaEventElapsedTime(&t, ctx->kev[i], ctx->kev[i + 1])) != cudaSuccess) return e;
+            const int k = ctx->kkind[i];
+            if (k >= 0) { ctx->kms[k] += t; ctx->kcount[k] += 1; }
+        }
+    }
+    return cudaSuccess;
+}
 
 extern "C" {
 
@@ -633,12 +1090,24 @@ const char* stitch_status_string(stitch_status s) {
     switch (s) {
         case STITCH_OK: return "ok";
         case STITCH_ERR_INVALID_ARG: return "invalid argument";
-        case STITCH_ERR_UNSUPPORTED: return "unsupported tile size";
+        case STITCH_ERR_UNSUPPORTED: return "unsupported tile size or mode";
         case STITCH_ERR_OUT_OF_MEMORY: return "out of device memory";
         case STITCH_ERR_CUDA: return "CUDA error";
+        case STITCH_ERR_NCCL: return "NCCL error";
         case STITCH_ERR_STATE: return "invalid call order";
     }
     return "unknown status";
+}
+
+stitch_status stitch_nccl_unique_id(void* out128) {
+    if (!out128) return STITCH_ERR_INVALID_ARG;
+    const NcclApi& api = nccl();
+    if (!api.ok) return STITCH_ERR_NCCL;
+    ncclUniqueId id;
+    if (api.get_unique_id(&id) != ncclSuccess) return STITCH_ERR_NCCL;
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId is 128 bytes");
+    std::memcpy(out128, &id, sizeof(id));
+    return STITCH_OK;
 }
 
 stitch_status stitch_workspace_size(const stitch_config* cfg, size_t* bytes) {
@@ -648,6 +1117,14 @@ stitch_status stitch_workspace_size(const stitch_config* cfg, size_t* bytes) {
     if (s != STITCH_OK) return s;
     Layout L;
     if ((s = make_layout(cfg, ops, &L)) != STITCH_OK) return s;
+    if (L.pool) {   // the bounded mode's schedule must exist for this pool (host simulation)
+        stitch_ctx tmp;
+        tmp.L = L;
+        tmp.n = cfg->grid_rows;
+        tmp.m = cfg->grid_cols;
+        std::string why;
+        if (!build_pooled(&tmp, &why)) return STITCH_ERR_INVALID_ARG;
+    }
     *bytes = L.total;
     return STITCH_OK;
 }
@@ -665,28 +1142,26 @@ stitch_status stitch_pair_count(const stitch_config* cfg, int64_t* count) {
 
 void stitch_destroy(stitch_ctx* ctx) {
     if (!ctx) return;
+    DevGuard guard(ctx->cfg.device);
     if (ctx->stream) cudaStreamSynchronize(ctx->stream);
+    if (ctx->comm) nccl().comm_destroy(ctx->comm);
     for (auto& e : ctx->ev)
         if (e) cudaEventDestroy(e);
     for (auto& e : ctx->kev)
         if (e) cudaEventDestroy(e);
-    for (auto& g : ctx->graphs) cudaGraphExecDestroy(g.second.exec);
+    for (auto& g : ctx->graphs) {
+        if (g.second.exec) cudaGraphExecDestroy(g.second.exec);
+        if (g.second.graph) cudaGraphDestroy(g.second.graph);
+    }
     if (ctx->cap_stream) cudaStreamDestroy(ctx->cap_stream);
-    for (auto& e : ctx->ev_fwd)
+    for (auto* v : {&ctx->ev_fwd, &ctx->ev_k4, &ctx->ev_k5, &ctx->ev_h2d, &ctx->tl_pool})
+        for (auto& e : *v)
+            if (e) cudaEventDestroy(e);
+    for (cudaEvent_t e : {ctx->ev_fork, ctx->ev_halo})
         if (e) cudaEventDestroy(e);
-    for (auto& e : ctx->ev_k4)
-        if (e) cudaEventDestroy(e);
-    for (auto& e : ctx->ev_h2d)
-        if (e) cudaEventDestroy(e);
-    for (auto& e : ctx->ev_k3)
-        if (e) cudaEventDestroy(e);
-    for (auto& e : ctx->tl_pool)
-        if (e) cudaEventDestroy(e);
-    if (ctx->s_pair4) cudaStreamDestroy(ctx->s_pair4);
-    if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
     for (auto& e : ctx->ev_join)
         if (e) cudaEventDestroy(e);
-    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d})
+    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d, ctx->s_comm})
         if (st) cudaStreamDestroy(st);
     if (ctx->own_mem && ctx->mem) cudaFree(ctx->mem);
     if (ctx->own_stream && ctx->stream) cudaStreamDestroy(ctx->stream);
@@ -714,99 +1189,59 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     ctx->m = cfg->grid_cols;
     ctx->H = ops->H;
     ctx->W = ops->W;
+    ctx->prec = L.prec;
+    // the static schedule (host only: an infeasible pool fails before any device work)
+    if (L.pool) {
+        std::string why;
+        if (!build_pooled(ctx, &why)) {
+            delete ctx;
+            return STITCH_ERR_INVALID_ARG;
+        }
+    } else {
+        build_resident(ctx);
+    }
+    ctx->res_h.resize((size_t)L.npairs);
+    DevGuard guard(cfg->device);
+    if (guard.err != cudaSuccess) {
+        delete ctx;
+        return STITCH_ERR_CUDA;
+    }
     auto bail = [&](stitch_status st) {
         stitch_destroy(ctx);
         return st;
     };
-    cudaError_t e = cudaSetDevice(cfg->device);
-    if (e != cudaSuccess) return bail(STITCH_ERR_CUDA);
-    if ((e = ops->setup(&ctx->grid_k1p, &ctx->grid_k4p, &ctx->grid_k1w, &ctx->grid_k4w)) !=
-        cudaSuccess)
-        return bail(STITCH_ERR_CUDA);
-    ctx->prec = L.prec;
+    cudaError_t e;
+    if ((e = ops->setup(&ctx->grid_k1, &ctx->grid_k4)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
     if (ctx->prec && (e = ops->d_setup()) != cudaSuccess) return bail(STITCH_ERR_CUDA);
-    {
-        const char* wenv = std::getenv("STITCH_ROWWARP");   // STITCH_ROWWARP=0: CTA row kernels
-        if (wenv && wenv[0] == '0') ctx->grid_k1w = ctx->grid_k4w = 0;
-    }
-    {
-        // column-kernel variant: one CTA per panel (default: several CTAs per SM overlap each
-        // other's TMA waits) or persistent with TMA prefetch (STITCH_COL_PERSIST=1; one CTA
-        // per SM, measured slower on B200: fewer resident warps)
-        const char* env = std::getenv("STITCH_COL_PERSIST");
-        int sms = 0;
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
-        ctx->grid_colp = (env && env[0] == '1') ? sms : 0;
-        // K2 / K3: L2 prefetch of the panels of the CTA one wave ahead (STITCH_L2PF /
-        // STITCH_L2PF3 = <CTAs>, 0 = off).  Measured: K2 7.25 -> 6.85 ms at one wave (2 CTAs
-        // x SMs); K3 slower (11.18 -> 11.53 ms: its prefetch needs the next pair's tile
-        // indices, a dependent global load in the prologue), so off for K3 by default.
-        {
-            const char* pf = std::getenv("STITCH_L2PF");
-            ctx->col_ahead = pf ? std::atoi(pf) : 2 * sms;
-            const char* pf3 = std::getenv("STITCH_L2PF3");
-            ctx->col_ahead3 = pf3 ? std::atoi(pf3) : 0;
-        }
-        // two-group persistent column kernels (STITCH_COLG=1)
-        {
-            const char* genv2 = std::getenv("STITCH_COLG");
-            if (!ctx->prec && genv2 && genv2[0] == '1')
-                if ((e = ops->setup_g(&ctx->grid_colg)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
-        }
-        // quad persistent column kernels (STITCH_COLQ=1; measured slower on B200, ncu r01q:
-        // the panel prefetch removes the TMA wait (30 % -> 3 % of K3's stall samples) but the
-        // 104-of-160-thread stage 1 leaves 22 % at barriers and the L1 twiddle loads another
-        // ~20 %: K3 11.2 -> 15.6 ms per step)
-        const char* qenv = std::getenv("STITCH_COLQ");
-        if (!ctx->prec && ops->col_p_q > 0 && qenv && qenv[0] == '1') {
-            if ((e = ops->setup_q(&ctx->grid_colq)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
-        }
-        const char* genv = std::getenv("STITCH_GRAPH");   // STITCH_GRAPH=0: direct launches
-        ctx->use_graph = !(genv && genv[0] == '0');
-        const char* cenv = std::getenv("STITCH_CONCURRENT");  // STITCH_CONCURRENT=0: one stream
-        ctx->concurrent = !(cenv && cenv[0] == '0') && !ctx->prec;
-        if (ctx->concurrent) {
-            for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf, &ctx->s_h2d})
-                if (cudaStreamCreateWithFlags(st, cudaStreamNonBlocking) != cudaSuccess)
-                    return bail(STITCH_ERR_CUDA);
-            const int nf = (L.nlocal + L.chunk_tiles - 1) / L.chunk_tiles;
-            const int nc = (int)((L.npairs + L.chunk_pairs - 1) / L.chunk_pairs);
-            ctx->ev_fwd.assign(nf, nullptr);
-            ctx->ev_h2d.assign(nf, nullptr);
-            ctx->ev_k4.assign(nc, nullptr);
-            for (auto& e : ctx->ev_h2d)
-                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                    return bail(STITCH_ERR_CUDA);
-            if (L.q_slots == 2 && ctx->grid_k4w > 0) {
-                if (cudaStreamCreateWithFlags(&ctx->s_pair4, cudaStreamNonBlocking) != cudaSuccess)
-                    return bail(STITCH_ERR_CUDA);
-                ctx->ev_k3.assign(nc, nullptr);
-                for (auto& e : ctx->ev_k3)
-                    if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                        return bail(STITCH_ERR_CUDA);
-                const char* ke = std::getenv("STITCH_DUAL_K4");
-                const int per_sm = ke ? std::max(1, std::atoi(ke)) : 1;
-                int sms = 0;
-                cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
-                ctx->grid_k4w_dual = std::min(ctx->grid_k4w, per_sm * sms);
-            }
-            for (auto& e : ctx->ev_fwd)
-                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                    return bail(STITCH_ERR_CUDA);
-            for (auto& e : ctx->ev_k4)
-                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                    return bail(STITCH_ERR_CUDA);
-            if (cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming) != cudaSuccess)
-                return bail(STITCH_ERR_CUDA);
-            for (auto& e : ctx->ev_join)
-                if (cudaEventCreateWithFlags(&e, cudaEventDisableTiming) != cudaSuccess)
-                    return bail(STITCH_ERR_CUDA);
-        }
-        if (ctx->use_graph &&
-            cudaStreamCreateWithFlags(&ctx->cap_stream, cudaStreamNonBlocking) != cudaSuccess)
-            return bail(STITCH_ERR_CUDA);
-    }
+    int sms = 0;
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
+    ctx->col_ahead = 2 * sms;   // K2's L2 prefetch one wave (2 CTAs per SM) ahead
+    ctx->use_graph = !(cfg->flags & STITCH_FLAG_NO_GRAPH);
+    ctx->concurrent = !(cfg->flags & STITCH_FLAG_SERIAL) && !ctx->prec;
 
+    if (ctx->concurrent) {
+        for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf, &ctx->s_h2d})
+            if (cudaStreamCreateWithFlags(st, cudaStreamNonBlocking) != cudaSuccess)
+                return bail(STITCH_ERR_CUDA);
+        auto mk = [&](std::vector<cudaEvent_t>& v, size_t k) {
+            v.assign(k, nullptr);
+            for (auto& ev : v)
+                if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess) return false;
+            return true;
+        };
+        if (!mk(ctx->ev_fwd, ctx->fwd.size()) || !mk(ctx->ev_h2d, ctx->fwd.size()) ||
+            !mk(ctx->ev_k4, ctx->pch.size()) || !mk(ctx->ev_k5, ctx->pch.size()))
+            return bail(STITCH_ERR_CUDA);
+        for (cudaEvent_t* ev : {&ctx->ev_fork, &ctx->ev_halo})
+            if (cudaEventCreateWithFlags(ev, cudaEventDisableTiming) != cudaSuccess)
+                return bail(STITCH_ERR_CUDA);
+        for (auto& ev : ctx->ev_join)
+            if (cudaEventCreateWithFlags(&ev, cudaEventDisableTiming) != cudaSuccess)
+                return bail(STITCH_ERR_CUDA);
+    }
+    if (ctx->use_graph &&
+        cudaStreamCreateWithFlags(&ctx->cap_stream, cudaStreamNonBlocking) != cudaSuccess)
+        return bail(STITCH_ERR_CUDA);
     if (cfg->stream) {
         ctx->stream = (cudaStream_t)cfg->stream;
     } else {
@@ -827,7 +1262,6 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     ctx->spec = (uint32_t*)(b + L.off_spec);
     ctx->G = (float2*)(b + L.off_g);
     ctx->Q = (float2*)(b + L.off_q);
-    if (L.q_slots == 2) ctx->Q2 = ctx->Q + (size_t)L.chunk_pairs * ops->H * ops->WP;
     ctx->pairs = (PairIdx*)(b + L.off_pairs);
     ctx->keys = (unsigned long long*)(b + L.off_keys);
     ctx->mom = (unsigned long long*)(b + L.off_mom);
@@ -835,6 +1269,7 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     ctx->twM = (float2*)(b + L.off_tw);
     ctx->twH = ctx->twM + tw_row(ops);
     ctx->twW = ctx->twH + tw_col(ops);
+    ctx->fslot = (int32_t*)(b + L.off_fslot);
     if (ctx->prec) {
         ctx->Ud = (double2*)(b + L.off_spec);
         ctx->Gd = (double2*)(b + L.off_g);
@@ -858,130 +1293,105 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
         const cuuint32_t boxh = (cuuint32_t)(ops->H / ((ops->H + 255) / 256));
         const cuuint32_t estr[2] = {1, 1};
-        // G: complex chunk [chunk_tiles*H][WP] as floats; spec: u32 Q15 phasors [nlocal*H][WP]
-        auto encode_pair = [&](CUtensorMap* mg, CUtensorMap* ms, int colp) {
-            const cuuint64_t gd[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
-            const cuuint64_t gs[1] = {(cuuint64_t)ops->WP * 8};
-            const cuuint32_t gb[2] = {(cuuint32_t)2 * colp, boxh};
-            const cuuint64_t sd[2] = {(cuuint64_t)ops->WP, (cuuint64_t)L.nlocal * ops->H};
-            const cuuint64_t ss[1] = {(cuuint64_t)ops->WP * 4};
-            const cuuint32_t sb[2] = {(cuuint32_t)colp, boxh};
-            return encode(mg, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, gd, gs, gb, estr,
-                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS &&
-                   encode(ms, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->spec, sd, ss, sb, estr,
-                          CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-                          CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
-        };
-        if (!encode_pair(&ctx->tmG, &ctx->tmS, ops->col_p)) return bail(STITCH_ERR_CUDA);
-        if (ctx->grid_colq > 0 && !encode_pair(&ctx->tmG4, &ctx->tmS4, ops->col_p_q))
+        // G: complex chunk [chunk_tiles*H][WP] as floats; spec: u32 Q15 phasors [nslots*H][WP]
+        const cuuint64_t gd[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
+        const cuuint64_t gs[1] = {(cuuint64_t)ops->WP * 8};
+        const cuuint32_t gb[2] = {(cuuint32_t)2 * ops->col_p, boxh};
+        const cuuint64_t sd[2] = {(cuuint64_t)ops->WP, (cuuint64_t)L.nslots * ops->H};
+        const cuuint64_t ss[1] = {(cuuint64_t)ops->WP * 4};
+        const cuuint32_t sb[2] = {(cuuint32_t)ops->col_p, boxh};
+        if (encode(&ctx->tmG, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, gd, gs, gb, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) !=
+                CUDA_SUCCESS ||
+            encode(&ctx->tmS, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->spec, sd, ss, sb, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) !=
+                CUDA_SUCCESS)
             return bail(STITCH_ERR_CUDA);
     }
 
     // Twiddles w_N^e = exp(-2 pi i e / N), computed in double, rounded once.
     //   stage-2 tables: tw2[b*(r1-1) + j-1] = w_N^{j b}, b < r0, 1 <= j < r1 (fft_engine.cuh)
+    auto fill_tw = [&](auto* dst, auto make) {
+        auto w = [&](long ex, long N) {
+            const double a = -2.0 * M_PI * (double)(ex % N) / (double)N;
+            return make(std::cos(a), std::sin(a));
+        };
+        auto fill2 = [&](auto* d, int r0, int r1) {
+            const int N = r0 * r1;
+            for (int bb = 0; bb < r0; ++bb)
+                for (int j = 1; j < r1; ++j) d[(size_t)bb * (r1 - 1) + j - 1] = w((long)j * bb, N);
+        };
+        fill2(dst, ops->row_r0, ops->row_r1);
+        fill2(dst + tw_row(ops), ops->col_r0, ops->col_r1);
+        for (int k = 0; k < ops->W; ++k) dst[tw_row(ops) + tw_col(ops) + k] = w(k, ops->W);
+    };
     std::vector<float2> tw(tw_count(ops));
-    auto w = [](long e, long N) {
-        const double a = -2.0 * M_PI * (double)(e % N) / (double)N;
-        return make_float2((float)std::cos(a), (float)std::sin(a));
-    };
-    auto fill2 = [&](float2* dst, int r0, int r1) {
-        const int N = r0 * r1;
-        for (int bb = 0; bb < r0; ++bb)
-            for (int j = 1; j < r1; ++j) dst[(size_t)bb * (r1 - 1) + j - 1] = w((long)j * bb, N);
-    };
-    fill2(tw.data(), ops->row_r0, ops->row_r1);
-    fill2(tw.data() + tw_row(ops), ops->col_r0, ops->col_r1);
-    for (int k = 0; k < ops->W; ++k) tw[tw_row(ops) + tw_col(ops) + k] = w(k, ops->W);
-
-    // Pair list: every owned tile's west and north pair, as (neighbour, tile) (Fig. 4).
-    // Processing order (results do not depend on it): tiles in bands of PAIR_BAND tile
-    // rows, column-major inside a band, so a tile's spectrum and raw pixels are reused by
-    // its <= 4 pairs while still in L2 (the paper's traversal-order idea).
-    // 4 rows: a tile's west-pair reuse 8 pairs (~90 MB of panels and Q) after its first use
-    // stays in the 126 MB L2 (bands of 1-8 measured: 3-4 best, K3 10.81 -> 10.63 ms), and the
-    // first pair chunk waits for 4 tile rows of forward transforms instead of 8.
-    // STITCH_PAIR_BAND overrides (experiments).
-    int PAIR_BAND = 4;
-    if (const char* benv = std::getenv("STITCH_PAIR_BAND")) PAIR_BAND = std::max(1, std::atoi(benv));
-    std::vector<int> order;
-    order.reserve((size_t)(L.t_end - L.t_begin));
-    for (int t = L.t_begin; t < L.t_end; ++t) order.push_back(t);
-    const int mm = ctx->m;
-    std::stable_sort(order.begin(), order.end(), [mm, PAIR_BAND](int a, int b) {
-        const int ra = a / mm, rb = b / mm, ba = ra / PAIR_BAND, bb = rb / PAIR_BAND;
-        if (ba != bb) return ba < bb;
-        if (a % mm != b % mm) return a % mm < b % mm;
-        return ra < rb;
-    });
-    std::vector<PairIdx> pl;
-    pl.reserve((size_t)L.npairs);
-    for (const int t : order) {
-        const int r = t / ctx->m, c = t % ctx->m;
-        if (c >= 1) {
-            pl.push_back(PairIdx{t - 1 - L.h_begin, t - L.h_begin});
-            ctx->pair_tile.push_back(t);
-            ctx->pair_kind.push_back(0);
-        }
-        if (r >= 1) {
-            pl.push_back(PairIdx{t - ctx->m - L.h_begin, t - L.h_begin});
-            ctx->pair_tile.push_back(t);
-            ctx->pair_kind.push_back(1);
-        }
-    }
-    ctx->res_h.resize((size_t)L.npairs);
-    // forward chunk that completes every tile a pair chunk reads (concurrent schedule)
-    for (int64_t p0 = 0; p0 < L.npairs; p0 += L.chunk_pairs) {
-        int mx = 0;
-        for (int64_t p = p0; p < L.npairs && p < p0 + L.chunk_pairs; ++p)
-            mx = std::max(mx, std::max(pl[(size_t)p].a, pl[(size_t)p].b));
-        ctx->pair_need.push_back(mx / L.chunk_tiles);
-    }
-    // fp64 twiddles: the same tables, rounded once to double
     std::vector<double2> twd;
     if (ctx->prec) {
         twd.resize(tw_count(ops));
-        auto wd = [](long e2, long N) {
-            const double a = -2.0 * M_PI * (double)(e2 % N) / (double)N;
-            return make_double2(std::cos(a), std::sin(a));
-        };
-        auto fill2d = [&](double2* dst, int r0, int r1) {
-            const int N = r0 * r1;
-            for (int bb = 0; bb < r0; ++bb)
-                for (int j = 1; j < r1; ++j) dst[(size_t)bb * (r1 - 1) + j - 1] = wd((long)j * bb, N);
-        };
-        fill2d(twd.data(), ops->row_r0, ops->row_r1);
-        fill2d(twd.data() + tw_row(ops), ops->col_r0, ops->col_r1);
-        for (int k = 0; k < ops->W; ++k) twd[tw_row(ops) + tw_col(ops) + k] = wd(k, ops->W);
-        if ((e = cudaMemcpyAsync(ctx->twMd, twd.data(), twd.size() * sizeof(double2),
-                                 cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
-            return bail(STITCH_ERR_CUDA);
-    } else if ((e = cudaMemcpyAsync(ctx->twM, tw.data(), tw.size() * sizeof(float2),
-                                    cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
+        fill_tw(twd.data(), [](double c, double sn) { return make_double2(c, sn); });
+        e = cudaMemcpyAsync(ctx->twMd, twd.data(), twd.size() * sizeof(double2),
+                            cudaMemcpyHostToDevice, ctx->stream);
+    } else {
+        fill_tw(tw.data(), [](double c, double sn) { return make_float2((float)c, (float)sn); });
+        e = cudaMemcpyAsync(ctx->twM, tw.data(), tw.size() * sizeof(float2),
+                            cudaMemcpyHostToDevice, ctx->stream);
+    }
+    if (e != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if (!ctx->pairs_h.empty() &&
+        cudaMemcpyAsync(ctx->pairs, ctx->pairs_h.data(), ctx->pairs_h.size() * sizeof(PairIdx),
+                        cudaMemcpyHostToDevice, ctx->stream) != cudaSuccess)
         return bail(STITCH_ERR_CUDA);
-    if (!pl.empty() &&
-        (e = cudaMemcpyAsync(ctx->pairs, pl.data(), pl.size() * sizeof(PairIdx),
-                             cudaMemcpyHostToDevice, ctx->stream)) != cudaSuccess)
+    if (cudaMemcpyAsync(ctx->fslot, ctx->fslot_h.data(), ctx->fslot_h.size() * sizeof(int32_t),
+                        cudaMemcpyHostToDevice, ctx->stream) != cudaSuccess)
         return bail(STITCH_ERR_CUDA);
     for (auto& ev : ctx->ev)
         if (cudaEventCreate(&ev) != cudaSuccess) return bail(STITCH_ERR_CUDA);
-    if ((e = cudaStreamSynchronize(ctx->stream)) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+    if (cudaStreamSynchronize(ctx->stream) != cudaSuccess) return bail(STITCH_ERR_CUDA);
+
+    // NCCL communicator (collective over the world: every rank calls stitch_init)
+    if (L.exchange) {
+        const NcclApi& api = nccl();
+        if (!api.ok) return bail(STITCH_ERR_NCCL);
+        ncclUniqueId id;
+        std::memcpy(&id, cfg->nccl_id, sizeof(id));
+        if (api.comm_init_rank(&ctx->comm, L.world, id, L.rank) != ncclSuccess) {
+            ctx->comm = nullptr;
+            return bail(STITCH_ERR_NCCL);
+        }
+        if (cudaStreamCreateWithFlags(&ctx->s_comm, cudaStreamNonBlocking) != cudaSuccess)
+            return bail(STITCH_ERR_CUDA);
+        const int64_t nt = (int64_t)ctx->n * ctx->m;
+        if (L.rank + 1 < L.world) {   // rank+1's halo: the last m tiles of this band
+            int nb, ne;
+            band_of(nt, L.rank + 1, L.world, &nb, &ne);
+            const int nh = nb - ctx->m > 0 ? nb - ctx->m : 0;
+            ctx->send_lt = nh - L.h_begin;
+            ctx->send_cnt = nb - nh;
+        }
+        ctx->recv_lt = 0;
+        ctx->recv_cnt = L.t_begin - L.h_begin;
+    }
     *out = ctx;
     return STITCH_OK;
 }
 
-static stitch_status load_common(stitch_ctx* ctx, const uint16_t* src, size_t n_bytes,
-                                 cudaMemcpyKind kind) {
-    if (!ctx) return STITCH_ERR_INVALID_ARG;
-    if (!src) return fail(ctx, STITCH_ERR_INVALID_ARG, "null grid pointer");
+static stitch_status load_common(stitch_ctx* ctx, const uint16_t* src, int first_tile,
+                                 int64_t count, bool on_device) {
+    if (ctx->L.pool)
+        return fail(ctx, STITCH_ERR_STATE,
+                    "bounded-mode context: tiles arrive with stitch_compute_translations_from_host_async");
+    if (first_tile > ctx->L.h_begin || first_tile + count < ctx->L.t_end || first_tile < 0)
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range does not cover [halo_begin, tile_end)");
     const size_t tile = (size_t)ctx->H * ctx->W;
-    if (n_bytes != (size_t)ctx->n * ctx->m * tile * sizeof(uint16_t))
-        return fail(ctx, STITCH_ERR_INVALID_ARG, "n_bytes != n*m*H*W*2");
-    CK(cudaMemcpyAsync(ctx->raw, src + (size_t)ctx->L.h_begin * tile,
-                       (size_t)ctx->L.nlocal * tile * sizeof(uint16_t), kind, ctx->stream),
-       "load grid");
+    CK(cudaMemcpyAsync(ctx->raw, src + (size_t)(ctx->L.h_begin - first_tile) * tile,
+                       (size_t)ctx->L.nlocal * tile * sizeof(uint16_t),
+                       on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->stream),
+       "load tiles");
+    // host memory: return only once the copy is done, so the caller may reuse the buffer
+    if (!on_device) CK(cudaStreamSynchronize(ctx->stream), "load synchronize");
     ctx->loaded = true;
     ctx->computed = false;
     return STITCH_OK;
@@ -991,16 +1401,8 @@ stitch_status stitch_load_tiles(stitch_ctx* ctx, const uint16_t* tiles, int32_t 
                                 int32_t count, int32_t on_device) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (!tiles) return fail(ctx, STITCH_ERR_INVALID_ARG, "null tiles pointer");
-    if (first_tile > ctx->L.h_begin || first_tile + (int64_t)count < ctx->L.t_end || first_tile < 0)
-        return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range does not cover [halo_begin, tile_end)");
-    const size_t tile = (size_t)ctx->H * ctx->W;
-    CK(cudaMemcpyAsync(ctx->raw, tiles + (size_t)(ctx->L.h_begin - first_tile) * tile,
-                       (size_t)ctx->L.nlocal * tile * sizeof(uint16_t),
-                       on_device ? cudaMemcpyDeviceToDevice : cudaMemcpyHostToDevice, ctx->stream),
-       "load tiles");
-    ctx->loaded = true;
-    ctx->computed = false;
-    return STITCH_OK;
+    GUARD(ctx);
+    return load_common(ctx, tiles, first_tile, count, on_device != 0);
 }
 
 stitch_status stitch_resident_range(stitch_ctx* ctx, int32_t* halo_begin, int32_t* tile_begin,
@@ -1012,343 +1414,100 @@ stitch_status stitch_resident_range(stitch_ctx* ctx, int32_t* halo_begin, int32_
     return STITCH_OK;
 }
 
+static stitch_status load_grid(stitch_ctx* ctx, const uint16_t* src, size_t n_bytes, bool dev) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!src) return fail(ctx, STITCH_ERR_INVALID_ARG, "null grid pointer");
+    if (n_bytes != (size_t)ctx->n * ctx->m * ctx->H * ctx->W * sizeof(uint16_t))
+        return fail(ctx, STITCH_ERR_INVALID_ARG, "n_bytes != n*m*H*W*2");
+    GUARD(ctx);
+    return load_common(ctx, src, 0, (int64_t)ctx->n * ctx->m, dev);
+}
+
 stitch_status stitch_load_grid(stitch_ctx* ctx, const uint16_t* host_grid, size_t n_bytes) {
-    return load_common(ctx, host_grid, n_bytes, cudaMemcpyHostToDevice);
+    return load_grid(ctx, host_grid, n_bytes, false);
 }
 
 stitch_status stitch_load_grid_device(stitch_ctx* ctx, const uint16_t* dev_grid, size_t n_bytes) {
-    return load_common(ctx, dev_grid, n_bytes, cudaMemcpyDeviceToDevice);
+    return load_grid(ctx, dev_grid, n_bytes, true);
 }
-
-// K6's divisor of the argmax value: max|c| / (W H) (C5); the fp32 path's NCPS carries the
-// Q15 phasor scale 32767^2 (pciam_kernels.cuh, phasor_q15).
-static double k6_peak_div(const stitch_ctx* ctx) {
-    const double wh = (double)ctx->W * (double)ctx->H;
-    return ctx->prec ? wh : wh * NCPS_Q15_SCALE;
-}
-
-// Row kernels: warp-per-line (K1w/K4w) where the plan allows, else
-// persistent CTA rows (K1p/K4p), else one CTA per row block (K1/K4).
-static void launch_k1_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
-    const PlanOps* o = ctx->ops;
-    if (ctx->grid_k1w > 0)
-        o->k1w(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1w, s);
-    else if (ctx->grid_k1p > 0)
-        o->k1p(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, ctx->grid_k1p, s);
-    else
-        o->k1(ctx->raw, ctx->G, t0, nt, ctx->twM, ctx->twW, s);
-}
-static void launch_k4_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
-                          const float2* Qp = nullptr, int grid_w = 0) {
-    const PlanOps* o = ctx->ops;
-    const float2* q = Qp ? Qp : ctx->Q;
-    if (ctx->grid_k4w > 0)
-        o->k4w(q, ctx->keys, p0, np, ctx->twM, ctx->twW, grid_w > 0 ? grid_w : ctx->grid_k4w, s);
-    else if (ctx->grid_k4p > 0)
-        o->k4p(q, ctx->keys, p0, np, ctx->twM, ctx->twW, ctx->grid_k4p, s);
-    else
-        o->k4(q, ctx->keys, p0, np, ctx->twM, ctx->twW, s);
-}
-
-// Column kernels: quad persistent (3 CTAs/SM, TMA prefetch) where available, else the
-// persistent single-CTA variant if requested, else one CTA per panel.
-static void launch_k2_any(stitch_ctx* ctx, int t0, int nt, cudaStream_t s) {
-    const PlanOps* o = ctx->ops;
-    if (ctx->grid_colg > 0)
-        o->k2g(ctx->tmG, ctx->spec, t0, nt, ctx->twH, ctx->grid_colg, s);
-    else if (ctx->grid_colq > 0)
-        o->k2q(ctx->tmG4, ctx->G, ctx->spec, t0, nt, ctx->twH, ctx->grid_colq, s);
-    else if (ctx->grid_colp > 0)
-        o->k2p(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->grid_colp, s);
-    else
-        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->twH, true, ctx->col_ahead, s);
-}
-static void launch_k3_any(stitch_ctx* ctx, int p0, int np, cudaStream_t s,
-                          float2* Qp = nullptr) {
-    const PlanOps* o = ctx->ops;
-    float2* q = Qp ? Qp : ctx->Q;
-    if (ctx->grid_colg > 0)
-        o->k3g(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colg, s);
-    else if (ctx->grid_colq > 0)
-        o->k3q(ctx->tmS4, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colq, s);
-    else if (ctx->grid_colp > 0)
-        o->k3p(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->grid_colp, s);
-    else
-        o->k3(ctx->tmS, q, ctx->pairs, p0, np, ctx->twH, ctx->col_ahead3, s);
-}
-
-// Forward transforms (K1 + K2) of the resident tiles with local indices [lt0, lt0 + count).
-static stitch_status forward_impl(stitch_ctx* ctx, int lt0, int count) {
-    const PlanOps* o = ctx->ops;
-    const int ct = ctx->L.chunk_tiles;
-    for (int t0 = lt0; t0 < lt0 + count; t0 += ct) {
-        const int nt = lt0 + count - t0 < ct ? lt0 + count - t0 : ct;
-        if (ctx->prec) {   // fp64 path (f2): D1, D2
-            o->d1(ctx->raw, ctx->Gd, t0, nt, ctx->twMd, ctx->twWd, ctx->stream);
-            CK(mark(ctx, 0), "event");
-            o->d2(ctx->Gd, ctx->Ud, t0, nt, ctx->twHd, true, ctx->stream);
-            CK(mark(ctx, 1), "event");
-            ctx->launches += 2;
-            continue;
-        }
-        launch_k1_any(ctx, t0, nt, ctx->stream);
-        CK(mark(ctx, 0), "event");
-        launch_k2_any(ctx, t0, nt, ctx->stream);
-        CK(mark(ctx, 1), "event");
-        ctx->launches += 2;
-    }
-    CK(cudaGetLastError(), "forward launch");
-    return STITCH_OK;
-}
-
-// Steps 3-7 (K3..K6) for every pair of the range; spectra must be resident.
-static stitch_status pairs_impl(stitch_ctx* ctx) {
-    const PlanOps* o = ctx->ops;
-    cudaStream_t s = ctx->stream;
-    const int64_t np = ctx->L.npairs;
-    if (np > 0) {
-        CK(cudaMemsetAsync(ctx->keys, 0, (size_t)np * sizeof(unsigned long long), s), "memset");
-        CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), s), "memset");
-        if (ctx->timing >= 2) CK(mark(ctx, -1), "event");
-        const int cp = ctx->L.chunk_pairs;
-        for (int64_t p0 = 0; p0 < np; p0 += cp) {
-            const int npc = (int)(np - p0 < cp ? np - p0 : cp);
-            if (ctx->prec) {   // fp64 path (f2): D3, D4 (block argmax partials)
-                o->d3(ctx->Ud, ctx->Qd, ctx->pairs, (int)p0, npc, ctx->twHd, s);
-                CK(mark(ctx, 2), "event");
-                o->d4(ctx->Qd, ctx->part_v, ctx->part_i, (int)p0, npc, ctx->twMd, ctx->twWd, s);
-                CK(mark(ctx, 3), "event");
-                ctx->launches += 2;
-                continue;
-            }
-            launch_k3_any(ctx, (int)p0, npc, s);
-            CK(mark(ctx, 2), "event");
-            launch_k4_any(ctx, (int)p0, npc, s);
-            CK(mark(ctx, 3), "event");
-            ctx->launches += 2;
-        }
-        if (ctx->prec) {   // D5: per-pair reduction of the partials into the K5/K6 key
-            d5_argmax_keys<<<(unsigned)((np + 7) / 8), 256, 0, s>>>(ctx->part_v, ctx->part_i,
-                                                                   ctx->keys, o->nblk64, (int)np);
-            CK(mark(ctx, 3), "event");
-            ctx->launches += 1;
-        }
-        CK(cudaGetLastError(), "pair launch");
-    }
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[2], s), "event");
-    if (np > 0) {
-        for (int64_t p0 = 0; p0 < np; p0 += 65535) {
-            const int npc = (int)(np - p0 < 65535 ? np - p0 : 65535);
-            o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, s);
-            CK(mark(ctx, 4), "event");
-            ctx->launches += 1;
-        }
-        k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, s>>>(ctx->keys, ctx->mom, ctx->res,
-                                                                 ctx->H, ctx->W, (int)np,
-                                                                 k6_peak_div(ctx));
-        CK(mark(ctx, 5), "event");
-        ctx->launches += 1;
-        CK(cudaGetLastError(), "ccf launch");
-    }
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[3], s), "event");
-    ctx->computed = true;
-    return STITCH_OK;
-}
-
-// Start of a step: reset launch counters and (timing modes) record the start events.
-static stitch_status step_begin(stitch_ctx* ctx) {
-    cudaStream_t s = ctx->stream;
-    ctx->launches = 0;
-    ctx->kkind.clear();
-    ctx->computed = false;
-    if (ctx->timing >= 2) {
-        if (ctx->kev.empty()) {
-            ctx->kev.resize(1024, nullptr);
-            for (auto& e : ctx->kev) CK(cudaEventCreate(&e), "event create");
-        }
-        CK(cudaEventRecord(ctx->kev[0], s), "event");
-    }
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[0], s), "event");
-    return STITCH_OK;
-}
-
-// Enqueue `body` (which launches on ctx->stream) directly, or -- graph mode, no event
-// timing -- as a CUDA graph captured once per key on the internal capture stream and
-// replayed on the caller's stream.  Every launch parameter (pointers, tensor maps, chunk
-// schedule) is fixed per context, so a replay is exactly the captured sequence.
-// Whole step on three streams (timing off): s_fwd runs the forward chunks (K1, K2) and
-// records an event per chunk; s_pair runs the pair chunks (K3, K4), each waiting for the
-// forward chunk that completes the tiles it reads; s_ccf runs K5 per pair chunk behind
-// its K4, then K6.  Buffers G (s_fwd) and Q (s_pair) are only touched by one stream.
-// host_src (optional): the caller's host copy of the resident tiles [h_begin, t_end); each
-// forward chunk's tiles are copied on a fourth stream just before that chunk's K1, so the
-// H2D of later chunks overlaps the transforms and pairs of earlier ones (step 1 pipelined
-// with steps 2-7, as the paper's read/copier stages feed its GPU stages).
-// forward = false: steps 3-7 only (the split multi-GPU step: spectra already resident).
-static stitch_status compute_concurrent(stitch_ctx* ctx, const uint16_t* host_src = nullptr,
-                                        bool forward = true) {
-    const PlanOps* o = ctx->ops;
-    cudaStream_t m = ctx->stream;
-    const int64_t np = ctx->L.npairs;
-    const int nl = ctx->L.nlocal, ct = ctx->L.chunk_tiles, cp = ctx->L.chunk_pairs;
-    if (np > 0) {
-        CK(cudaMemsetAsync(ctx->keys, 0, (size_t)np * sizeof(unsigned long long), m), "memset");
-        CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), m), "memset");
-    }
-    if (ctx->timing == 3) {
-        ctx->tl.clear();
-        ctx->tl_used = 0;
-        CK(tl_event(ctx, &ctx->tl_origin), "event");
-        CK(cudaEventRecord(ctx->tl_origin, m), "event");
-    }
-    CK(cudaEventRecord(ctx->ev_fork, m), "fork");
-    for (cudaStream_t st : {ctx->s_fwd, ctx->s_pair, ctx->s_ccf, ctx->s_h2d, ctx->s_pair4})
-        if (st) CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
-    cudaStream_t sf = ctx->s_fwd, sp = ctx->s_pair, sk = ctx->s_ccf;
-    const size_t tile_px = (size_t)ctx->H * ctx->W;
-    for (int f = 0, t0 = 0; forward && t0 < nl; ++f, t0 += ct) {
-        const int nt = nl - t0 < ct ? nl - t0 : ct;
-        if (host_src) {
-            CK(cudaMemcpyAsync(ctx->raw + (size_t)t0 * tile_px, host_src + (size_t)t0 * tile_px,
-                               (size_t)nt * tile_px * sizeof(uint16_t), cudaMemcpyHostToDevice,
-                               ctx->s_h2d),
-               "chunk H2D");
-            CK(cudaEventRecord(ctx->ev_h2d[f], ctx->s_h2d), "event");
-            CK(cudaStreamWaitEvent(sf, ctx->ev_h2d[f], 0), "wait H2D");
-        }
-        CK(tl_wrap(ctx, sf, 0, 0, [&] { launch_k1_any(ctx, t0, nt, sf); }), "timeline");
-        CK(tl_wrap(ctx, sf, 0, 1, [&] { launch_k2_any(ctx, t0, nt, sf); }), "timeline");
-        CK(cudaEventRecord(ctx->ev_fwd[f], sf), "event");
-        ctx->launches += 2;
-    }
-    int waited = -1;
-    for (int c = 0; (int64_t)c * cp < np; ++c) {
-        const int64_t p0 = (int64_t)c * cp;
-        const int npc = (int)(np - p0 < cp ? np - p0 : cp);
-        const int need = ctx->pair_need[c];
-        if (forward && need > waited) {
-            CK(cudaStreamWaitEvent(sp, ctx->ev_fwd[need], 0), "wait forward");
-            waited = need;
-        }
-        if (ctx->s_pair4) {   // dual schedule: slot c&1, K3 and K4 on their own streams
-            float2* q = (c & 1) ? ctx->Q2 : ctx->Q;
-            if (c >= 2) CK(cudaStreamWaitEvent(sp, ctx->ev_k4[c - 2], 0), "wait slot");
-            launch_k3_any(ctx, (int)p0, npc, sp, q);
-            CK(cudaEventRecord(ctx->ev_k3[c], sp), "event");
-            CK(cudaStreamWaitEvent(ctx->s_pair4, ctx->ev_k3[c], 0), "wait k3");
-            launch_k4_any(ctx, (int)p0, npc, ctx->s_pair4, q, ctx->grid_k4w_dual);
-            CK(cudaEventRecord(ctx->ev_k4[c], ctx->s_pair4), "event");
-        } else {
-            CK(tl_wrap(ctx, sp, 1, 2, [&] { launch_k3_any(ctx, (int)p0, npc, sp); }), "timeline");
-            CK(tl_wrap(ctx, sp, 1, 3, [&] { launch_k4_any(ctx, (int)p0, npc, sp); }), "timeline");
-            CK(cudaEventRecord(ctx->ev_k4[c], sp), "event");
-        }
-        CK(cudaStreamWaitEvent(sk, ctx->ev_k4[c], 0), "wait k4");
-        CK(tl_wrap(ctx, sk, 2, 4, [&] {
-               o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)p0, npc, sk);
-           }), "timeline");
-        ctx->launches += 3;
-    }
-    if (np > 0) {
-        CK(tl_wrap(ctx, sk, 2, 5, [&] {
-               k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
-                   ctx->keys, ctx->mom, ctx->res, ctx->H, ctx->W, (int)np, k6_peak_div(ctx));
-           }), "timeline");
-        ctx->launches += 1;
-    }
-    CK(cudaGetLastError(), "concurrent launch");
-    // (s_h2d's last copy is ordered before the last K1 on s_fwd, and every K4 on s_pair4 before
-    // a K5 on s_ccf, so joining s_fwd, s_pair and s_ccf covers all streams)
-    cudaStream_t ss[3] = {sf, sp, sk};
-    for (int i = 0; i < 3; ++i) {
-        CK(cudaEventRecord(ctx->ev_join[i], ss[i]), "join");
-        CK(cudaStreamWaitEvent(m, ctx->ev_join[i], 0), "join wait");
-    }
-    ctx->computed = true;
-    return STITCH_OK;
-}
-
-extern "C++" {
-template <class F>
-static stitch_status run_graphed(stitch_ctx* ctx, uint64_t key, F body) {
-    if (ctx->timing || !ctx->use_graph) return body();
-    auto it = ctx->graphs.find(key);
-    if (it == ctx->graphs.end()) {
-        cudaStream_t user = ctx->stream;
-        const int64_t l0 = ctx->launches;
-        ctx->stream = ctx->cap_stream;
-        cudaError_t e = cudaStreamBeginCapture(ctx->cap_stream, cudaStreamCaptureModeThreadLocal);
-        if (e != cudaSuccess) {
-            ctx->stream = user;
-            return cuda_fail(ctx, e, "begin capture");
-        }
-        stitch_status st = body();
-        cudaGraph_t g = nullptr;
-        e = cudaStreamEndCapture(ctx->cap_stream, &g);
-        ctx->stream = user;
-        if (st != STITCH_OK) {
-            if (g) cudaGraphDestroy(g);
-            return st;
-        }
-        if (e != cudaSuccess) return cuda_fail(ctx, e, "end capture");
-        cudaGraphExec_t ex = nullptr;
-        e = cudaGraphInstantiate(&ex, g, 0);
-        cudaGraphDestroy(g);
-        if (e != cudaSuccess) return cuda_fail(ctx, e, "graph instantiate");
-        it = ctx->graphs.emplace(key, stitch_ctx::GraphRec{ex, ctx->launches - l0}).first;
-        ctx->launches = l0;
-    }
-    CK(cudaGraphLaunch(it->second.exec, ctx->stream), "graph launch");
-    ctx->launches += it->second.launches;
-    return STITCH_OK;
-}
-}  // extern "C++" 
 
 stitch_status stitch_forward_async(stitch_ctx* ctx) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
-    if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
     return stitch_forward_range_async(ctx, ctx->L.h_begin, ctx->L.nlocal);
 }
 
 stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, int32_t count) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (ctx->L.pool) return fail(ctx, STITCH_ERR_STATE, "split step: not in the bounded mode");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "forward before load");
     if (count < 0 || first_tile < ctx->L.h_begin || first_tile + (int64_t)count > ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
+    GUARD(ctx);
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
+    const int lt0 = first_tile - ctx->L.h_begin, ct = ctx->L.chunk_tiles;
     const uint64_t key = (2ull << 60) | ((uint64_t)(uint32_t)first_tile << 30) | (uint32_t)count;
-    st = run_graphed(ctx, key, [&]() { return forward_impl(ctx, first_tile - ctx->L.h_begin, count); });
+    st = run_graphed(ctx, key, [&]() -> stitch_status {
+        for (int t0 = lt0; t0 < lt0 + count; t0 += ct) {
+            const int nt = std::min(ct, lt0 + count - t0);
+            if (ctx->prec) {
+                ctx->ops->d1(ctx->raw, ctx->Gd, t0, nt, ctx->twMd, ctx->twWd, ctx->stream);
+                ctx->ops->d2(ctx->Gd, ctx->Ud, t0, nt, ctx->twHd, true, ctx->stream);
+                ctx->launches += 2;
+            } else {
+                launch_fwd(ctx, t0, nt, ctx->stream, 0);
+            }
+        }
+        CK(cudaGetLastError(), "forward launch");
+        return STITCH_OK;
+    });
     if (st == STITCH_OK && ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
     return st;
 }
 
-stitch_status stitch_pairs_async(stitch_ctx* ctx) {
+stitch_status stitch_pairs_part_async(stitch_ctx* ctx, int32_t part) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (part < 0 || part > 2) return fail(ctx, STITCH_ERR_INVALID_ARG, "part must be 0, 1 or 2");
+    if (ctx->L.pool) return fail(ctx, STITCH_ERR_STATE, "split step: not in the bounded mode");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "pairs before load");
-    stitch_status st = run_graphed(ctx, 3ull << 60, [&]() {
-        // K5 on its own stream beside the K3/K4 chunks, as in the whole step
-        if (ctx->concurrent && !ctx->timing) return compute_concurrent(ctx, nullptr, false);
-        return pairs_impl(ctx);
-    });
+    if (ctx->prec && part != 0) return fail(ctx, STITCH_ERR_UNSUPPORTED, "fp64: part 0 only");
+    GUARD(ctx);
+    if (ctx->prec) {
+        stitch_status st = step_begin(ctx);
+        if (st != STITCH_OK) return st;
+        st = enqueue_fp64(ctx, false, true);
+        if (st == STITCH_OK) ctx->computed = true;
+        return st == STITCH_OK ? step_end(ctx) : st;
+    }
+    const int c0 = part == 2 ? ctx->c_boundary : 0;
+    const int c1 = part == 1 ? ctx->c_boundary : (int)ctx->pch.size();
+    const int64_t pa = part == 2 ? ctx->n_interior : 0;
+    const int64_t pb = part == 1 ? ctx->n_interior : ctx->L.npairs;
+    std::vector<Op> ops;
+    for (int c = c0; c < c1; ++c) ops.push_back(Op{Op::PAIR, c});
+    stitch_status st = run_graphed(ctx, (3ull << 60) | (uint64_t)part,
+                                   [&]() { return enqueue_ops(ctx, ops, nullptr, false, pa, pb); });
     if (st == STITCH_OK) ctx->computed = true;
     return st;
 }
 
+stitch_status stitch_pairs_async(stitch_ctx* ctx) { return stitch_pairs_part_async(ctx, 0); }
+
 stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (ctx->L.pool)
+        return fail(ctx, STITCH_ERR_STATE,
+                    "bounded-mode context: use stitch_compute_translations_from_host_async");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "compute before load");
+    GUARD(ctx);
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
     st = run_graphed(ctx, 1ull << 60, [&]() {
-        if (ctx->concurrent && (!ctx->timing || ctx->timing == 3)) return compute_concurrent(ctx);
-        stitch_status s2 = forward_impl(ctx, 0, ctx->L.nlocal);
-        if (s2 != STITCH_OK) return s2;
-        if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], ctx->stream), "event");
-        return pairs_impl(ctx);
+        if (ctx->prec) return enqueue_fp64(ctx, true, true);
+        return enqueue_ops(ctx, ctx->ops_step, nullptr, true, 0, ctx->L.npairs);
     });
     if (st == STITCH_OK) ctx->computed = true;
-    return st;
+    return st == STITCH_OK ? step_end(ctx) : st;
 }
 
 stitch_status stitch_compute_translations_from_host_async(stitch_ctx* ctx, const uint16_t* tiles,
@@ -1357,73 +1516,48 @@ stitch_status stitch_compute_translations_from_host_async(stitch_ctx* ctx, const
     if (!tiles) return fail(ctx, STITCH_ERR_INVALID_ARG, "null tiles pointer");
     if (first_tile > ctx->L.h_begin || first_tile + (int64_t)count < ctx->L.t_end || first_tile < 0)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range does not cover [halo_begin, tile_end)");
+    GUARD(ctx);
     const uint16_t* src = tiles + (size_t)(ctx->L.h_begin - first_tile) * ctx->H * ctx->W;
     cudaPointerAttributes pa;
     const bool pinned = cudaPointerGetAttributes(&pa, tiles) == cudaSuccess &&
                         pa.type == cudaMemoryTypeHost;
     cudaGetLastError();   // clear a pointer-query error on pageable memory
-    if (!ctx->concurrent || ctx->timing || !pinned) {   // no pipelining: load, then the step
-        stitch_status st = stitch_load_tiles(ctx, tiles, first_tile, count, 0);
+    if (ctx->prec) {      // fp64: load, then compute
+        stitch_status st = load_common(ctx, tiles, first_tile, count, false);
         if (st != STITCH_OK) return st;
         return stitch_compute_translations_async(ctx);
     }
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
-    ctx->loaded = true;
-    // one captured graph per host buffer address (the copies' source is baked into it)
-    const uint64_t key = (4ull << 60) ^ (uint64_t)reinterpret_cast<uintptr_t>(src);
-    st = run_graphed(ctx, key, [&]() { return compute_concurrent(ctx, src); });
-    if (st == STITCH_OK) ctx->computed = true;
-    return st;
+    auto body = [&]() { return enqueue_ops(ctx, ctx->ops_step, src, true, 0, ctx->L.npairs); };
+    // pinned: one captured graph whose H2D nodes are re-pointed at each new buffer; pageable
+    // memory cannot be captured (its copies are staged by the driver): direct launches
+    st = pinned ? run_graphed(ctx, 4ull << 60, body, src) : body();
+    if (st != STITCH_OK) return st;
+    if (!ctx->L.pool) ctx->loaded = true;   // resident: every tile is now on the device
+    ctx->computed = true;
+    return step_end(ctx);
 }
 
 stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t count,
                                    void** dev_ptr, size_t* bytes) {
     if (!ctx || !dev_ptr || !bytes) return STITCH_ERR_INVALID_ARG;
+    if (ctx->L.pool) return fail(ctx, STITCH_ERR_STATE, "bounded mode: spectra are not resident");
     if (count < 0 || first_tile < ctx->L.h_begin || first_tile + (int64_t)count > ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
     const size_t per =
         (size_t)ctx->H * ctx->ops->WP * (ctx->prec ? sizeof(double2) : sizeof(uint32_t));
-    *dev_ptr = reinterpret_cast<char*>(ctx->spec) + (size_t)(first_tile - ctx->L.h_begin) * per;
+    *dev_ptr = reinterpret_cast<char*>(ctx->prec ? (void*)ctx->Ud : (void*)ctx->spec) +
+               (size_t)(first_tile - ctx->L.h_begin) * per;
     *bytes = (size_t)count * per;
     return STITCH_OK;
-}
-
-static cudaError_t collect_timings(stitch_ctx* ctx) {
-    cudaError_t e = cudaSuccess;
-    if (ctx->timing == 3) {
-        ctx->tl_ms.assign(2 * ctx->tl.size(), 0.f);
-        for (size_t i = 0; i < ctx->tl.size(); ++i) {
-            if ((e = cudaEventElapsedTime(&ctx->tl_ms[2 * i], ctx->tl_origin, ctx->tl[i].a)) !=
-                    cudaSuccess ||
-                (e = cudaEventElapsedTime(&ctx->tl_ms[2 * i + 1], ctx->tl_origin, ctx->tl[i].b)) !=
-                    cudaSuccess)
-                return e;
-        }
-        return cudaSuccess;
-    }
-    if (ctx->timing) {
-        for (int i = 0; i < 3; ++i)
-            if ((e = cudaEventElapsedTime(&ctx->ms[i], ctx->ev[i], ctx->ev[i + 1])) != cudaSuccess)
-                return e;
-        if ((e = cudaEventElapsedTime(&ctx->ms[3], ctx->ev[0], ctx->ev[3])) != cudaSuccess) return e;
-    }
-    if (ctx->timing >= 2) {
-        for (int k = 0; k < 6; ++k) { ctx->kms[k] = 0.f; ctx->kcount[k] = 0; }
-        for (size_t i = 0; i < ctx->kkind.size(); ++i) {
-            float t = 0.f;
-            if ((e = cudaEventElapsedTime(&t, ctx->kev[i], ctx->kev[i + 1])) != cudaSuccess) return e;
-            const int k = ctx->kkind[i];
-            if (k >= 0) { ctx->kms[k] += t; ctx->kcount[k] += 1; }
-        }
-    }
-    return cudaSuccess;
 }
 
 stitch_status stitch_get_translations(stitch_ctx* ctx, stitch_pair* west, stitch_pair* north) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (!west || !north) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output array");
     if (!ctx->computed) return fail(ctx, STITCH_ERR_STATE, "no computed translations");
+    GUARD(ctx);
     const int64_t np = ctx->L.npairs;
     if (np > 0)
         CK(cudaMemcpyAsync(ctx->res_h.data(), ctx->res, (size_t)np * sizeof(stitch_pair),
@@ -1461,12 +1595,13 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
     if (ctx->prec) return fail(ctx, STITCH_ERR_STATE, "fp64 context: use stitch_debug_spectrum_f64");
+    GUARD(ctx);
     // The resident store keeps Q15 unit phasors; recompute the complex spectrum of this tile
     // with the same K1 + K2 kernels into the chunk buffer G (slot 0) and copy it out.
     const int lt = tile - ctx->L.h_begin;
     const PlanOps* o = ctx->ops;
-    launch_k1_any(ctx, lt, 1, ctx->stream);
-    o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->twH, false, 0, ctx->stream);
+    o->k1(ctx->raw, ctx->G, lt, 1, ctx->fslot, ctx->twM, ctx->twW, ctx->grid_k1, ctx->stream);
+    o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->fslot, ctx->twH, false, 0, ctx->stream);
     CK(cudaGetLastError(), "spectrum launch");
     CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->G,
                          ctx->ops->WP * sizeof(float2), ctx->ops->WC * sizeof(float2), ctx->H,
@@ -1483,6 +1618,7 @@ stitch_status stitch_debug_spectrum_f64(stitch_ctx* ctx, int32_t tile, double* h
     if (tile < ctx->L.h_begin || tile >= ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile not resident");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
+    GUARD(ctx);
     // the resident store keeps unit phasors: recompute this tile's complex spectrum with the
     // same D1 + D2 kernels into chunk slot 0 of Gd (D2 writing complex values in place)
     const int lt = tile - ctx->L.h_begin;
@@ -1498,8 +1634,33 @@ stitch_status stitch_debug_spectrum_f64(stitch_ctx* ctx, int32_t tile, double* h
     return STITCH_OK;
 }
 
+stitch_status stitch_debug_surface(stitch_ctx* ctx, int32_t tile, int32_t kind, float* host_out) {
+    if (!ctx) return STITCH_ERR_INVALID_ARG;
+    if (!host_out) return fail(ctx, STITCH_ERR_INVALID_ARG, "null output");
+    if (ctx->prec || ctx->L.pool)
+        return fail(ctx, STITCH_ERR_STATE, "surface hook: fp32 resident contexts only");
+    if (!ctx->computed) return fail(ctx, STITCH_ERR_STATE, "surface before a compute");
+    int64_t p = -1;
+    for (int64_t i = 0; i < ctx->L.npairs; ++i)
+        if (ctx->pair_tile[i] == tile && ctx->pair_kind[i] == kind) p = i;
+    if (p < 0) return fail(ctx, STITCH_ERR_INVALID_ARG, "the context computes no such pair");
+    GUARD(ctx);
+    const PlanOps* o = ctx->ops;
+    float* surf = reinterpret_cast<float*>(ctx->G);   // H*W floats fit one chunk slot of G
+    const float scale = (float)(1.0 / ((double)ctx->W * ctx->H * NCPS_Q15_SCALE));
+    o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p, 1, ctx->twH, ctx->stream);
+    o->k4s(ctx->Q, surf, scale, ctx->twM, ctx->twW, ctx->grid_k4, ctx->stream);
+    CK(cudaGetLastError(), "surface launch");
+    CK(cudaMemcpyAsync(host_out, surf, (size_t)ctx->H * ctx->W * sizeof(float),
+                       cudaMemcpyDeviceToHost, ctx->stream),
+       "copy surface");
+    CK(cudaStreamSynchronize(ctx->stream), "synchronize");
+    return STITCH_OK;
+}
+
 stitch_status stitch_synchronize(stitch_ctx* ctx) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
+    GUARD(ctx);
     CK(cudaStreamSynchronize(ctx->stream), "synchronize");
     if (ctx->computed) CK(collect_timings(ctx), "event timing");
     return STITCH_OK;
@@ -1518,7 +1679,11 @@ stitch_status stitch_last_counts(stitch_ctx* ctx, int64_t* launches, int64_t* fo
                                  int64_t* pairs) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (launches) *launches = ctx->launches;
-    if (forward_ffts) *forward_ffts = ctx->L.nlocal;
+    if (forward_ffts) {
+        int64_t f = 0;
+        for (const FwdChunk& fc : ctx->fwd) f += fc.nt;
+        *forward_ffts = f;
+    }
     if (pairs) *pairs = ctx->L.npairs;
     return STITCH_OK;
 }
@@ -1532,6 +1697,8 @@ stitch_status stitch_last_timings(stitch_ctx* ctx, float* ms4) {
 stitch_status stitch_set_timing(stitch_ctx* ctx, int enabled) {
     if (!ctx) return STITCH_ERR_INVALID_ARG;
     if (enabled < 0 || enabled > 3) return fail(ctx, STITCH_ERR_INVALID_ARG, "timing mode 0..3");
+    if (enabled == 3 && !ctx->concurrent)
+        return fail(ctx, STITCH_ERR_STATE, "timeline needs the concurrent schedule");
     ctx->timing = enabled;
     return STITCH_OK;
 }

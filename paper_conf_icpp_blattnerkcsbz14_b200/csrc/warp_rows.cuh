@@ -154,7 +154,8 @@ __device__ __forceinline__ void rowwarp_tables(float2* tw2s, float2* twWs, const
 template <class PL>
 __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB1)
     k1w_fwd_rows(const uint16_t* __restrict__ raw, float2* __restrict__ G, int tile0, int ntiles,
-                 const float2* __restrict__ tw2, const float2* __restrict__ twW) {
+                 const int32_t* __restrict__ fslot, const float2* __restrict__ tw2,
+                 const float2* __restrict__ twW) {
     using RW = RowWarp<PL>;
     constexpr int M = PL::M, H = PL::H;
     extern __shared__ __align__(128) unsigned char smem_w[];
@@ -175,9 +176,11 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB1)
     const long long nrows = (long long)ntiles * H;
     const long long gw = (long long)blockIdx.x * ROWW_WARPS + warp, nw = (long long)gridDim.x * ROWW_WARPS;
     const int r0 = (int)(nrows * gw / nw), r1 = (int)(nrows * (gw + 1) / nw);
-    auto issue = [&](int r) {                  // global row r = tile*H + y of this chunk
+    auto issue = [&](int r) {                  // row r = tl*H + y of this chunk, tile in its slot
+        const int tl = r / H;
+        const size_t slot = (size_t)__ldg(fslot + tile0 + tl);
         mbar_arrive_expect_tx(bar, RW::RAWB);
-        bulk_g2s(mine, raw + ((size_t)tile0 * H + r) * PL::W, RW::RAWB, bar);
+        bulk_g2s(mine, raw + (slot * H + (r - tl * H)) * PL::W, RW::RAWB, bar);
     };
     if (lane == 0 && r0 < r1) issue(r0);
     int k = 0;
@@ -281,12 +284,54 @@ struct WarpArgmaxPfa {
     }
 };
 
+// Test hook (stitch_debug_surface): the same two transforms with the correlation surface
+// |x| * scale stored row-major instead of reduced (best_v / best_i unused).
+struct WarpSurfaceDst {
+    float best_v;
+    uint32_t best_i;
+    int row_base, W;
+    float* out;
+    float scale;
+    static constexpr bool BATCH = true;
+    template <int R, int STRIDE>
+    __device__ __forceinline__ void store_batch(int line, int b, const float2 (&v)[R]) {
+        float* o = out + (size_t)(row_base + line) * W;
+#pragma unroll
+        for (int j = 0; j < R; ++j) {
+            const int n = b + j * STRIDE;
+            o[2 * n] = fabsf(v[j].x) * scale;
+            o[2 * n + 1] = fabsf(v[j].y) * scale;
+        }
+    }
+};
+template <int R1, int C1, int C2, int N>
+struct WarpSurfacePfa {
+    float best_v;
+    uint32_t best_i;
+    int row_base, W;
+    float* out;
+    float scale;
+    __device__ __forceinline__ void store_pfa(int k1, const float2 (&v)[R1]) {
+        float* o = out + (size_t)row_base * W;
+        int n = (C1 * k1) % N;
+#pragma unroll
+        for (int j = 0; j < R1; ++j) {
+            o[2 * n] = fabsf(v[j].x) * scale;
+            o[2 * n + 1] = fabsf(v[j].y) * scale;
+            n += C2;
+            if (n >= N) n -= N;
+        }
+    }
+};
+
 // PFA: the prime-factor row transform (WarpFftPfa + WarpArgmaxPfa) where the radices are
 // coprime; otherwise Stockham with stage-2 twiddles (WarpFft2 + WarpArgmaxDst).
-template <class PL, bool PFA = false>
+// SURF: the test hook's surface output (one pair, `surf` [H][W]) instead of the argmax.
+template <class PL, bool PFA = false, bool SURF = false>
 __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
     k4w_pair_rows(const float2* __restrict__ Q, unsigned long long* __restrict__ keys, int pair0,
-                  int npairs, const float2* __restrict__ tw2, const float2* __restrict__ twW) {
+                  int npairs, const float2* __restrict__ tw2, const float2* __restrict__ twW,
+                  float* __restrict__ surf = nullptr, float scale = 0.f) {
     using RW = RowWarp<PL>;
     constexpr int M = PL::M, H = PL::H;
     extern __shared__ __align__(128) unsigned char smem_w[];
@@ -321,16 +366,22 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
     };
     if (lane == 0 && r0 < r1) issue(r0);
     using Pfa = WarpFftPfa<typename PL::Row, +1>;
-    using Acc = std::conditional_t<PFA,
-                                   WarpArgmaxPfa<RW::RI::R0, RW::RI::R1, Pfa::C1, Pfa::C2, PL::M>,
-                                   WarpArgmaxDst<RW::RI::R0>>;
-    Acc acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
+    using ArgAcc = std::conditional_t<PFA,
+                                      WarpArgmaxPfa<RW::RI::R0, RW::RI::R1, Pfa::C1, Pfa::C2, PL::M>,
+                                      WarpArgmaxDst<RW::RI::R0>>;
+    using SurfAcc = std::conditional_t<PFA, WarpSurfacePfa<RW::RI::R1, Pfa::C1, Pfa::C2, PL::M>,
+                                       WarpSurfaceDst>;
+    using Acc = std::conditional_t<SURF, SurfAcc, ArgAcc>;
+    Acc acc = [&] {
+        if constexpr (SURF) return Acc{-1.f, 0xFFFFFFFFu, 0, PL::W, surf, scale};
+        else return Acc{-1.f, 0xFFFFFFFFu, 0, PL::W};
+    }();
     int cur = r0 < r1 ? r0 / H : -1;
     int k = 0;
     for (int r = r0; r < r1; ++r, ++k) {
         const int pl = r / H, y = r - pl * H;
         if (pl != cur) {                       // warp-uniform
-            flush(cur, acc.best_v, acc.best_i);
+            if constexpr (!SURF) flush(cur, acc.best_v, acc.best_i);
             cur = pl;
             acc.best_v = -1.f;
             acc.best_i = 0xFFFFFFFFu;
@@ -367,7 +418,8 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
             RW::IFft::run(src, xc, acc, tw2s, lane, prefetch);
         __syncwarp();                          // exchange free for the next row
     }
-    if (cur >= 0) flush(cur, acc.best_v, acc.best_i);
+    if constexpr (!SURF)
+        if (cur >= 0) flush(cur, acc.best_v, acc.best_i);
 }
 
 }  // namespace stitch

@@ -113,19 +113,46 @@ def gather_translations(west: np.ndarray, north: np.ndarray, bd: Band, group=Non
 
 
 class BandPciam:
-    """One rank's share of a grid: a PciamGrid over its band plus the halo exchange."""
+    """One rank's share of a grid: a PciamGrid over its band plus the halo exchange.
+
+    transport:
+      "library"   -- the library's own NCCL send/recv (stitch_config.nccl_id; rank 0 makes the
+                     id, torch.distributed broadcasts it): one call per step, the exchange on
+                     the library's comm stream overlapped with the interior pairs;
+      "torch"     -- the same exchange through torch.distributed (NCCL, or gloo staging through
+                     host memory in the CPU tests) on a side stream, overlapped the same way:
+                     forward(owned) -> [interior pairs || halo exchange] -> boundary pairs;
+      "recompute" -- no exchange: the halo row's forward transforms are recomputed locally.
+    The exchange needs every band but the last to hold >= one tile row (exchange_feasible);
+    otherwise every transport falls back to "recompute"."""
 
     def __init__(self, n: int, m: int, H: int, W: int, rank: int, world: int, device: int = 0,
-                 exchange: bool = True, group=None, **kw):
-        from . import PciamGrid
+                 exchange: bool = True, group=None, transport: str | None = None, **kw):
+        from . import PciamGrid, nccl_unique_id
         self.n, self.m, self.H, self.W = n, m, H, W
         self.rank, self.world, self.group = rank, world, group
         self.bd = band(rank, world, n, m)
         self.plan = halo_plan(rank, world, n, m)
-        self.use_exchange = exchange and exchange_feasible(world, n, m)
-        self.grid = PciamGrid(n, m, H, W, device=device, tile_begin=self.bd.t_begin,
-                              tile_end=self.bd.t_end, **kw)
+        if transport is None:
+            transport = "torch" if exchange else "recompute"
+        if transport not in ("library", "torch", "recompute"):
+            raise ValueError("transport must be library, torch or recompute")
+        if not exchange_feasible(world, n, m):
+            transport = "recompute"
+        self.transport = transport
+        self.use_exchange = transport != "recompute"
+        if transport == "library":
+            import torch.distributed as dist
+            obj = [nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0, group=group)
+            self.grid = PciamGrid(n, m, H, W, device=device, rank=rank, world_size=world,
+                                  nccl_id=obj[0], **kw)
+        else:
+            self.grid = PciamGrid(n, m, H, W, device=device, tile_begin=self.bd.t_begin,
+                                  tile_end=self.bd.t_end, **kw)
+        assert (self.grid.tile_begin, self.grid.tile_end) == (self.bd.t_begin, self.bd.t_end)
         self.npairs = self.grid.npairs
+        self._comm_stream = None
 
     def load_rows(self, rows, first_tile: int | None = None) -> None:
         """Tiles of rows [row_begin, row_end) ([rows, m, H, W], host or device)."""
@@ -133,18 +160,28 @@ class BandPciam:
                              else first_tile)
 
     def step_async(self) -> None:
-        """Steps 2-7 for the band: forward the owned tiles, exchange the halo row's
-        spectra with the neighbouring ranks, then every owned pair."""
-        if not self.use_exchange:
-            self.grid.compute_translations_async()     # halo recomputed locally
+        """Steps 2-7 for the band: forward the owned tiles; then the interior pairs while the
+        halo row's spectra move from rank-1 (and this band's last row to rank+1); then the
+        boundary pairs (tile A in the halo)."""
+        if self.transport in ("recompute", "library"):
+            self.grid.compute_translations_async()     # halo recomputed / exchanged inside
             return
         import torch
-        self.grid.forward_range_async(self.bd.t_begin, self.bd.owned)
-        send = self.grid.spectra_view(*self.plan.send) if self.plan.send else None
-        recv = self.grid.spectra_view(*self.plan.recv) if self.plan.recv else None
-        with torch.cuda.stream(self.grid.stream):   # NCCL ordered after the forward, before pairs
+        g = self.grid
+        g.forward_range_async(self.bd.t_begin, self.bd.owned)
+        fwd_done = torch.cuda.Event()
+        fwd_done.record(g.stream)
+        g.pairs_async(1)                               # interior: no halo spectrum needed
+        if self._comm_stream is None:
+            self._comm_stream = torch.cuda.Stream(g.device)
+        cs = self._comm_stream
+        cs.wait_event(fwd_done)
+        send = g.spectra_view(*self.plan.send) if self.plan.send else None
+        recv = g.spectra_view(*self.plan.recv) if self.plan.recv else None
+        with torch.cuda.stream(cs):                    # exchange beside the interior pairs
             exchange_halo(send, recv, self.rank, self.world, self.group)
-        self.grid.pairs_async()
+        g.stream.wait_stream(cs)
+        g.pairs_async(2)                               # boundary pairs after the halo landed
 
     def translations(self):
         return self.grid.get_translations()

@@ -60,6 +60,10 @@ def _load():
         lib.synth_tiles.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,
                                     ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_int,
                                     ctypes.c_void_p]
+        lib.synth_tiles_tex.restype = ctypes.c_int
+        lib.synth_tiles_tex.argtypes = [ctypes.c_uint64, ctypes.c_void_p, ctypes.c_void_p,
+                                        ctypes.c_int64, ctypes.c_int, ctypes.c_int, ctypes.c_int,
+                                        ctypes.c_int, ctypes.c_uint32, ctypes.c_void_p]
         lib.synth_jitter.restype = ctypes.c_int64
         lib.synth_jitter.argtypes = [ctypes.c_uint64, ctypes.c_uint64, ctypes.c_uint64,
                                      ctypes.c_int64]
@@ -121,10 +125,14 @@ def origins(n: int, m: int, H: int, W: int, overlap: float = 0.10, delta: int | 
 
 def make_grid(n: int, m: int, H: int, W: int, overlap: float = 0.10, delta: int | None = None,
               seed: int = SEED, scan: int = 0, channel: int = 0, threads: int | None = None,
-              out: np.ndarray | None = None, rows: tuple[int, int] | None = None) -> Grid:
+              out: np.ndarray | None = None, rows: tuple[int, int] | None = None,
+              texture: str = "default", density: float = 0.02) -> Grid:
     """Render an n x m grid of H x W uint16 tiles (optionally only tile rows [r0, r1)).
 
     ``out`` may be a caller-owned (e.g. pinned) uint16 array of the right shape.
+    ``texture``: "default" (value noise + per-pixel scene detail) or "cells" (the low-texture
+    scene: flat background + sparse bright cells, ``density`` = occupancy per 64 px lattice
+    cell, the paper's sparse early colonies).
     """
     lib = _load()
     if delta is None:
@@ -142,8 +150,13 @@ def make_grid(n: int, m: int, H: int, W: int, overlap: float = 0.10, delta: int 
     tex_seed = seed + 0x9E37 * channel
     if threads is None:
         threads = os.cpu_count() or 1
-    rc = lib.synth_tiles(tex_seed, sub.ctypes.data, keys.ctypes.data, nr * m, H, W, threads,
-                         out.ctypes.data)
+    if texture not in ("default", "cells"):
+        raise ValueError("texture must be 'default' or 'cells'")
+    dens = int(round(density * 65536))
+    if not 0 <= dens <= 65536:
+        raise ValueError("density must be in [0, 1]")
+    rc = lib.synth_tiles_tex(tex_seed, sub.ctypes.data, keys.ctypes.data, nr * m, H, W, threads,
+                             0 if texture == "default" else 1, dens, out.ctypes.data)
     if rc != 0:
         raise RuntimeError("synth_tiles failed")
     return Grid(out, o[r0:r1], nr, m, H, W, seed, overlap, delta)

@@ -106,6 +106,54 @@ void synth_tile(uint64_t seed, int64_t ox, int64_t oy, int H, int W,
     }
 }
 
+/*
+ * Low-texture scene ("cells" texture): the paper's
+ * sparse early colonies with "few distinguishable features".  A flat background
+ * of 2000 DN plus isolated bright cells and nothing else (no value noise, no per-pixel scene
+ * detail): lattice cell (i, j) of CELL_G px holds a cell with probability density/65536, at a
+ * hashed centre inside it, radius R in [5, 30] px, amplitude A in [3000, 30000] DN, profile
+ * A (1 - d^2/R^2)^2 for d < R (a compactly supported, Gaussian-like bump in integer
+ * arithmetic).  Per-tile read noise as above.  An overlap without cells correlates noise only.
+ */
+#define CELL_G 64
+static inline int64_t cells_at(uint64_t seed, int64_t X, int64_t Y, uint32_t density) {
+    int64_t v = 2000;
+    const int64_t ci = X / CELL_G, cj = Y / CELL_G;
+    for (int64_t j = cj - 1; j <= cj + 1; ++j) {
+        if (j < 0) continue;
+        for (int64_t i = ci - 1; i <= ci + 1; ++i) {
+            if (i < 0) continue;
+            const uint64_t h = hash3(seed ^ 0x5EEDCE11ULL, (uint64_t)i, (uint64_t)j);
+            if ((h & 0xFFFF) >= density) continue;
+            const int64_t cx = i * CELL_G + (int64_t)((h >> 16) % CELL_G);
+            const int64_t cy = j * CELL_G + (int64_t)((h >> 24) % CELL_G);
+            const int64_t R = 5 + (int64_t)((h >> 32) % 26);
+            const int64_t A = 3000 + (int64_t)((h >> 40) % 27001);
+            const int64_t dx = X - cx, dy = Y - cy, d2 = dx * dx + dy * dy, R2 = R * R;
+            if (d2 >= R2) continue;
+            const int64_t q = R2 - d2;
+            v += A * q * q / (R2 * R2);
+        }
+    }
+    return v;
+}
+
+void synth_tile_cells(uint64_t seed, int64_t ox, int64_t oy, int H, int W, uint64_t tile_key,
+                      uint32_t density, uint16_t* out) {
+    const uint64_t kn = mix64(seed ^ tile_key ^ 0x8CB92BA72F3D8DD7ULL);
+    for (int y = 0; y < H; ++y) {
+        uint16_t* row = out + (size_t)y * (size_t)W;
+        for (int x = 0; x < W; ++x) {
+            int64_t v = cells_at(seed, ox + x, oy + y, density);
+            const uint64_t hn = hash_px(kn, (uint64_t)x, (uint64_t)y);
+            for (int q = 0; q < 4; ++q) v += (int64_t)((hn >> (16 * q)) & 0xFFFF) % 35 - 17;
+            if (v < 0) v = 0;
+            if (v > 65535) v = 65535;
+            row[x] = (uint16_t)v;
+        }
+    }
+}
+
 typedef struct {
     uint64_t seed;
     const int64_t* origins;   /* [count][2] = (ox, oy) */
@@ -115,6 +163,8 @@ typedef struct {
     uint16_t* out;
     int64_t next;
     pthread_mutex_t mu;
+    int texture;          /* 0: value noise + detail (default), 1: sparse cells */
+    uint32_t density;     /* cells: lattice-cell occupancy in 1/65536 */
 } job_t;
 
 static void* worker(void* p) {
@@ -124,24 +174,37 @@ static void* worker(void* p) {
         const int64_t t = j->next++;
         pthread_mutex_unlock(&j->mu);
         if (t >= j->count) break;
-        synth_tile(j->seed, j->origins[2 * t], j->origins[2 * t + 1], j->H, j->W, j->keys[t],
-                   j->out + (size_t)t * (size_t)j->H * (size_t)j->W);
+        uint16_t* dst = j->out + (size_t)t * (size_t)j->H * (size_t)j->W;
+        if (j->texture == 1)
+            synth_tile_cells(j->seed, j->origins[2 * t], j->origins[2 * t + 1], j->H, j->W,
+                             j->keys[t], j->density, dst);
+        else
+            synth_tile(j->seed, j->origins[2 * t], j->origins[2 * t + 1], j->H, j->W, j->keys[t],
+                       dst);
     }
     return NULL;
 }
 
 /* Render `count` tiles (origins[t] = (ox, oy), keys[t] = noise key) into out[count][H][W]
- * using `threads` POSIX threads.  Returns 0 on success. */
-int synth_tiles(uint64_t seed, const int64_t* origins, const uint64_t* keys, int64_t count,
-                int H, int W, int threads, uint16_t* out) {
+ * using `threads` POSIX threads; texture 0 = the default scene, 1 = sparse cells at
+ * `density` / 65536 per lattice cell.  Returns 0 on success. */
+int synth_tiles_tex(uint64_t seed, const int64_t* origins, const uint64_t* keys, int64_t count,
+                    int H, int W, int threads, int texture, uint32_t density, uint16_t* out) {
     if (!origins || !keys || !out || H <= 0 || W <= 0 || count < 0) return 1;
+    if (texture != 0 && texture != 1) return 1;
     if (threads < 1) threads = 1;
     if (threads > 256) threads = 256;
-    job_t j = {seed, origins, keys, H, W, count, out, 0, PTHREAD_MUTEX_INITIALIZER};
+    job_t j = {seed, origins, keys, H, W, count, out, 0, PTHREAD_MUTEX_INITIALIZER, texture,
+               density};
     pthread_t th[256];
     for (int i = 0; i < threads; ++i) pthread_create(&th[i], NULL, worker, &j);
     for (int i = 0; i < threads; ++i) pthread_join(th[i], NULL);
     return 0;
+}
+
+int synth_tiles(uint64_t seed, const int64_t* origins, const uint64_t* keys, int64_t count,
+                int H, int W, int threads, uint16_t* out) {
+    return synth_tiles_tex(seed, origins, keys, count, H, W, threads, 0, 0, out);
 }
 
 /* Per-key uniform integer in [0, bound] (used for origin jitter in Python). */

@@ -1,0 +1,120 @@
+#!/usr/bin/env python3
+"""Write the full-grid oracle results the GPU parity tests compare against, element by element.
+
+    python tests/golden/make_oracle_golden.py [case ...]      (default: every case)
+
+Calls only ``oracle/`` (the fp64 CPU oracle, Fig. 4 over Fig. 2) on grids rendered by
+``synthgrid/`` (the shared seeded input generator, no method arithmetic); nothing here comes
+from the CUDA path.  The grid is processed in bands of tile rows (each band re-reads the row
+above it for its north pairs), so the oracle's resident fp64 spectra stay bounded
+(8 rows x 59 tiles x 23 MB = 11 GB at 1392x1040); results do not depend on the banding (every
+pair is pciam(neighbour, tile)).
+
+Each case is saved as ``oracle_<case>.npz``: ``west``, ``north`` ([n, m] oracle.PAIR_DTYPE) and
+``tiles_sha256`` (of the rendered uint16 grid, so a drift of the generator is caught before any
+comparison), plus the generator parameters.
+"""
+from __future__ import annotations
+
+import hashlib
+import os
+import sys
+import time
+
+import numpy as np
+
+HERE = os.path.dirname(os.path.abspath(__file__))
+ROOT = os.path.dirname(os.path.dirname(HERE))
+sys.path.insert(0, ROOT)
+
+import oracle  # noqa: E402
+import synthgrid  # noqa: E402
+
+# name -> generator parameters (BASELINE.json configs)
+CASES = {
+    # configs[1]: the paper's 18x22 cell-colony grid, 10 % overlap
+    "cfg2": dict(n=18, m=22, H=1040, W=1392, overlap=0.10, delta=12, seed=synthgrid.SEED),
+    # configs[2]: the headline 42x59 grid, 10 % overlap -- the bench's workload
+    "cfg3": dict(n=42, m=59, H=1040, W=1392, overlap=0.10, delta=12, seed=synthgrid.SEED),
+    # configs[2] at the paper-implied ~70 % overlap (reading C13)
+    "cfg3_ov70": dict(n=42, m=59, H=1040, W=1392, overlap=0.70, delta=12, seed=synthgrid.SEED),
+    # low texture (the paper's sparse early colonies): flat background + sparse
+    # cells only, so many overlaps hold no feature and their correlation peak is a near-tie of
+    # noise; the seed is the first one from `start` whose oracle result has at least
+    # `min_ambiguous` pairs with (peak - runner_up)/peak < 1e-4 (reading C17's near-tie set)
+    "lowtex256": dict(n=16, m=16, H=192, W=256, overlap=0.10, delta=4, texture="cells",
+                      density=0.02, search=dict(start=1000, min_ambiguous=3)),
+    "lowtex1392": dict(n=10, m=12, H=1040, W=1392, overlap=0.10, delta=12, texture="cells",
+                       density=0.01, search=dict(start=2000, min_ambiguous=1)),
+}
+NEAR_TIE = 1e-4
+BAND = 8
+
+
+def grid_sha(tiles_iter) -> str:
+    h = hashlib.sha256()
+    for t in tiles_iter:
+        h.update(np.ascontiguousarray(t).tobytes())
+    return h.hexdigest()
+
+
+def render(p, rows):
+    kw = {k: p[k] for k in ("overlap", "delta", "seed") if k in p}
+    if "texture" in p:
+        kw["texture"] = p["texture"]
+        kw["density"] = p["density"]
+    return synthgrid.make_grid(p["n"], p["m"], p["H"], p["W"], rows=rows, **kw)
+
+
+def ambiguous(west, north) -> int:
+    k = 0
+    for a in (west, north):
+        v = a[a["peak"] > 0]
+        k += int(((v["peak"] - v["runner_up"]) / v["peak"] < NEAR_TIE).sum())
+    return k
+
+
+def run_case(name: str, p: dict) -> None:
+    if "search" in p:
+        p = dict(p)
+        srch = p.pop("search")
+        seed = srch["start"]
+        while True:
+            p["seed"] = seed
+            g = render(p, None)
+            w, nn = oracle.grid(g.tiles)
+            k = ambiguous(w, nn)
+            print(f"{name}: seed {seed}: {k} near-tie pairs", flush=True)
+            if k >= srch["min_ambiguous"]:
+                break
+            seed += 1
+    n, m = p["n"], p["m"]
+    west = np.zeros((n, m), oracle.PAIR_DTYPE)
+    north = np.zeros((n, m), oracle.PAIR_DTYPE)
+    h = hashlib.sha256()
+    t0 = time.time()
+    for start in range(0, n, BAND):
+        end = min(n, start + BAND)
+        r0 = max(0, start - 1)
+        g = render(p, (r0, end))
+        h.update(np.ascontiguousarray(g.tiles[start - r0:]).tobytes())
+        w, nn = oracle.grid(g.tiles)
+        west[start:end] = w[start - r0:]
+        north[start:end] = nn[start - r0:]
+        if start == 0:
+            north[0] = nn[0]          # row 0 has no north pair (absent record)
+        print(f"{name}: rows {start}-{end - 1} done, {time.time() - t0:.0f} s", flush=True)
+    out = os.path.join(HERE, f"oracle_{name}.npz")
+    np.savez_compressed(out, west=west, north=north, tiles_sha256=np.array(h.hexdigest()),
+                        params=np.array(repr(sorted(p.items()))))
+    print(f"wrote {out} ({os.path.getsize(out)} bytes)", flush=True)
+
+
+def main(argv):
+    names = argv or list(CASES)
+    for name in names:
+        run_case(name, CASES[name])
+
+
+if __name__ == "__main__":
+    main(sys.argv[1:])

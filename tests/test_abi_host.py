@@ -228,3 +228,60 @@ def test_q15_phasor_encoder_and_ncps_decoder():
     p = za * np.conj(zb)
     ref = p / np.abs(p) * 32767.0 ** 2
     assert np.abs((re + 1j * im) - ref).max() <= 1e-4 * 32767.0 ** 2
+
+def test_flags_and_multirank_validation(lib):
+    """stitch_config.flags accepts only STITCH_FLAG_*; rank / world_size / nccl_id are
+    validated on the host (the library derives the band only when it owns the exchange)."""
+    b = ctypes.c_size_t()
+    cfg = pkg.make_config(3, 3, 192, 256, flags=4)
+    assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 1
+    cfg = pkg.make_config(3, 3, 192, 256, flags=pkg.FLAG_NO_GRAPH | pkg.FLAG_SERIAL)
+    assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 0
+    nid = ctypes.create_string_buffer(128)
+    vid = ctypes.cast(nid, ctypes.c_void_p)
+    for kw in (dict(world_size=1, nccl_id=vid),                         # no peers
+               dict(world_size=2, rank=2, nccl_id=vid),                 # rank out of range
+               dict(world_size=2, rank=0, tile_begin=0, tile_end=4, nccl_id=vid),
+               dict(world_size=10, rank=0)):                            # more ranks than tiles
+        cfg = pkg.make_config(3, 3, 192, 256, **kw)
+        assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 1, kw
+    cfg = pkg.make_config(3, 3, 192, 256, world_size=2, rank=0, nccl_id=vid, precision=1)
+    assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 2
+
+
+@pytest.mark.parametrize("R", [2, 3, 8])
+def test_library_derived_bands_partition_the_pairs(lib, R):
+    """world_size > 1 with tile_begin = tile_end = 0: the library's balanced band of each rank
+     -- the bands' pairs partition Table I's count."""
+    n, m = 42, 59
+    total = sum(pkg.pair_count(pkg.make_config(n, m, 1040, 1392, rank=k, world_size=R))
+                for k in range(R))
+    assert total == 2 * n * m - n - m
+
+
+def test_nccl_unique_id(lib):
+    """stitch_nccl_unique_id loads NCCL at run time (no GPU needed for the id)."""
+    a, b = pkg.nccl_unique_id(), pkg.nccl_unique_id()
+    assert len(a) == 128 and len(b) == 128 and a != b
+    assert lib.stitch_nccl_unique_id(None) == 1
+
+
+def test_bounded_pool_validation_and_size(lib):
+    """Bounded mode (row f1): the host simulation of the refcounted slot schedule rejects a pool
+    that cannot hold one tile row + one forward chunk (INVALID_ARG), accepts the smallest one
+    that can, and the workspace then shrinks with the pool instead of the grid."""
+    b = ctypes.c_size_t()
+    n, m, H, W = 6, 7, 192, 256
+    for pool, want in ((4, 1), (8, 1), (9, 0), (12, 0)):
+        cfg = pkg.make_config(n, m, H, W, pool_tiles=pool, chunk_tiles=2, chunk_pairs=3)
+        assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == want, pool
+    cfg = pkg.make_config(n, m, H, W, pool_tiles=-1)
+    assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 1
+    cfg = pkg.make_config(n, m, H, W, pool_tiles=12, precision=1)
+    assert lib.stitch_workspace_size(ctypes.byref(cfg), ctypes.byref(b)) == 2
+    # 42x59 @ 1392x1040: 128 slots instead of 2478 tiles
+    big = pkg.workspace_size(pkg.make_config(42, 59, 1040, 1392))
+    small = pkg.workspace_size(pkg.make_config(42, 59, 1040, 1392, pool_tiles=128))
+    per_tile = 1040 * 1392 * 2 + 1040 * 704 * 4
+    assert big - small >= (2478 - 128) * per_tile
+    assert small < 2.0e9

@@ -1,0 +1,79 @@
+"""The committed full-grid oracle results (tests/golden/oracle_*.npz, written by
+make_oracle_golden.py from oracle/ only) are what the oracle computes on these inputs:
+sampled pairs re-evaluated by oracle.pciam on freshly rendered tiles agree field for field,
+and every file is complete (Fig. 4: every west pair with c >= 1, every north pair with
+r >= 1, absent records elsewhere).  The low-texture fixtures hold near-tie pairs (the C17
+rule's near-tie set, margin < 1e-4), so the GPU comparison exercises that rule."""
+import ast
+import hashlib
+import os
+
+import numpy as np
+import pytest
+
+import oracle
+import synthgrid
+
+GOLD = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
+CASES = ["cfg2", "cfg3", "cfg3_ov70", "lowtex256", "lowtex1392"]
+FIELDS = ["dx", "dy", "candidate", "peak_x", "peak_y", "peak", "runner_up", "ccf"]
+
+
+def load(name):
+    path = os.path.join(GOLD, f"oracle_{name}.npz")
+    if not os.path.exists(path):
+        pytest.skip(f"{path} not generated yet")
+    z = np.load(path)
+    return dict(ast.literal_eval(str(z["params"]))), z["west"], z["north"], str(z["tiles_sha256"])
+
+
+def render(p, rows=None):
+    kw = dict(overlap=p["overlap"], delta=p["delta"], seed=p["seed"])
+    if "texture" in p:
+        kw.update(texture=p["texture"], density=p["density"])
+    return synthgrid.make_grid(p["n"], p["m"], p["H"], p["W"], rows=rows, **kw)
+
+
+@pytest.mark.parametrize("name", CASES)
+def test_golden_is_complete_and_reproduced_by_the_oracle(name):
+    p, west, north, sha = load(name)
+    n, m = p["n"], p["m"]
+    assert west.shape == (n, m) and north.shape == (n, m)
+    assert (west["candidate"][:, 0] == 0).all() and np.isnan(west["ccf"][:, 0]).all()
+    assert (north["candidate"][0] == 0).all() and np.isnan(north["ccf"][0]).all()
+    assert (west["peak"][:, 1:] > 0).all() and (north["peak"][1:] > 0).all()
+    assert (west["max_imag_ratio"] <= 1e-9).all() and (north["max_imag_ratio"] <= 1e-9).all()
+    rng = np.random.default_rng(len(name))
+    r = int(rng.integers(1, n))
+    g = render(p, rows=(r - 1, r + 1))           # rows r-1, r only
+    for c in sorted({1, int(rng.integers(1, m)), m - 1}):
+        for kind, gold in (("w", west), ("n", north)):
+            A = g.tiles[1, c - 1] if kind == "w" else g.tiles[0, c]
+            got = oracle.pciam(A, g.tiles[1, c])
+            ref = gold[r, c]
+            for f in FIELDS:
+                assert got[f] == ref[f] or (np.isnan(got[f]) and np.isnan(ref[f])), (name, r, c, f)
+    if n * m <= 400:                              # small grids: the tiles' digest too
+        assert hashlib.sha256(render(p).tiles.tobytes()).hexdigest() == sha
+
+
+@pytest.mark.parametrize("name,k", [("lowtex256", 3), ("lowtex1392", 1)])
+def test_low_texture_fixtures_hold_near_ties(name, k):
+    _, west, north, _ = load(name)
+    amb = 0
+    for a in (west, north):
+        v = a[a["peak"] > 0]
+        amb += int(((v["peak"] - v["runner_up"]) / v["peak"] < 1e-4).sum())
+    assert amb >= k
+
+
+def test_full_size_fixtures_recover_the_known_shifts():
+    """At 10 % and 70 % overlap the oracle recovers every generator shift of the headline grid
+    (a pin of the oracle at full size, independent of the GPU)."""
+    for name in ("cfg2", "cfg3", "cfg3_ov70"):
+        p, west, north, _ = load(name)
+        o = synthgrid.origins(p["n"], p["m"], p["H"], p["W"], p["overlap"], p["delta"], p["seed"])
+        assert np.array_equal(west["dx"][:, 1:], (o[:, 1:, 0] - o[:, :-1, 0])), name
+        assert np.array_equal(west["dy"][:, 1:], (o[:, 1:, 1] - o[:, :-1, 1])), name
+        assert np.array_equal(north["dx"][1:], (o[1:, :, 0] - o[:-1, :, 0])), name
+        assert np.array_equal(north["dy"][1:], (o[1:, :, 1] - o[:-1, :, 1])), name

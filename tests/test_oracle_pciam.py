@@ -207,3 +207,24 @@ def test_full_size_exact_recovery(overlap):
     valid = np.concatenate([west[:, 1:].ravel(), north[1:].ravel()])
     assert (valid["candidate"] == 1).all()
     assert ((valid["peak"] - valid["runner_up"]) / valid["peak"] > 1e-2).all()
+
+
+@pytest.mark.parametrize("shape", [(1, 2), (3, 4), (40, 48)])
+def test_zero_spectrum_branch_and_first_index_tie(shape):
+    """Readings C4 and C6 pinned with exact arithmetic.  Tile B all zeros: F_B = 0 exactly in
+    every bin (0 times any twiddle is 0), so |F_A conj(F_B)| = 0 everywhere and step 3's
+    branch sets NCC = 0 (C4) -- without it every bin is 0/0 = NaN.  The inverse of an all-zero
+    NCC is exactly 0, so all H*W surface values tie and step 5 must return the first index in
+    row-major order, (0, 0) (C6: a '>=' scan would return the last).  Every candidate then has
+    B's zero variance, so none is valid (C8): candidate 0, ccf NaN, (dx, dy) = the peak."""
+    H, W = shape
+    A = tex(max(H, 2), max(W, 2))[:H, :W] if H > 1 else np.array([[1, 0]], np.uint16)
+    B = np.zeros((H, W), np.uint16)
+    for a, b in ((A, B), (B, A)):   # also A all zeros (F_A = 0)
+        s = oracle.surface(a, b)
+        assert np.all(s == 0.0)                  # exactly zero, no NaN
+        p = oracle.pciam(a, b)
+        assert (p["peak_x"], p["peak_y"]) == (0, 0)
+        assert p["peak"] == 0.0 and p["runner_up"] == 0.0
+        assert p["candidate"] == 0 and np.isnan(p["ccf"]) and (p["dx"], p["dy"]) == (0, 0)
+        assert np.isnan(p["ccf_k"]).all()

@@ -1,14 +1,18 @@
 #!/bin/bash
 # compute-sanitizer passes over config 1 (3x3 grid of 256x192) and a 2x2 grid of 1392x1040
-# (run on the GPU box).  Graphs/concurrency off so every launch is checked directly.
-export STITCH_GRAPH=0
+# (run on the GPU box).  Graph replay off so every launch is checked directly.
 SMOKE='import __graft_entry__ as g; g.smoke()'
-BIG='import numpy as np, synthgrid; from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid
+BIG='import numpy as np, torch, synthgrid; from paper_conf_icpp_blattnerkcsbz14_b200 import PciamGrid, FLAG_NO_GRAPH
 g = synthgrid.make_grid(2, 2, 1040, 1392)
-p = PciamGrid(2, 2, 1040, 1392, chunk_pairs=2, chunk_tiles=2); p.load_grid(g.tiles); w, n = p.compute_translations()
+p = PciamGrid(2, 2, 1040, 1392, chunk_pairs=2, chunk_tiles=2, flags=FLAG_NO_GRAPH); p.load_grid(g.tiles); w, n = p.compute_translations()
+b = PciamGrid(2, 2, 1040, 1392, chunk_pairs=1, chunk_tiles=1, pool_tiles=4, flags=FLAG_NO_GRAPH)
+h = torch.empty(g.tiles.shape, dtype=torch.uint16, pin_memory=True); h.numpy()[...] = g.tiles
+b.compute_from_host_async(h, 0); wb, nb = b.get_translations()
+assert wb.tobytes() == w.tobytes() and nb.tobytes() == n.tobytes()
+s = p.surface(1, 0)
 q = PciamGrid(2, 2, 1040, 1392, precision=1); q.load_grid(g.tiles); w2, n2 = q.compute_translations()
 assert (w["dx"] == w2["dx"]).all() and (n["dy"] == n2["dy"]).all()
-print("big ok (fp32 + fp64)", w["dx"].tolist(), n["dy"].tolist())'
+print("big ok (fp32 + bounded pool + surface hook + fp64)", w["dx"].tolist(), n["dy"].tolist())'
 for tool in memcheck racecheck synccheck initcheck; do
   echo "== $tool (config 1)"
   timeout 900 compute-sanitizer --tool $tool --print-limit 20 python -c "$SMOKE" 2>&1 | tail -6
