@@ -61,6 +61,22 @@ __device__ __forceinline__ void bulk_g2s(void* dst_smem, const void* src_gmem, u
         : "memory");
 }
 
+// 1-D bulk copy shared -> global (bytes % 16 == 0, 16-byte aligned), tracked by the issuing
+// thread's bulk group: commit it, then wait until the shared source has been read (before the
+// CTA may exit or reuse the buffer).  Every thread that wrote the source must have executed
+// fence_proxy_async() and a barrier first.
+__device__ __forceinline__ void bulk_s2g(void* dst_gmem, const void* src_smem, uint32_t bytes) {
+    asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst_gmem),
+                 "r"(smem_u32(src_smem)), "r"(bytes)
+                 : "memory");
+}
+__device__ __forceinline__ void bulk_commit() {
+    asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read_all() {
+    asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
+
 }  // namespace stitch
 
 namespace stitch {

@@ -5,9 +5,11 @@
 //   raw   uint16 [slots][H][W]           tile pixels by slot (slot = tile in the resident mode;
 //                                        a recycled pool slot in the bounded mode, row f1)
 //   G     float2 [chunk][H][WP]          row-transformed tiles of a forward chunk
-//   spec  u32    [slots][H][WP]          half spectrum kx in [0, W/2] (WP = pad16(W/2+1))
-//                                        stored as its Q15 unit phasor F/|F| (2 x int16),
-//                                        reused by <= 4 pairs
+//   spec  u32    [slots][WP][HP]         half spectrum kx in [0, W/2] (WP = pad16(W/2+1)),
+//                                        COLUMN-major (ky contiguous, pitch HP = H rounded up to
+//                                        4 mod 8 words), stored as its Q15 unit phasor F/|F|
+//                                        (2 x int16), reused by <= 4 pairs: K3's
+//                                        column panel of a tile is one contiguous run
 //   Q     float2 [chunk][H][WP]          per-pair column-inverse intermediate
 //   fslot i32    [local tiles]           slot of each local tile (K1/K2 write there)
 //   pairs {a, b} [pairs]                 slots of the pair's tiles (K3/K5 read there)
@@ -58,6 +60,10 @@ struct Plan {
     static constexpr int M = W / 2;           // complex row length
     static constexpr int WC = M + 1;          // kept bins kx in [0, M]
     static constexpr int WP = pad16(WC);      // row pitch of spectra (float2)
+    // column pitch of the resident (column-major) phasor spectrum, in u32: >= H, a multiple of
+    // 4 (16-byte bulk copies) and 4 mod 8, so the 8 columns of a landed panel start in 8
+    // distinct 4-bank groups (conflict-free stage-1 reads)
+    static constexpr int HP = H % 8 <= 4 ? H + (4 - H % 8) : H + (12 - H % 8);
     using Row = RowRX;
     using Col = ColRX;
     using RI = RadixInfo<RowRX>;
@@ -70,16 +76,20 @@ struct Plan {
     static constexpr size_t ROW_SMEM = sizeof(float2) * ROW_L * RowX::LSTRIDE;
     // column kernels: a TMA landing panel [H][COL_P] (complex, or two phasor panels), reused
     // in place as the stage exchange buffer once stage 1 has read it into registers
-    // K3 lands two phasor panels: the second starts 128-byte aligned (TMA destination rule)
-    static constexpr size_t COL_PHASE_B = (sizeof(uint32_t) * COL_P * H + 127) / 128 * 128;
+    // K3 lands two phasor panels [COL_P][HP] (one bulk copy each), the second 128-B aligned
+    static constexpr size_t COL_PANEL_P = sizeof(uint32_t) * COL_P * HP;
+    static constexpr size_t COL_PHASE_B = (COL_PANEL_P + 127) / 128 * 128;
     static constexpr size_t COL_LAND_C = sizeof(float2) * COL_P * H;
-    static constexpr size_t COL_LAND_P = COL_PHASE_B + sizeof(uint32_t) * COL_P * H;
+    static constexpr size_t COL_LAND_P = COL_PHASE_B + COL_PANEL_P;
     static constexpr size_t COL_LAND = COL_LAND_C > COL_LAND_P ? COL_LAND_C : COL_LAND_P;
     static constexpr size_t COL_XCH =
         CI::STAGES == 1 ? 0 : sizeof(float2) * COL_P * CI::R1 * (CI::R0 + COL_PAD);
     static constexpr size_t COL_BUF = ((COL_LAND > COL_XCH ? COL_LAND : COL_XCH) + 15) / 16 * 16;
     static constexpr int COL_TW2N = CI::R0 * (CI::R1 - 1);      // stage-2 twiddles in smem
     static constexpr size_t COL_SMEM = COL_BUF + sizeof(float2) * (COL_TW2N > 0 ? COL_TW2N : 1);
+    // K2 stages its phasor panel [COL_P][HP] behind that and stores it with one bulk copy
+    static constexpr size_t COL_STG_OFF = (COL_SMEM + 127) / 128 * 128;
+    static constexpr size_t COL_SMEM_K2 = COL_STG_OFF + COL_PANEL_P;
     static constexpr int BOXH = H / ((H + 255) / 256);   // TMA box rows (<= 256)
     static_assert(H % BOXH == 0, "H must split into equal TMA boxes of <= 256 rows");
     static_assert((BOXH * COL_P * 4) % 128 == 0 || H == BOXH, "TMA boxes must land 128-B aligned");
@@ -204,10 +214,10 @@ __device__ __forceinline__ int32_t q15_hi(uint32_t w) { return (int32_t)w >> 16;
 constexpr double NCPS_Q15_SCALE = 32767.0 * 32767.0;
 
 template <class PL>
-struct PhaseDst {  // K2 output: Q15 unit phasors of a panel of the resident spectrum
+struct PhaseDst {  // K2 output: Q15 unit phasors of a panel [COL_P][HP] (staged in shared memory)
     uint32_t* p;
     __device__ __forceinline__ void store(int line, int n, float2 v) const {
-        p[(size_t)n * PL::WP + line] = phasor_q15(v);
+        p[line * PL::HP + n] = phasor_q15(v);
     }
 };
 
@@ -289,8 +299,20 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     typename PL::ColX xc{reinterpret_cast<float2*>(csmem)};
     using Run = FftRun<typename PL::Col, -1, PL::COL_P, PL::COL_T, ColMap, true>;
     if constexpr (PHASE_OUT) {
-        PhaseDst<PL> dst{spec + (size_t)fslot[tile0 + tl] * PL::H * PL::WP + c0};
+        // the panel's 8 columns are contiguous in the column-major spectrum: staged in shared
+        // memory (conflict-free: column pitch HP) and written with one bulk copy, instead of
+        // 8 scattered 16-byte pieces per warp store
+        uint32_t* stage = reinterpret_cast<uint32_t*>(csmem + PL::COL_STG_OFF);
+        PhaseDst<PL> dst{stage};
         Run::template run<true>(src, xc, dst, tws);
+        fence_proxy_async();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            bulk_s2g(spec + ((size_t)fslot[tile0 + tl] * PL::WP + c0) * PL::HP, stage,
+                     (uint32_t)PL::COL_PANEL_P);
+            bulk_commit();
+            bulk_wait_read_all();
+        }
     } else {
         PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
         Run::template run<true>(src, xc, dst, tws);
@@ -303,7 +325,7 @@ struct NcpsPhaseSrc {  // step 3 from two landed phasor panels: U_A conj(U_B) (x
     const uint32_t* a;
     const uint32_t* b;
     __device__ __forceinline__ float2 load(int line, int n) const {
-        const uint32_t ua = a[n * PL::COL_P + line], ub = b[n * PL::COL_P + line];
+        const uint32_t ua = a[line * PL::HP + n], ub = b[line * PL::HP + n];
         const int32_t ax = q15_lo(ua), ay = q15_hi(ua), bx = q15_lo(ub), by = q15_hi(ub);
         return make_float2((float)(ax * bx + ay * by), (float)(ay * bx - ax * by));
     }
@@ -311,7 +333,7 @@ struct NcpsPhaseSrc {  // step 3 from two landed phasor panels: U_A conj(U_B) (x
 
 template <class PL>
 __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
-    k3t_pair_cols(const __grid_constant__ CUtensorMap tmS, float2* __restrict__ Q,
+    k3t_pair_cols(const uint32_t* __restrict__ spec, float2* __restrict__ Q,
                   const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2) {
     extern __shared__ __align__(128) unsigned char csmem[];
     __shared__ uint64_t bar;
@@ -320,16 +342,16 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     uint32_t* la = reinterpret_cast<uint32_t*>(csmem);
     uint32_t* lb = reinterpret_cast<uint32_t*>(csmem + PL::COL_PHASE_B);
     if (threadIdx.x == 0) {
-        prefetch_tensormap(&tmS);
         mbar_init(&bar, 1);
         fence_mbar_init();
     }
     __syncthreads();
     float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
-    if (threadIdx.x == 0) {
-        mbar_arrive_expect_tx(&bar, (uint32_t)(2 * PL::H * PL::COL_P * 4) + ColTw<PL>::BYTES);
-        tma_panel<PL>(la, &tmS, c0, pr.a * PL::H, 4, &bar);
-        tma_panel<PL>(lb, &tmS, c0, pr.b * PL::H, 4, &bar);
+    if (threadIdx.x == 0) {   // each tile's panel is one contiguous run: one bulk copy each
+        constexpr uint32_t PB = (uint32_t)PL::COL_PANEL_P;
+        mbar_arrive_expect_tx(&bar, 2 * PB + ColTw<PL>::BYTES);
+        bulk_g2s(la, spec + ((size_t)pr.a * PL::WP + c0) * PL::HP, PB, &bar);
+        bulk_g2s(lb, spec + ((size_t)pr.b * PL::WP + c0) * PL::HP, PB, &bar);
         ColTw<PL>::issue(tws, tw2, &bar);
     }
     ColTw<PL>::fallback(tws, tw2);

@@ -53,14 +53,14 @@ using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 32, 8, 32, 0, 0>;
 constexpr int PAIR_BAND = 4;
 
 struct PlanOps {
-    int W, H, M, WC, WP, col_p;
+    int W, H, M, WC, WP, HP, col_p;
     int row_r0, row_r1, col_r0, col_r1;   // stage radices (r1 = 1: single stage)
     cudaError_t (*setup)(int* grid_k1, int* grid_k4);
     void (*k1)(const uint16_t*, float2*, int, int, const int32_t*, const float2*, const float2*,
                int, cudaStream_t);
     void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const int32_t*, const float2*,
                bool, int, cudaStream_t);
-    void (*k3)(const CUtensorMap&, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
+    void (*k3)(const uint32_t*, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
                cudaStream_t);
     void (*k4s)(const float2*, float*, float, const float2*, const float2*, int, cudaStream_t);
@@ -109,7 +109,7 @@ cudaError_t plan_setup(int* grid_k1, int* grid_k4) {
     CKE(cudaGetDevice(&dev));
     CKE(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     CKE(max_smem(k5_ccf_moments<PL::W, PL::H>, k5_smem_bytes(PL::W)));
-    CKE(max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM));
+    CKE(max_smem(k2t_fwd_cols<PL, true>, PL::COL_SMEM_K2));
     CKE(max_smem(k2t_fwd_cols<PL, false>, PL::COL_SMEM));
     CKE(max_smem(k3t_pair_cols<PL>, PL::COL_SMEM));
     if constexpr (RowWarp<PL>::OK) {
@@ -151,16 +151,16 @@ void launch_k2(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt
                const int32_t* fslot, const float2* tw2, bool phase_out, int ahead, cudaStream_t s) {
     const dim3 grid(PL::WP / PL::COL_P, nt);
     if (phase_out)
-        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, fslot, tw2,
-                                                                     ahead);
+        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM_K2, s>>>(tmG, G, spec, t0, fslot,
+                                                                        tw2, ahead);
     else
         k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, fslot, tw2,
                                                                       0);
 }
 template <class PL>
-void launch_k3(const CUtensorMap& tmS, float2* Q, const PairIdx* pairs, int p0, int np,
+void launch_k3(const uint32_t* spec, float2* Q, const PairIdx* pairs, int p0, int np,
                const float2* tw2, cudaStream_t s) {
-    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(tmS, Q, pairs,
+    k3t_pair_cols<PL><<<dim3(PL::WP / PL::COL_P, np), PL::COL_T, PL::COL_SMEM, s>>>(spec, Q, pairs,
                                                                                    p0, tw2);
 }
 template <class PL>
@@ -239,7 +239,8 @@ void launch_d4(const double2* Q, double* pv, uint32_t* pi, int p0, int np, const
 template <class PL>
 PlanOps make_ops() {
     PlanOps o;
-    o.W = PL::W; o.H = PL::H; o.M = PL::M; o.WC = PL::WC; o.WP = PL::WP; o.col_p = PL::COL_P;
+    o.W = PL::W; o.H = PL::H; o.M = PL::M; o.WC = PL::WC; o.WP = PL::WP; o.HP = PL::HP;
+    o.col_p = PL::COL_P;
     o.row_r0 = PL::RI::R0; o.row_r1 = PL::RI::R1; o.col_r0 = PL::CI::R0; o.col_r1 = PL::CI::R1;
     o.setup = plan_setup<PL>;
     o.k1 = launch_k1<PL>; o.k2 = launch_k2<PL>; o.k3 = launch_k3<PL>; o.k4 = launch_k4<PL>;
@@ -320,6 +321,7 @@ struct Layout {
     int pool;            // bounded mode (row f1)
     int world, rank;
     bool exchange;       // in-library NCCL halo exchange
+    size_t spec_tile_bytes;   // one slot's spectrum
     size_t off_raw, off_spec, off_g, off_q, off_pairs, off_keys, off_mom, off_res, off_tw,
         off_part, off_fslot, total;
 };
@@ -378,13 +380,13 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
                          : (L->prec ? 8 : (L->pool ? std::max(1, std::min(64, L->nslots / 4)) : 64));
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
-    // spectrum by slot: u32 Q15 unit phasor (fp32) or double2 unit phasor (fp64)
-    const size_t spec_el = L->prec ? sizeof(double2) : sizeof(uint32_t);
+    // spectrum by slot: u32 Q15 unit phasor [WP][HP] (fp32) or double2 unit phasor [H][WP] (fp64)
+    L->spec_tile_bytes = L->prec ? H * WP * sizeof(double2) : (size_t)ops->HP * WP * sizeof(uint32_t);
     const size_t cplx = L->prec ? sizeof(double2) : sizeof(float2);
     const size_t np1 = (size_t)(np > 0 ? np : 1);
     size_t o = 0;
     L->off_raw = o;   o += align256((size_t)L->nslots * H * W * sizeof(uint16_t));
-    L->off_spec = o;  o += align256((size_t)L->nslots * H * WP * spec_el);
+    L->off_spec = o;  o += align256((size_t)L->nslots * L->spec_tile_bytes);
     L->off_g = o;     o += align256((size_t)L->chunk_tiles * H * WP * cplx);
     L->off_q = o;     o += align256((size_t)L->chunk_pairs * H * WP * cplx);
     L->off_pairs = o; o += align256(np1 * sizeof(PairIdx));
@@ -465,7 +467,7 @@ struct stitch_ctx {
     double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
     double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
     uint32_t* part_i = nullptr;
-    CUtensorMap tmG, tmS;             // TMA descriptors of G (complex) and spec (Q15 phasors)
+    CUtensorMap tmG;                  // TMA descriptor of G (complex), K2's column panels
     int grid_k1 = 0, grid_k4 = 0;     // persistent grids of the warp row kernels (0: CTA kernels)
     int col_ahead = 0;                // K2 L2 prefetch distance in CTAs (one wave)
     PairIdx* pairs;
@@ -757,6 +759,14 @@ static stitch_status copy_chunk_in(stitch_ctx* ctx, const FwdChunk& fc, const ui
 
 static void launch_fwd(stitch_ctx* ctx, int t0, int nt, cudaStream_t s, int si) {
     const PlanOps* o = ctx->ops;
+    if (ctx->prec) {   // fp64 path (f2): D1, D2 (resident tiles: slot = local tile)
+        tl_wrap(ctx, s, si, 0, [&] { o->d1(ctx->raw, ctx->Gd, t0, nt, ctx->twMd, ctx->twWd, s); });
+        mark(ctx, 0);
+        tl_wrap(ctx, s, si, 1, [&] { o->d2(ctx->Gd, ctx->Ud, t0, nt, ctx->twHd, true, s); });
+        mark(ctx, 1);
+        ctx->launches += 2;
+        return;
+    }
     tl_wrap(ctx, s, si, 0, [&] {
         o->k1(ctx->raw, ctx->G, t0, nt, ctx->fslot, ctx->twM, ctx->twW, ctx->grid_k1, s);
     });
@@ -772,7 +782,7 @@ static void launch_fwd(stitch_ctx* ctx, int t0, int nt, cudaStream_t s, int si) 
 // row from k-1), one NCCL group on stream s.
 static stitch_status exchange(stitch_ctx* ctx, cudaStream_t s) {
     const NcclApi& api = nccl();
-    const size_t per = (size_t)ctx->H * ctx->ops->WP * sizeof(uint32_t);
+    const size_t per = ctx->L.spec_tile_bytes;
     ncclResult_t r;
     if ((r = api.group_start()) != ncclSuccess) return nccl_fail(ctx, r, "ncclGroupStart");
     if (ctx->send_cnt > 0 &&
@@ -823,11 +833,45 @@ static stitch_status enqueue_ops(stitch_ctx* ctx, const std::vector<Op>& ops, co
         for (cudaStream_t st : {sf, sp, sk, sh, sc})
             if (st) CK(cudaStreamWaitEvent(st, ctx->ev_fork, 0), "fork wait");
     }
+    if (src && ctx->L.exchange && ctx->recv_cnt > 0) {
+        // the halo's spectra arrive by NCCL, its pixels (K5 reads tile A) from the host: copied
+        // ahead of the first forward chunk's tiles on the same stream, so every pair chunk
+        // (ordered after a forward chunk) finds them
+        FwdChunk halo{ctx->recv_lt, ctx->recv_cnt};
+        stitch_status st = copy_chunk_in(ctx, halo, src, sh);
+        if (st != STITCH_OK) return st;
+    }
     int waited = -1, last_fwd = -1;
     bool halo_waited = false, any_k4 = false;
+    // K5 runs over groups of consecutive pair chunks holding >= K5_MIN_PAIRS pairs (a K5
+    // launch of a few pairs cannot fill the GPU: the fp64 path's 8-pair chunks made it 5x
+    // slower); every chunk of a group gets its ev_k5 once the group's K5 is enqueued.
+    constexpr int K5_MIN_PAIRS = 128;
+    int g_first = -1, g_last = -1;   // pending group: pair chunks [g_first, g_last]
+    auto flush_k5 = [&]() -> stitch_status {
+        if (g_first < 0) return STITCH_OK;
+        const PairChunk &a = ctx->pch[g_first], &b = ctx->pch[g_last];
+        const int64_t q0 = a.p0;
+        const int nq = (int)(b.p0 + b.np - a.p0);
+        if (!ser) CK(cudaStreamWaitEvent(sk, ctx->ev_k4[g_last], 0), "wait k4");
+        tl_wrap(ctx, sk, 2, 4, [&] {
+            o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)q0, nq, sk);
+        });
+        mark(ctx, 4);
+        ctx->launches += 1;
+        if (!ser)
+            for (int c = g_first; c <= g_last; ++c)
+                CK(cudaEventRecord(ctx->ev_k5[c], sk), "event");
+        g_first = g_last = -1;
+        return STITCH_OK;
+    };
     for (const Op& op : ops) {
         if (op.kind == Op::FWD) {
             const FwdChunk& fc = ctx->fwd[op.idx];
+            if (fc.wait_pair >= 0 && g_first >= 0 && fc.wait_pair >= g_first) {
+                stitch_status st = flush_k5();   // the slots it waits for are freed by this K5
+                if (st != STITCH_OK) return st;
+            }
             if (!ser) {   // bounded mode: the slots this chunk takes must be free
                 if (fc.wait_pair >= 0) {
                     CK(cudaStreamWaitEvent(sf, ctx->ev_k5[fc.wait_pair], 0), "wait slot");
@@ -866,32 +910,57 @@ static stitch_status enqueue_ops(stitch_ctx* ctx, const std::vector<Op>& ops, co
             }
             if (ctx->timing && !any_k4 && ser) CK(cudaEventRecord(ctx->ev[1], m), "event");
             any_k4 = true;
-            tl_wrap(ctx, sp, 1, 2, [&] {
-                o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)pc.p0, pc.np, ctx->twH, sp);
-            });
-            mark(ctx, 2);
-            tl_wrap(ctx, sp, 1, 3, [&] {
-                o->k4(ctx->Q, ctx->keys, (int)pc.p0, pc.np, ctx->twM, ctx->twW, ctx->grid_k4, sp);
-            });
-            mark(ctx, 3);
-            if (!ser) {
-                CK(cudaEventRecord(ctx->ev_k4[op.idx], sp), "event");
-                CK(cudaStreamWaitEvent(sk, ctx->ev_k4[op.idx], 0), "wait k4");
+            if (ctx->prec) {   // fp64 path (f2): D3, D4 (per-block argmax partials), D5 -> keys
+                tl_wrap(ctx, sp, 1, 2, [&] {
+                    o->d3(ctx->Ud, ctx->Qd, ctx->pairs, (int)pc.p0, pc.np, ctx->twHd, sp);
+                });
+                mark(ctx, 2);
+                tl_wrap(ctx, sp, 1, 3, [&] {
+                    o->d4(ctx->Qd, ctx->part_v, ctx->part_i, (int)pc.p0, pc.np, ctx->twMd,
+                          ctx->twWd, sp);
+                    const size_t pb0 = (size_t)pc.p0 * o->nblk64;
+                    d5_argmax_keys<<<(unsigned)((pc.np + 7) / 8), 256, 0, sp>>>(
+                        ctx->part_v + pb0, ctx->part_i + pb0, ctx->keys + pc.p0, o->nblk64, pc.np);
+                });
+                mark(ctx, 3);
+                ctx->launches += 1;
+            } else {
+                tl_wrap(ctx, sp, 1, 2, [&] {
+                    o->k3(ctx->spec, ctx->Q, ctx->pairs, (int)pc.p0, pc.np, ctx->twH, sp);
+                });
+                mark(ctx, 2);
+                tl_wrap(ctx, sp, 1, 3, [&] {
+                    o->k4(ctx->Q, ctx->keys, (int)pc.p0, pc.np, ctx->twM, ctx->twW, ctx->grid_k4,
+                          sp);
+                });
+                mark(ctx, 3);
             }
-            tl_wrap(ctx, sk, 2, 4, [&] {
-                o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)pc.p0, pc.np, sk);
-            });
-            mark(ctx, 4);
-            if (!ser) CK(cudaEventRecord(ctx->ev_k5[op.idx], sk), "event");
-            ctx->launches += 3;
+            if (!ser) CK(cudaEventRecord(ctx->ev_k4[op.idx], sp), "event");
+            ctx->launches += 2;
+            if (g_first < 0 || g_last != op.idx - 1 ||
+                ctx->pch[op.idx].p0 + pc.np - ctx->pch[g_first].p0 > 65535) {
+                stitch_status st = flush_k5();
+                if (st != STITCH_OK) return st;
+                g_first = op.idx;
+            }
+            g_last = op.idx;
+            if (pc.p0 + pc.np - ctx->pch[g_first].p0 >= K5_MIN_PAIRS) {
+                stitch_status st = flush_k5();
+                if (st != STITCH_OK) return st;
+            }
         }
+    }
+    {
+        stitch_status st = flush_k5();
+        if (st != STITCH_OK) return st;
     }
     if (ctx->timing && ser) CK(cudaEventRecord(ctx->ev[2], m), "event");
     if (np > 0) {
         tl_wrap(ctx, sk, 2, 5, [&] {
+            // the key's value is max |c| (fp64 path) or max |c| x 32767^2 (Q15 phasor NCPS)
             k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
                 ctx->keys + pa, ctx->mom + pa * 20, ctx->res + pa, ctx->H, ctx->W, (int)np,
-                (double)ctx->W * ctx->H * NCPS_Q15_SCALE);
+                (double)ctx->W * ctx->H * (ctx->prec ? 1.0 : NCPS_Q15_SCALE));
         });
         mark(ctx, 5);
         ctx->launches += 1;
@@ -906,50 +975,6 @@ static stitch_status enqueue_ops(stitch_ctx* ctx, const std::vector<Op>& ops, co
             ++j;
         }
     }
-    return STITCH_OK;
-}
-
-// fp64 path (f2): serial on the context stream -- D1 + D2 per forward chunk, D3 + D4 per pair
-// chunk (per-block argmax partials), D5 reducing them into the K5/K6 key, K5 per chunk, K6.
-static stitch_status enqueue_fp64(stitch_ctx* ctx, bool forward, bool pairs) {
-    const PlanOps* o = ctx->ops;
-    cudaStream_t s = ctx->stream;
-    if (forward) {
-        for (const FwdChunk& fc : ctx->fwd) {
-            o->d1(ctx->raw, ctx->Gd, fc.t0, fc.nt, ctx->twMd, ctx->twWd, s);
-            CK(mark(ctx, 0), "event");
-            o->d2(ctx->Gd, ctx->Ud, fc.t0, fc.nt, ctx->twHd, true, s);
-            CK(mark(ctx, 1), "event");
-            ctx->launches += 2;
-        }
-    }
-    if (ctx->timing) CK(cudaEventRecord(ctx->ev[1], s), "event");
-    const int64_t np = ctx->L.npairs;
-    if (pairs && np > 0) {
-        CK(cudaMemsetAsync(ctx->mom, 0, (size_t)np * 20 * sizeof(unsigned long long), s), "memset");
-        for (const PairChunk& pc : ctx->pch) {
-            o->d3(ctx->Ud, ctx->Qd, ctx->pairs, (int)pc.p0, pc.np, ctx->twHd, s);
-            CK(mark(ctx, 2), "event");
-            o->d4(ctx->Qd, ctx->part_v, ctx->part_i, (int)pc.p0, pc.np, ctx->twMd, ctx->twWd, s);
-            CK(mark(ctx, 3), "event");
-            ctx->launches += 2;
-        }
-        d5_argmax_keys<<<(unsigned)((np + 7) / 8), 256, 0, s>>>(ctx->part_v, ctx->part_i,
-                                                               ctx->keys, o->nblk64, (int)np);
-        CK(mark(ctx, 3), "event");
-        ctx->launches += 1;
-        if (ctx->timing) CK(cudaEventRecord(ctx->ev[2], s), "event");
-        for (const PairChunk& pc : ctx->pch) {
-            o->k5(ctx->raw, ctx->pairs, ctx->keys, ctx->mom, (int)pc.p0, pc.np, s);
-            CK(mark(ctx, 4), "event");
-            ctx->launches += 1;
-        }
-        k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, s>>>(
-            ctx->keys, ctx->mom, ctx->res, ctx->H, ctx->W, (int)np, (double)ctx->W * ctx->H);
-        CK(mark(ctx, 5), "event");
-        ctx->launches += 1;
-    }
-    CK(cudaGetLastError(), "fp64 launch");
     return STITCH_OK;
 }
 
@@ -1217,7 +1242,7 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, cfg->device);
     ctx->col_ahead = 2 * sms;   // K2's L2 prefetch one wave (2 CTAs per SM) ahead
     ctx->use_graph = !(cfg->flags & STITCH_FLAG_NO_GRAPH);
-    ctx->concurrent = !(cfg->flags & STITCH_FLAG_SERIAL) && !ctx->prec;
+    ctx->concurrent = !(cfg->flags & STITCH_FLAG_SERIAL);
 
     if (ctx->concurrent) {
         for (cudaStream_t* st : {&ctx->s_fwd, &ctx->s_pair, &ctx->s_ccf, &ctx->s_h2d})
@@ -1293,18 +1318,11 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
         const cuuint32_t boxh = (cuuint32_t)(ops->H / ((ops->H + 255) / 256));
         const cuuint32_t estr[2] = {1, 1};
-        // G: complex chunk [chunk_tiles*H][WP] as floats; spec: u32 Q15 phasors [nslots*H][WP]
+        // G: complex chunk [chunk_tiles*H][WP] as floats, landed by K2 in [H][COL_P] panels
         const cuuint64_t gd[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
         const cuuint64_t gs[1] = {(cuuint64_t)ops->WP * 8};
         const cuuint32_t gb[2] = {(cuuint32_t)2 * ops->col_p, boxh};
-        const cuuint64_t sd[2] = {(cuuint64_t)ops->WP, (cuuint64_t)L.nslots * ops->H};
-        const cuuint64_t ss[1] = {(cuuint64_t)ops->WP * 4};
-        const cuuint32_t sb[2] = {(cuuint32_t)ops->col_p, boxh};
         if (encode(&ctx->tmG, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, gd, gs, gb, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) !=
-                CUDA_SUCCESS ||
-            encode(&ctx->tmS, CU_TENSOR_MAP_DATA_TYPE_UINT32, 2, ctx->spec, sd, ss, sb, estr,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) !=
                 CUDA_SUCCESS)
@@ -1450,13 +1468,7 @@ stitch_status stitch_forward_range_async(stitch_ctx* ctx, int32_t first_tile, in
     st = run_graphed(ctx, key, [&]() -> stitch_status {
         for (int t0 = lt0; t0 < lt0 + count; t0 += ct) {
             const int nt = std::min(ct, lt0 + count - t0);
-            if (ctx->prec) {
-                ctx->ops->d1(ctx->raw, ctx->Gd, t0, nt, ctx->twMd, ctx->twWd, ctx->stream);
-                ctx->ops->d2(ctx->Gd, ctx->Ud, t0, nt, ctx->twHd, true, ctx->stream);
-                ctx->launches += 2;
-            } else {
-                launch_fwd(ctx, t0, nt, ctx->stream, 0);
-            }
+            launch_fwd(ctx, t0, nt, ctx->stream, 0);
         }
         CK(cudaGetLastError(), "forward launch");
         return STITCH_OK;
@@ -1470,15 +1482,7 @@ stitch_status stitch_pairs_part_async(stitch_ctx* ctx, int32_t part) {
     if (part < 0 || part > 2) return fail(ctx, STITCH_ERR_INVALID_ARG, "part must be 0, 1 or 2");
     if (ctx->L.pool) return fail(ctx, STITCH_ERR_STATE, "split step: not in the bounded mode");
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "pairs before load");
-    if (ctx->prec && part != 0) return fail(ctx, STITCH_ERR_UNSUPPORTED, "fp64: part 0 only");
     GUARD(ctx);
-    if (ctx->prec) {
-        stitch_status st = step_begin(ctx);
-        if (st != STITCH_OK) return st;
-        st = enqueue_fp64(ctx, false, true);
-        if (st == STITCH_OK) ctx->computed = true;
-        return st == STITCH_OK ? step_end(ctx) : st;
-    }
     const int c0 = part == 2 ? ctx->c_boundary : 0;
     const int c1 = part == 1 ? ctx->c_boundary : (int)ctx->pch.size();
     const int64_t pa = part == 2 ? ctx->n_interior : 0;
@@ -1503,7 +1507,6 @@ stitch_status stitch_compute_translations_async(stitch_ctx* ctx) {
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
     st = run_graphed(ctx, 1ull << 60, [&]() {
-        if (ctx->prec) return enqueue_fp64(ctx, true, true);
         return enqueue_ops(ctx, ctx->ops_step, nullptr, true, 0, ctx->L.npairs);
     });
     if (st == STITCH_OK) ctx->computed = true;
@@ -1522,11 +1525,6 @@ stitch_status stitch_compute_translations_from_host_async(stitch_ctx* ctx, const
     const bool pinned = cudaPointerGetAttributes(&pa, tiles) == cudaSuccess &&
                         pa.type == cudaMemoryTypeHost;
     cudaGetLastError();   // clear a pointer-query error on pageable memory
-    if (ctx->prec) {      // fp64: load, then compute
-        stitch_status st = load_common(ctx, tiles, first_tile, count, false);
-        if (st != STITCH_OK) return st;
-        return stitch_compute_translations_async(ctx);
-    }
     stitch_status st = step_begin(ctx);
     if (st != STITCH_OK) return st;
     auto body = [&]() { return enqueue_ops(ctx, ctx->ops_step, src, true, 0, ctx->L.npairs); };
@@ -1545,8 +1543,7 @@ stitch_status stitch_spectra_range(stitch_ctx* ctx, int32_t first_tile, int32_t 
     if (ctx->L.pool) return fail(ctx, STITCH_ERR_STATE, "bounded mode: spectra are not resident");
     if (count < 0 || first_tile < ctx->L.h_begin || first_tile + (int64_t)count > ctx->L.t_end)
         return fail(ctx, STITCH_ERR_INVALID_ARG, "tile range not resident");
-    const size_t per =
-        (size_t)ctx->H * ctx->ops->WP * (ctx->prec ? sizeof(double2) : sizeof(uint32_t));
+    const size_t per = ctx->L.spec_tile_bytes;
     *dev_ptr = reinterpret_cast<char*>(ctx->prec ? (void*)ctx->Ud : (void*)ctx->spec) +
                (size_t)(first_tile - ctx->L.h_begin) * per;
     *bytes = (size_t)count * per;
@@ -1648,7 +1645,7 @@ stitch_status stitch_debug_surface(stitch_ctx* ctx, int32_t tile, int32_t kind, 
     const PlanOps* o = ctx->ops;
     float* surf = reinterpret_cast<float*>(ctx->G);   // H*W floats fit one chunk slot of G
     const float scale = (float)(1.0 / ((double)ctx->W * ctx->H * NCPS_Q15_SCALE));
-    o->k3(ctx->tmS, ctx->Q, ctx->pairs, (int)p, 1, ctx->twH, ctx->stream);
+    o->k3(ctx->spec, ctx->Q, ctx->pairs, (int)p, 1, ctx->twH, ctx->stream);
     o->k4s(ctx->Q, surf, scale, ctx->twM, ctx->twW, ctx->grid_k4, ctx->stream);
     CK(cudaGetLastError(), "surface launch");
     CK(cudaMemcpyAsync(host_out, surf, (size_t)ctx->H * ctx->W * sizeof(float),

@@ -61,8 +61,8 @@ class GridStream:
                 self._collect(sl, sink)
             src = fill(idx, sl["host"].numpy())
             sl["src"] = src                      # keep the source alive until collected
-            sl["grid"].load_tiles(sl["host"] if src is None else src, 0)
-            sl["grid"].compute_translations_async()
+            # steps 1-7 on the slot's stream, the H2D pipelined per forward chunk
+            sl["grid"].compute_from_host_async(sl["host"] if src is None else src, 0)
             sl["pending"] = idx
             count += 1
         for sl in self.slots:

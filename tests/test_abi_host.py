@@ -80,7 +80,7 @@ def test_workspace_size_matches_layout(lib):
     ws = pkg.workspace_size(cfg)
     H, W, WP = 1040, 1392, 704
     raw = 2478 * H * W * 2
-    spec = 2478 * H * WP * 4          # resident Q15 unit phasors (u32)
+    spec = 2478 * WP * 1044 * 4       # resident Q15 unit phasors (u32), column pitch 1044
     chunks = 2 * 8 * H * WP * 8       # G (forward chunk) + Q (pair chunk), complex (8 each)
     assert raw + spec + chunks < ws < raw + spec + chunks + 5 * 2**20
 
@@ -282,6 +282,6 @@ def test_bounded_pool_validation_and_size(lib):
     # 42x59 @ 1392x1040: 128 slots instead of 2478 tiles
     big = pkg.workspace_size(pkg.make_config(42, 59, 1040, 1392))
     small = pkg.workspace_size(pkg.make_config(42, 59, 1040, 1392, pool_tiles=128))
-    per_tile = 1040 * 1392 * 2 + 1040 * 704 * 4
+    per_tile = 1040 * 1392 * 2 + 1044 * 704 * 4
     assert big - small >= (2478 - 128) * per_tile
     assert small < 2.0e9
