@@ -4,7 +4,8 @@
 //   raw   uint16 [tiles][H][W]           W contiguous (the caller's tile layout)
 //   raw   uint16 [slots][H][W]           tile pixels by slot (slot = tile in the resident mode;
 //                                        a recycled pool slot in the bounded mode, row f1)
-//   G     float2 [chunk][H][WP]          row-transformed tiles of a forward chunk
+//   G     float2 [chunk][WP/COL_P][H][COL_P]  row-transformed tiles of a forward chunk, in
+//                                        column panels (each K2 panel one contiguous run)
 //   spec  u32    [slots][WP][HP]         half spectrum kx in [0, W/2] (WP = pad16(W/2+1)),
 //                                        COLUMN-major (ky contiguous, pitch HP = H rounded up to
 //                                        4 mod 8 words), stored as its Q15 unit phasor F/|F|
@@ -90,9 +91,6 @@ struct Plan {
     // K2 stages its phasor panel [COL_P][HP] behind that and stores it with one bulk copy
     static constexpr size_t COL_STG_OFF = (COL_SMEM + 127) / 128 * 128;
     static constexpr size_t COL_SMEM_K2 = COL_STG_OFF + COL_PANEL_P;
-    static constexpr int BOXH = H / ((H + 255) / 256);   // TMA box rows (<= 256)
-    static_assert(H % BOXH == 0, "H must split into equal TMA boxes of <= 256 rows");
-    static_assert((BOXH * COL_P * 4) % 128 == 0 || H == BOXH, "TMA boxes must land 128-B aligned");
     // CTAs per SM the column kernels are register-budgeted for (shared memory allows this many)
     static constexpr int COL_MINB_RAW = (int)((220 * 1024) / (COL_SMEM + 1024));
     static constexpr int COL_MINB = COL_MINB_RAW > 4 ? 4 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
@@ -125,6 +123,18 @@ struct U16RowSrc {  // z[n] = x[2n] + i x[2n+1], straight from the uint16 row
     }
 };
 
+// G's panel-blocked layout: bin q of row y of a tile sits in column panel q / COL_P, whose
+// H rows of COL_P bins are contiguous (K2 lands a panel with one bulk copy); a warp's 32
+// consecutive bins of a row are 4 whole 64-byte runs (K1's stores stay sector-complete).
+template <class PL>
+struct GRow {
+    float2* t;   // the tile's G block
+    int y;
+    __device__ __forceinline__ float2& operator[](int q) const {
+        return t[((size_t)(q / PL::COL_P) * PL::H + y) * PL::COL_P + q % PL::COL_P];
+    }
+};
+
 // Real-to-complex post-processing of one line (Z = the length-M complex FFT of the packed
 // row, in the exchange buffer, natural order; Z[M] == Z[0]).  For q in [0, M/2]:
 //   E = (Z[q] + conj Z[M-q]) / 2,  O = (Z[q] - conj Z[M-q]) / (2i)
@@ -132,7 +142,7 @@ struct U16RowSrc {  // z[n] = x[2n] + i x[2n+1], straight from the uint16 row
 // (E and O of M-q are conj(E), conj(O), and w_W^{M-q} = -conj(w_W^q)), so one iteration
 // writes the mirror pair; bins [M+1, WP) of the padded row are zeroed.
 template <class PL, class Xc, class TwLoad>
-__device__ __forceinline__ void r2c_post_line(const Xc& xc, int line, float2* __restrict__ out,
+__device__ __forceinline__ void r2c_post_line(const Xc& xc, int line, const GRow<PL>& out,
                                               const TwLoad& twq) {
     constexpr int M = PL::M;
     for (int q = threadIdx.x; q <= M / 2; q += PL::ROW_T) {
@@ -164,7 +174,7 @@ __global__ void __launch_bounds__(PL::ROW_T) k1_fwd_rows(const uint16_t* __restr
     __syncthreads();
 #pragma unroll 1
     for (int line = 0; line < L; ++line)
-        r2c_post_line<PL>(xc, line, G + ((size_t)blockIdx.y * PL::H + y0 + line) * PL::WP,
+        r2c_post_line<PL>(xc, line, GRow<PL>{G + (size_t)blockIdx.y * PL::H * PL::WP, y0 + line},
                           [&](int q) { return __ldg(&twW[q]); });
 }
 
@@ -221,22 +231,6 @@ struct PhaseDst {  // K2 output: Q15 unit phasors of a panel [COL_P][HP] (staged
     }
 };
 
-template <class PL>
-__device__ __forceinline__ void tma_panel(void* land, const CUtensorMap* map, int x, int row0,
-                                          int elem_bytes, uint64_t* bar) {
-    // one panel = H rows of COL_P elements, in boxes of BOXH rows
-    char* d = reinterpret_cast<char*>(land);
-#pragma unroll 1
-    for (int y = 0; y < PL::H; y += PL::BOXH)
-        tma_load_2d(d + (size_t)y * PL::COL_P * elem_bytes, map, x, row0 + y, bar);
-}
-
-template <class PL>
-__device__ __forceinline__ void l2_prefetch_panel(const CUtensorMap* map, int x, int row0) {
-#pragma unroll 1
-    for (int y = 0; y < PL::H; y += PL::BOXH) tma_prefetch_l2_2d(map, x, row0 + y);
-}
-
 // L2 prefetch for the CTA `ahead` launch slots later (about one wave of resident CTAs): its
 // panel is pulled from DRAM into L2 while this CTA computes, so its own TMA loads hit L2
 // (the column kernels spend ~30 % of their stall samples waiting for their panel, ncu r01c).
@@ -266,20 +260,20 @@ struct ColTw {
     }
 };
 
-// K2: column FFT of a chunk of row-transformed tiles (G, complex), panel of COL_P columns
-// landed by TMA; writes the phase spectrum of each tile's slot (or, for the test hook, the
-// complex spectrum back into G).  `ahead`: L2 prefetch of the panel of the CTA that many
-// launch slots later (one wave of resident CTAs: K2 7.25 -> 6.86 ms).
+// K2: column FFT of a chunk of row-transformed tiles (G, complex), one column panel per CTA
+// landed by one bulk copy (G is panel-blocked); writes the phase spectrum of each tile's slot
+// (or, for the test hook, the complex spectrum row-major [H][WP] into `out`).  `ahead`: L2
+// prefetch of the panel of the CTA that many launch slots later (one wave of resident CTAs:
+// K2 7.25 -> 6.86 ms).
 template <class PL, bool PHASE_OUT>
 __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
-    k2t_fwd_cols(const __grid_constant__ CUtensorMap tmG, float2* __restrict__ G,
+    k2t_fwd_cols(const float2* __restrict__ G, float2* __restrict__ out,
                  uint32_t* __restrict__ spec, int tile0, const int32_t* __restrict__ fslot,
                  const float2* __restrict__ tw2, int ahead) {
     extern __shared__ __align__(128) unsigned char csmem[];
     __shared__ uint64_t bar;
     const int tl = blockIdx.y, c0 = blockIdx.x * PL::COL_P;
     if (threadIdx.x == 0) {
-        prefetch_tensormap(&tmG);
         mbar_init(&bar, 1);
         fence_mbar_init();
     }
@@ -287,11 +281,13 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
     float2* tws = reinterpret_cast<float2*>(csmem + PL::COL_BUF);
     if (threadIdx.x == 0) {
         mbar_arrive_expect_tx(&bar, (uint32_t)PL::COL_LAND_C + ColTw<PL>::BYTES);
-        tma_panel<PL>(csmem, &tmG, 2 * c0, tl * PL::H, 8, &bar);
+        bulk_g2s(csmem, G + ((size_t)tl * PL::WP + c0) * PL::H, (uint32_t)PL::COL_LAND_C, &bar);
         ColTw<PL>::issue(tws, tw2, &bar);
         int pn, it;
         ahead_cta(ahead, pn, it);
-        if (it >= 0) l2_prefetch_panel<PL>(&tmG, 2 * pn * PL::COL_P, it * PL::H);
+        if (it >= 0)
+            bulk_prefetch_l2(G + ((size_t)it * PL::WP + pn * PL::COL_P) * PL::H,
+                             (uint32_t)PL::COL_LAND_C);
     }
     ColTw<PL>::fallback(tws, tw2);
     mbar_wait(&bar, 0);
@@ -314,7 +310,7 @@ __global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
             bulk_wait_read_all();
         }
     } else {
-        PanelIO<PL> dst{G + (size_t)tl * PL::H * PL::WP + c0};
+        PanelIO<PL> dst{out + (size_t)tl * PL::H * PL::WP + c0};
         Run::template run<true>(src, xc, dst, tws);
     }
 }

@@ -58,8 +58,8 @@ struct PlanOps {
     cudaError_t (*setup)(int* grid_k1, int* grid_k4);
     void (*k1)(const uint16_t*, float2*, int, int, const int32_t*, const float2*, const float2*,
                int, cudaStream_t);
-    void (*k2)(const CUtensorMap&, float2*, uint32_t*, int, int, const int32_t*, const float2*,
-               bool, int, cudaStream_t);
+    void (*k2)(const float2*, float2*, uint32_t*, int, int, const int32_t*, const float2*, bool,
+               int, cudaStream_t);
     void (*k3)(const uint32_t*, float2*, const PairIdx*, int, int, const float2*, cudaStream_t);
     void (*k4)(const float2*, unsigned long long*, int, int, const float2*, const float2*, int,
                cudaStream_t);
@@ -147,14 +147,14 @@ void launch_k1(const uint16_t* raw, float2* G, int t0, int nt, const int32_t* fs
     }
 }
 template <class PL>
-void launch_k2(const CUtensorMap& tmG, float2* G, uint32_t* spec, int t0, int nt,
-               const int32_t* fslot, const float2* tw2, bool phase_out, int ahead, cudaStream_t s) {
+void launch_k2(const float2* G, float2* out, uint32_t* spec, int t0, int nt, const int32_t* fslot,
+               const float2* tw2, bool phase_out, int ahead, cudaStream_t s) {
     const dim3 grid(PL::WP / PL::COL_P, nt);
     if (phase_out)
-        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM_K2, s>>>(tmG, G, spec, t0, fslot,
+        k2t_fwd_cols<PL, true><<<grid, PL::COL_T, PL::COL_SMEM_K2, s>>>(G, out, spec, t0, fslot,
                                                                         tw2, ahead);
     else
-        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(tmG, G, spec, t0, fslot, tw2,
+        k2t_fwd_cols<PL, false><<<grid, PL::COL_T, PL::COL_SMEM, s>>>(G, out, spec, t0, fslot, tw2,
                                                                       0);
 }
 template <class PL>
@@ -467,7 +467,6 @@ struct stitch_ctx {
     double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
     double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
     uint32_t* part_i = nullptr;
-    CUtensorMap tmG;                  // TMA descriptor of G (complex), K2's column panels
     int grid_k1 = 0, grid_k4 = 0;     // persistent grids of the warp row kernels (0: CTA kernels)
     int col_ahead = 0;                // K2 L2 prefetch distance in CTAs (one wave)
     PairIdx* pairs;
@@ -772,7 +771,7 @@ static void launch_fwd(stitch_ctx* ctx, int t0, int nt, cudaStream_t s, int si) 
     });
     mark(ctx, 0);
     tl_wrap(ctx, s, si, 1, [&] {
-        o->k2(ctx->tmG, ctx->G, ctx->spec, t0, nt, ctx->fslot, ctx->twH, true, ctx->col_ahead, s);
+        o->k2(ctx->G, nullptr, ctx->spec, t0, nt, ctx->fslot, ctx->twH, true, ctx->col_ahead, s);
     });
     mark(ctx, 1);
     ctx->launches += 2;
@@ -1307,28 +1306,6 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
         ctx->part_i = (uint32_t*)(b + L.off_part + np1 * sizeof(double));
     }
 
-    // TMA descriptors (driver entry point through the runtime; no libcuda link needed);
-    // the fp64 path uses plain loads
-    if (!ctx->prec) {
-        void* fn = nullptr;
-        cudaDriverEntryPointQueryResult q;
-        if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &fn, cudaEnableDefault, &q) !=
-                cudaSuccess || !fn)
-            return bail(STITCH_ERR_CUDA);
-        auto encode = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(fn);
-        const cuuint32_t boxh = (cuuint32_t)(ops->H / ((ops->H + 255) / 256));
-        const cuuint32_t estr[2] = {1, 1};
-        // G: complex chunk [chunk_tiles*H][WP] as floats, landed by K2 in [H][COL_P] panels
-        const cuuint64_t gd[2] = {(cuuint64_t)2 * ops->WP, (cuuint64_t)L.chunk_tiles * ops->H};
-        const cuuint64_t gs[1] = {(cuuint64_t)ops->WP * 8};
-        const cuuint32_t gb[2] = {(cuuint32_t)2 * ops->col_p, boxh};
-        if (encode(&ctx->tmG, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, ctx->G, gd, gs, gb, estr,
-                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
-                   CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) !=
-                CUDA_SUCCESS)
-            return bail(STITCH_ERR_CUDA);
-    }
-
     // Twiddles w_N^e = exp(-2 pi i e / N), computed in double, rounded once.
     //   stage-2 tables: tw2[b*(r1-1) + j-1] = w_N^{j b}, b < r0, 1 <= j < r1 (fft_engine.cuh)
     auto fill_tw = [&](auto* dst, auto make) {
@@ -1594,13 +1571,14 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
     if (ctx->prec) return fail(ctx, STITCH_ERR_STATE, "fp64 context: use stitch_debug_spectrum_f64");
     GUARD(ctx);
     // The resident store keeps Q15 unit phasors; recompute the complex spectrum of this tile
-    // with the same K1 + K2 kernels into the chunk buffer G (slot 0) and copy it out.
+    // with the same K1 + K2 kernels (G slot 0, K2 writing the complex spectrum row-major into
+    // the Q chunk buffer) and copy it out.
     const int lt = tile - ctx->L.h_begin;
     const PlanOps* o = ctx->ops;
     o->k1(ctx->raw, ctx->G, lt, 1, ctx->fslot, ctx->twM, ctx->twW, ctx->grid_k1, ctx->stream);
-    o->k2(ctx->tmG, ctx->G, ctx->spec, lt, 1, ctx->fslot, ctx->twH, false, 0, ctx->stream);
+    o->k2(ctx->G, ctx->Q, ctx->spec, lt, 1, ctx->fslot, ctx->twH, false, 0, ctx->stream);
     CK(cudaGetLastError(), "spectrum launch");
-    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->G,
+    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(float2), ctx->Q,
                          ctx->ops->WP * sizeof(float2), ctx->ops->WC * sizeof(float2), ctx->H,
                          cudaMemcpyDeviceToHost, ctx->stream),
        "copy spectrum");

@@ -201,15 +201,22 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB1)
         };
         RW::Fft::run(src, xc, xc, tw2s, lane, prefetch);   // natural-order Z back in place
         __syncwarp();
-        float2* out = G + (size_t)r * PL::WP;
-        for (int q = lane; q <= M / 2; q += 32) {
+        const int tl = r / H;
+        const GRow<PL> out{G + (size_t)tl * H * PL::WP, r - tl * H};   // panel-blocked (K2)
+        // bin q = lane + 32k sits at &out[lane] + k * 32H (4 panels further per k), its mirror
+        // M - q at &out[M - lane] - k * 32H (M is a multiple of the panel width)
+        static_assert(M % PL::COL_P == 0 && 32 % PL::COL_P == 0, "panel-blocked G strides");
+        constexpr int STEP = 32 / PL::COL_P * H * PL::COL_P;
+        float2* pf = &out[lane];
+        float2* pm = &out[M - lane];
+        for (int q = lane; q <= M / 2; q += 32, pf += STEP, pm -= STEP) {
             const float2 zq = xc.nat(q);
             const float2 zm = xc.nat(q == 0 ? 0 : M - q);
             const float2 E = make_float2(0.5f * (zq.x + zm.x), 0.5f * (zq.y - zm.y));
             const float2 O = make_float2(0.5f * (zq.y + zm.y), -0.5f * (zq.x - zm.x));
             const float2 wo = cmul(twWs[q], O);
-            out[q] = make_float2(E.x + wo.x, E.y + wo.y);
-            if (2 * q != M) out[M - q] = make_float2(E.x - wo.x, wo.y - E.y);
+            *pf = make_float2(E.x + wo.x, E.y + wo.y);
+            if (2 * q != M) *pm = make_float2(E.x - wo.x, wo.y - E.y);
         }
         for (int q = M + 1 + lane; q < PL::WP; q += 32) out[q] = make_float2(0.f, 0.f);
         __syncwarp();                          // exchange free for the next row
