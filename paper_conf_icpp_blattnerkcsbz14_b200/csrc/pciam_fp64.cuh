@@ -13,10 +13,13 @@
 //     (the key's value field carries |c| rounded to float, used only for the reported peak).
 // Kernels (plain CTA-per-block launches, coalesced global loads; no TMA: the fp64 path is
 // FP64-issue-bound on B200 long before it is HBM-bound):
-//   D1 fwd_rows   raw -> Gd   R2C along x (uint16 -> double fused into the load)
-//   D2 fwd_cols   Gd -> U     C2C along y, epilogue: unit phasor (or the complex spectrum
-//                             back into Gd for the parity hook)
-//   D3 pair_cols  U -> Qd     step 3 (U_A conj U_B) fused into the inverse C2C along y
+//   D1 fwd_rows   raw -> Gd   R2C along x (uint16 -> double fused into the load); Gd is
+//                             panel-blocked ([tile][WP/4][H][4]) like the fp32 G
+//   D2 fwd_cols   Gd -> U     C2C along y on a panel landed by one bulk copy, epilogue: unit
+//                             phasor, U column-major [slot][WP][HP64] (or the complex spectrum
+//                             row-major into Qd for the parity hook)
+//   D3 pair_cols  U -> Qd     the two tiles' panels land by one bulk copy each; step 3
+//                             (U_A conj U_B) fused into the inverse C2C along y
 //   D4 pair_rows  Qd -> part  C2R along x, |.| + per-block argmax (surface never stored)
 //   D5 argmax     part -> key per-pair reduction of the block partials
 #pragma once
@@ -43,10 +46,36 @@ struct Plan64 {
                                                            : COL_P * CI::R0);
     static constexpr int COL_T = (COL_WORK + 31) / 32 * 32;
     using ColX = ColXchg<CI::R0, CI::R1, PL::COL_PAD, COL_P, double2>;
-    static constexpr size_t COL_SMEM =
+    static constexpr size_t COL_XCH =
         CI::STAGES == 1 ? 16 : sizeof(double2) * COL_P * CI::R1 * (CI::R0 + PL::COL_PAD);
+    // column pitch of the column-major unit phasor U (double2): >= H, 2 mod 8, so the 16-byte
+    // loads of a landed 4-column panel (8 lanes per wavefront: 4 columns x 2 rows) are
+    // bank-conflict-free
+    static constexpr int HP64 = H % 8 <= 2 ? H + (2 - H % 8) : H + (10 - H % 8);
+    static constexpr size_t PANEL_G = sizeof(double2) * COL_P * H;      // D2's landed Gd panel
+    static constexpr size_t D2_SMEM = (PANEL_G > COL_XCH ? PANEL_G : COL_XCH);
+    // D3 takes 2-column panels of U (any column run of the column-major U is contiguous): two
+    // landed panels (2 x 33 KB) + the aliased exchange let two 3-warp CTAs share an SM, so one
+    // CTA's landing overlaps the other's butterflies (the radix-40 double butterfly's 254
+    // registers allow no more warps)
+    static constexpr int COL_P3 = 2;
+    static constexpr int COL_WORK3 = CI::STAGES == 1 ? COL_P3
+                                                     : (CI::R1 > CI::R0 ? COL_P3 * CI::R1
+                                                                        : COL_P3 * CI::R0);
+    static constexpr int COL_T3 = (COL_WORK3 + 31) / 32 * 32;
+    using ColX3 = ColXchg<CI::R0, CI::R1, PL::COL_PAD, COL_P3, double2>;
+    static constexpr size_t COL_XCH3 =
+        CI::STAGES == 1 ? 16 : sizeof(double2) * COL_P3 * CI::R1 * (CI::R0 + PL::COL_PAD);
+    static constexpr size_t PANEL_U = sizeof(double2) * COL_P3 * HP64;  // one tile's U panel
+    static constexpr size_t U_B_OFF = (PANEL_U + 127) / 128 * 128;      // D3's second panel
+    static constexpr size_t D3_SMEM =
+        (U_B_OFF + PANEL_U > COL_XCH3 ? U_B_OFF + PANEL_U : COL_XCH3);
+    // D4: the block's ROW_L rows of Q land by one bulk copy, reused as the exchange
+    static constexpr size_t ROWS_Q = sizeof(double2) * ROW_L * WP;
+    static constexpr size_t D4_SMEM = ROWS_Q > ROW_SMEM ? ROWS_Q : ROW_SMEM;
     static_assert(WP % COL_P == 0, "fp64 column panel must divide the pitch");
-    static_assert(ROW_SMEM <= 200 * 1024 && COL_SMEM <= 200 * 1024, "fp64 shared memory");
+    static_assert(D2_SMEM <= 200 * 1024 && D3_SMEM <= 200 * 1024 && D4_SMEM <= 200 * 1024,
+                  "fp64 shared memory");
 };
 
 // ------------------------------------------------------------------ D1 ----
@@ -62,8 +91,19 @@ struct U16RowSrcD {  // z[n] = x[2n] + i x[2n+1] (exact in double)
 // R2C post-processing of one line in double (the fp32 r2c_post_line, pciam_kernels.cuh):
 //   E = (Z[q] + conj Z[M-q]) / 2,  O = (Z[q] - conj Z[M-q]) / (2i)
 //   X[q] = E + w_W^q O,   X[M-q] = conj(E - w_W^q O)
+// Gd's panel-blocked layout (the fp32 GRow with 4-column double2 panels: 64-byte runs)
+template <class PL>
+struct GRowD {
+    double2* t;
+    int y;
+    __device__ __forceinline__ double2& operator[](int q) const {
+        constexpr int P = Plan64<PL>::COL_P;
+        return t[((size_t)(q / P) * PL::H + y) * P + q % P];
+    }
+};
+
 template <class PL, class Xc>
-__device__ __forceinline__ void r2c_post_line_d(const Xc& xc, int line, double2* __restrict__ out,
+__device__ __forceinline__ void r2c_post_line_d(const Xc& xc, int line, const GRowD<PL>& out,
                                                 const double2* __restrict__ twW) {
     constexpr int M = PL::M;
     for (int q = threadIdx.x; q <= M / 2; q += PL::ROW_T) {
@@ -84,7 +124,7 @@ __global__ void __launch_bounds__(PL::ROW_T) d1_fwd_rows(const uint16_t* __restr
                                                          const double2* __restrict__ tw2,
                                                          const double2* __restrict__ twW) {
     using P64 = Plan64<PL>;
-    extern __shared__ __align__(16) unsigned char smem64[];
+    extern __shared__ __align__(128) unsigned char smem64[];
     constexpr int L = P64::ROW_L, T = P64::ROW_T;
     const size_t t = (size_t)tile0 + blockIdx.y;
     const int y0 = blockIdx.x * L;
@@ -94,7 +134,8 @@ __global__ void __launch_bounds__(PL::ROW_T) d1_fwd_rows(const uint16_t* __restr
     __syncthreads();
 #pragma unroll 1
     for (int line = 0; line < L; ++line)
-        r2c_post_line_d<PL>(xc, line, G + ((size_t)blockIdx.y * PL::H + y0 + line) * PL::WP, twW);
+        r2c_post_line_d<PL>(xc, line, GRowD<PL>{G + (size_t)blockIdx.y * PL::H * PL::WP, y0 + line},
+                            twW);
 }
 
 // ------------------------------------------------------------------ D2 ----
@@ -110,63 +151,99 @@ struct PanelIOD {  // a panel of columns of one [H][WP] double2 array
 };
 
 template <class PL>
-struct UnitDst {  // resident spectrum: U = F/|F|, 0 where F = 0 (reading C4)
+struct UnitDst {  // spectrum: U = F/|F|, 0 where F = 0 (reading C4), column-major panel
     double2* p;
     __device__ __forceinline__ void store(int line, int n, double2 v) const {
         const double m2 = fma(v.x, v.x, v.y * v.y);
         const double r = m2 > 0.0 ? rsqrt(m2) : 0.0;
-        p[(size_t)n * PL::WP + line] = make_double2(v.x * r, v.y * r);
+        p[(size_t)line * Plan64<PL>::HP64 + n] = make_double2(v.x * r, v.y * r);
     }
 };
 
-// Every stage-1 read of the panel precedes the barrier before stage 2 (or, single-stage,
-// each butterfly owns its whole column), so the complex output may overwrite Gd in place.
+template <class PL>
+struct LandSrcD {  // a landed Gd panel [H][COL_P] in shared memory
+    const double2* s;
+    __device__ __forceinline__ double2 load(int line, int n) const {
+        return s[n * Plan64<PL>::COL_P + line];
+    }
+};
+
+// The panel lands by one bulk copy (Gd is panel-blocked); the landing buffer becomes the
+// exchange once stage 1 has read it (IN_PLACE).  UNIT_OUT = false: the parity hook's complex
+// spectrum, row-major [H][WP], into `out`.
+// two 5-warp CTAs per SM (register-budgeted by the launch bounds)
 template <class PL, bool UNIT_OUT>
-__global__ void __launch_bounds__(Plan64<PL>::COL_T) d2_fwd_cols(double2* __restrict__ G,
+__global__ void __launch_bounds__(Plan64<PL>::COL_T, 2) d2_fwd_cols(const double2* __restrict__ G,
                                                                  double2* __restrict__ U,
+                                                                 double2* __restrict__ out,
                                                                  int tile0,
                                                                  const double2* __restrict__ tw2) {
     using P64 = Plan64<PL>;
-    extern __shared__ __align__(16) unsigned char smem64[];
+    extern __shared__ __align__(128) unsigned char smem64[];
+    __shared__ uint64_t bar;
     const int tl = blockIdx.y, c0 = blockIdx.x * P64::COL_P;
-    PanelIOD<PL> src{G + (size_t)tl * PL::H * PL::WP + c0};
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        mbar_arrive_expect_tx(&bar, (uint32_t)P64::PANEL_G);
+        bulk_g2s(smem64, G + ((size_t)tl * PL::WP + c0) * PL::H, (uint32_t)P64::PANEL_G, &bar);
+    }
+    mbar_wait(&bar, 0);
+    LandSrcD<PL> src{reinterpret_cast<const double2*>(smem64)};
     typename P64::ColX xc{reinterpret_cast<double2*>(smem64)};
     using Run = FftRun<typename P64::Col, -1, P64::COL_P, P64::COL_T, ColMap, false, double2>;
     if constexpr (UNIT_OUT) {
-        UnitDst<PL> dst{U + (size_t)(tile0 + tl) * PL::H * PL::WP + c0};
-        Run::run(src, xc, dst, tw2);
+        UnitDst<PL> dst{U + ((size_t)(tile0 + tl) * PL::WP + c0) * P64::HP64};
+        Run::template run<true>(src, xc, dst, tw2);
     } else {
-        Run::run(src, xc, src, tw2);
+        PanelIOD<PL> dst{out + (size_t)tl * PL::H * PL::WP + c0};
+        Run::template run<true>(src, xc, dst, tw2);
     }
 }
 
 // ------------------------------------------------------------------ D3 ----
 template <class PL>
 struct NcpsUnitSrc {  // step 3: U_A conj(U_B) = F_A conj(F_B) / |F_A conj(F_B)| (0 if either is 0)
-    const double2* a;
+    const double2* a;  // landed column-major panels [COL_P][HP64]
     const double2* b;
     __device__ __forceinline__ double2 load(int line, int n) const {
-        const size_t o = (size_t)n * PL::WP + line;
-        return cmulc(__ldg(a + o), __ldg(b + o));
+        const int o = line * Plan64<PL>::HP64 + n;
+        return cmulc(a[o], b[o]);
     }
 };
 
 template <class PL>
-__global__ void __launch_bounds__(Plan64<PL>::COL_T) d3_pair_cols(const double2* __restrict__ U,
+__global__ void __launch_bounds__(Plan64<PL>::COL_T3, 2) d3_pair_cols(const double2* __restrict__ U,
                                                                   double2* __restrict__ Q,
                                                                   const PairIdx* __restrict__ pairs,
                                                                   int pair0,
                                                                   const double2* __restrict__ tw2) {
     using P64 = Plan64<PL>;
-    extern __shared__ __align__(16) unsigned char smem64[];
+    extern __shared__ __align__(128) unsigned char smem64[];
+    __shared__ uint64_t bar;
     const PairIdx pr = pairs[pair0 + blockIdx.y];
-    const int c0 = blockIdx.x * P64::COL_P;
-    NcpsUnitSrc<PL> src{U + (size_t)pr.a * PL::H * PL::WP + c0,
-                        U + (size_t)pr.b * PL::H * PL::WP + c0};
+    const int c0 = blockIdx.x * P64::COL_P3;
+    double2* la = reinterpret_cast<double2*>(smem64);
+    double2* lb = reinterpret_cast<double2*>(smem64 + P64::U_B_OFF);
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {   // each tile's panel is one contiguous run of U: one bulk copy each
+        mbar_arrive_expect_tx(&bar, 2 * (uint32_t)P64::PANEL_U);
+        bulk_g2s(la, U + ((size_t)pr.a * PL::WP + c0) * P64::HP64, (uint32_t)P64::PANEL_U, &bar);
+        bulk_g2s(lb, U + ((size_t)pr.b * PL::WP + c0) * P64::HP64, (uint32_t)P64::PANEL_U, &bar);
+    }
+    mbar_wait(&bar, 0);
+    NcpsUnitSrc<PL> src{la, lb};
     PanelIOD<PL> dst{Q + (size_t)blockIdx.y * PL::H * PL::WP + c0};
-    typename P64::ColX xc{reinterpret_cast<double2*>(smem64)};
-    FftRun<typename P64::Col, +1, P64::COL_P, P64::COL_T, ColMap, false, double2>::run(src, xc, dst,
-                                                                                      tw2);
+    typename P64::ColX3 xc{reinterpret_cast<double2*>(smem64)};
+    FftRun<typename P64::Col, +1, P64::COL_P3, P64::COL_T3, ColMap, false, double2>::template run<
+        true>(src, xc, dst, tw2);
 }
 
 // ------------------------------------------------------------------ D4 ----
@@ -220,22 +297,35 @@ __device__ __forceinline__ void warp_argmax(double& v, uint32_t& i) {
 }
 
 template <class PL>
-__global__ void __launch_bounds__(PL::ROW_T) d4_pair_rows(const double2* __restrict__ Q,
+__global__ void __launch_bounds__(PL::ROW_T, 3) d4_pair_rows(const double2* __restrict__ Q,
                                                           double* __restrict__ part_v,
                                                           uint32_t* __restrict__ part_i,
                                                           int pair0,
                                                           const double2* __restrict__ tw2,
                                                           const double2* __restrict__ twW) {
     using P64 = Plan64<PL>;
-    extern __shared__ __align__(16) unsigned char smem64[];
+    extern __shared__ __align__(128) unsigned char smem64[];
     __shared__ double rv[(PL::ROW_T + 31) / 32];
     __shared__ uint32_t ri[(PL::ROW_T + 31) / 32];
     constexpr int L = P64::ROW_L, T = P64::ROW_T;
     const int y0 = blockIdx.x * L;
-    C2RSrcD<PL> src{Q + ((size_t)blockIdx.y * PL::H + y0) * PL::WP, twW};
+    __shared__ uint64_t bar;
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {   // the block's L consecutive rows of Q: one bulk copy
+        mbar_arrive_expect_tx(&bar, (uint32_t)P64::ROWS_Q);
+        bulk_g2s(smem64, Q + ((size_t)blockIdx.y * PL::H + y0) * PL::WP, (uint32_t)P64::ROWS_Q,
+                 &bar);
+    }
+    mbar_wait(&bar, 0);
+    C2RSrcD<PL> src{reinterpret_cast<const double2*>(smem64), twW};
     ArgmaxDstD dst{-1.0, 0xFFFFFFFFu, y0, PL::W};
-    typename P64::RowX xc{reinterpret_cast<double2*>(smem64)};
-    FftRun<typename P64::Row, +1, L, T, RowMap, false, double2>::run(src, xc, dst, tw2);
+    typename P64::RowX xc{reinterpret_cast<double2*>(smem64)};   // reuses the landing buffer
+    FftRun<typename P64::Row, +1, L, T, RowMap, false, double2>::template run<true>(src, xc, dst,
+                                                                                   tw2);
     double v = dst.best_v;
     uint32_t i = dst.best_i;
     warp_argmax(v, i);

@@ -92,14 +92,10 @@ struct Plan {
     static constexpr size_t COL_STG_OFF = (COL_SMEM + 127) / 128 * 128;
     static constexpr size_t COL_SMEM_K2 = COL_STG_OFF + COL_PANEL_P;
     // CTAs per SM the column kernels are register-budgeted for (shared memory allows this many)
+    // CTAs per SM the column kernels are built for (shared memory allows this many, <= 2:
+    // the radix-40 butterfly's registers fit two 7-warp CTAs)
     static constexpr int COL_MINB_RAW = (int)((220 * 1024) / (COL_SMEM + 1024));
-    static constexpr int COL_MINB = COL_MINB_RAW > 4 ? 4 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
-    // register cap so COL_MINB CTAs of COL_T threads fit: the 64K-register file is split
-    // over the 4 SM sub-partitions (16K each) and warps are dealt to them round robin
-    static constexpr int COL_WARPS = (COL_T + 31) / 32;
-    static constexpr int COL_WPS = (COL_MINB * COL_WARPS + 3) / 4;   // warps per sub-partition
-    static constexpr int COL_MAXREG_RAW = (16384 / (COL_WPS * 32)) / 8 * 8;
-    static constexpr int COL_MAXREG = COL_MAXREG_RAW > 255 ? 255 : COL_MAXREG_RAW;
+    static constexpr int COL_MINB = COL_MINB_RAW > 2 ? 2 : (COL_MINB_RAW < 1 ? 1 : COL_MINB_RAW);
     // stage-2 twiddle tables (w_N^{-j b}, see fft_engine.cuh)
     static constexpr int ROW_TW2 = RI::R0 * (RI::R1 - 1);
     static constexpr int COL_TW2 = CI::R0 * (CI::R1 - 1);
@@ -266,7 +262,7 @@ struct ColTw {
 // prefetch of the panel of the CTA that many launch slots later (one wave of resident CTAs:
 // K2 7.25 -> 6.86 ms).
 template <class PL, bool PHASE_OUT>
-__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
+__global__ void __launch_bounds__(PL::COL_T, PL::COL_MINB)
     k2t_fwd_cols(const float2* __restrict__ G, float2* __restrict__ out,
                  uint32_t* __restrict__ spec, int tile0, const int32_t* __restrict__ fslot,
                  const float2* __restrict__ tw2, int ahead) {
@@ -328,7 +324,7 @@ struct NcpsPhaseSrc {  // step 3 from two landed phasor panels: U_A conj(U_B) (x
 };
 
 template <class PL>
-__global__ void __launch_bounds__(PL::COL_T) __maxnreg__(PL::COL_MAXREG)
+__global__ void __launch_bounds__(PL::COL_T, PL::COL_MINB)
     k3t_pair_cols(const uint32_t* __restrict__ spec, float2* __restrict__ Q,
                   const PairIdx* __restrict__ pairs, int pair0, const float2* __restrict__ tw2) {
     extern __shared__ __align__(128) unsigned char csmem[];

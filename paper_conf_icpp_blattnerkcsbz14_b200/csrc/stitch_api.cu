@@ -53,7 +53,7 @@ using P58 = Plan<58, 26, Radix<29, 29>, Radix<26, 26>, 2, 32, 8, 32, 0, 0>;
 constexpr int PAIR_BAND = 4;
 
 struct PlanOps {
-    int W, H, M, WC, WP, HP, col_p;
+    int W, H, M, WC, WP, HP, HP64, col_p;
     int row_r0, row_r1, col_r0, col_r1;   // stage radices (r1 = 1: single stage)
     cudaError_t (*setup)(int* grid_k1, int* grid_k4);
     void (*k1)(const uint16_t*, float2*, int, int, const int32_t*, const float2*, const float2*,
@@ -70,7 +70,7 @@ struct PlanOps {
     int nblk64;
     cudaError_t (*d_setup)();
     void (*d1)(const uint16_t*, double2*, int, int, const double2*, const double2*, cudaStream_t);
-    void (*d2)(double2*, double2*, int, int, const double2*, bool, cudaStream_t);
+    void (*d2)(const double2*, double2*, double2*, int, int, const double2*, bool, cudaStream_t);
     void (*d3)(const double2*, double2*, const PairIdx*, int, int, const double2*, cudaStream_t);
     void (*d4)(const double2*, double*, uint32_t*, int, int, const double2*, const double2*,
                cudaStream_t);
@@ -200,10 +200,10 @@ template <class PL>
 cudaError_t d_setup() {
     using P64 = Plan64<PL>;
     CKE(max_smem(d1_fwd_rows<PL>, P64::ROW_SMEM));
-    CKE(max_smem(d4_pair_rows<PL>, P64::ROW_SMEM));
-    CKE(max_smem(d2_fwd_cols<PL, true>, P64::COL_SMEM));
-    CKE(max_smem(d2_fwd_cols<PL, false>, P64::COL_SMEM));
-    return max_smem(d3_pair_cols<PL>, P64::COL_SMEM);
+    CKE(max_smem(d4_pair_rows<PL>, P64::D4_SMEM));
+    CKE(max_smem(d2_fwd_cols<PL, true>, P64::D2_SMEM));
+    CKE(max_smem(d2_fwd_cols<PL, false>, P64::D2_SMEM));
+    return max_smem(d3_pair_cols<PL>, P64::D3_SMEM);
 }
 template <class PL>
 void launch_d1(const uint16_t* raw, double2* G, int t0, int nt, const double2* tw2,
@@ -212,34 +212,34 @@ void launch_d1(const uint16_t* raw, double2* G, int t0, int nt, const double2* t
     d1_fwd_rows<PL><<<dim3(P64::NBLK, nt), P64::ROW_T, P64::ROW_SMEM, s>>>(raw, G, t0, tw2, twW);
 }
 template <class PL>
-void launch_d2(double2* G, double2* U, int t0, int nt, const double2* tw2, bool unit_out,
-               cudaStream_t s) {
+void launch_d2(const double2* G, double2* U, double2* out, int t0, int nt, const double2* tw2,
+               bool unit_out, cudaStream_t s) {
     using P64 = Plan64<PL>;
     const dim3 grid(PL::WP / P64::COL_P, nt);
     if (unit_out)
-        d2_fwd_cols<PL, true><<<grid, P64::COL_T, P64::COL_SMEM, s>>>(G, U, t0, tw2);
+        d2_fwd_cols<PL, true><<<grid, P64::COL_T, P64::D2_SMEM, s>>>(G, U, out, t0, tw2);
     else
-        d2_fwd_cols<PL, false><<<grid, P64::COL_T, P64::COL_SMEM, s>>>(G, U, t0, tw2);
+        d2_fwd_cols<PL, false><<<grid, P64::COL_T, P64::D2_SMEM, s>>>(G, U, out, t0, tw2);
 }
 template <class PL>
 void launch_d3(const double2* U, double2* Q, const PairIdx* pairs, int p0, int np,
                const double2* tw2, cudaStream_t s) {
     using P64 = Plan64<PL>;
-    d3_pair_cols<PL><<<dim3(PL::WP / P64::COL_P, np), P64::COL_T, P64::COL_SMEM, s>>>(U, Q, pairs,
+    d3_pair_cols<PL><<<dim3(PL::WP / P64::COL_P3, np), P64::COL_T3, P64::D3_SMEM, s>>>(U, Q, pairs,
                                                                                       p0, tw2);
 }
 template <class PL>
 void launch_d4(const double2* Q, double* pv, uint32_t* pi, int p0, int np, const double2* tw2,
                const double2* twW, cudaStream_t s) {
     using P64 = Plan64<PL>;
-    d4_pair_rows<PL><<<dim3(P64::NBLK, np), P64::ROW_T, P64::ROW_SMEM, s>>>(Q, pv, pi, p0, tw2,
+    d4_pair_rows<PL><<<dim3(P64::NBLK, np), P64::ROW_T, P64::D4_SMEM, s>>>(Q, pv, pi, p0, tw2,
                                                                             twW);
 }
 
 template <class PL>
 PlanOps make_ops() {
     PlanOps o;
-    o.W = PL::W; o.H = PL::H; o.M = PL::M; o.WC = PL::WC; o.WP = PL::WP; o.HP = PL::HP;
+    o.W = PL::W; o.H = PL::H; o.M = PL::M; o.WC = PL::WC; o.WP = PL::WP; o.HP = PL::HP; o.HP64 = Plan64<PL>::HP64;
     o.col_p = PL::COL_P;
     o.row_r0 = PL::RI::R0; o.row_r1 = PL::RI::R1; o.col_r0 = PL::CI::R0; o.col_r1 = PL::CI::R1;
     o.setup = plan_setup<PL>;
@@ -381,7 +381,8 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     // spectrum by slot: u32 Q15 unit phasor [WP][HP] (fp32) or double2 unit phasor [H][WP] (fp64)
-    L->spec_tile_bytes = L->prec ? H * WP * sizeof(double2) : (size_t)ops->HP * WP * sizeof(uint32_t);
+    L->spec_tile_bytes = L->prec ? (size_t)ops->HP64 * WP * sizeof(double2)
+                                 : (size_t)ops->HP * WP * sizeof(uint32_t);
     const size_t cplx = L->prec ? sizeof(double2) : sizeof(float2);
     const size_t np1 = (size_t)(np > 0 ? np : 1);
     size_t o = 0;
@@ -761,7 +762,7 @@ static void launch_fwd(stitch_ctx* ctx, int t0, int nt, cudaStream_t s, int si) 
     if (ctx->prec) {   // fp64 path (f2): D1, D2 (resident tiles: slot = local tile)
         tl_wrap(ctx, s, si, 0, [&] { o->d1(ctx->raw, ctx->Gd, t0, nt, ctx->twMd, ctx->twWd, s); });
         mark(ctx, 0);
-        tl_wrap(ctx, s, si, 1, [&] { o->d2(ctx->Gd, ctx->Ud, t0, nt, ctx->twHd, true, s); });
+        tl_wrap(ctx, s, si, 1, [&] { o->d2(ctx->Gd, ctx->Ud, nullptr, t0, nt, ctx->twHd, true, s); });
         mark(ctx, 1);
         ctx->launches += 2;
         return;
@@ -1595,13 +1596,13 @@ stitch_status stitch_debug_spectrum_f64(stitch_ctx* ctx, int32_t tile, double* h
     if (!ctx->loaded) return fail(ctx, STITCH_ERR_STATE, "spectrum before load");
     GUARD(ctx);
     // the resident store keeps unit phasors: recompute this tile's complex spectrum with the
-    // same D1 + D2 kernels into chunk slot 0 of Gd (D2 writing complex values in place)
+    // same D1 + D2 kernels (Gd slot 0; D2 writing the complex spectrum row-major into Qd)
     const int lt = tile - ctx->L.h_begin;
     const PlanOps* o = ctx->ops;
     o->d1(ctx->raw, ctx->Gd, lt, 1, ctx->twMd, ctx->twWd, ctx->stream);
-    o->d2(ctx->Gd, ctx->Ud, lt, 1, ctx->twHd, false, ctx->stream);
+    o->d2(ctx->Gd, ctx->Ud, ctx->Qd, lt, 1, ctx->twHd, false, ctx->stream);
     CK(cudaGetLastError(), "spectrum launch");
-    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(double2), ctx->Gd,
+    CK(cudaMemcpy2DAsync(host_out, ctx->ops->WC * sizeof(double2), ctx->Qd,
                          ctx->ops->WP * sizeof(double2), ctx->ops->WC * sizeof(double2), ctx->H,
                          cudaMemcpyDeviceToHost, ctx->stream),
        "copy spectrum");
