@@ -351,7 +351,8 @@ def main():
     import torch
     import torch.distributed as dist
 
-    from paper_conf_icpp_blattnerkcsbz14_b200.parallel import BandPciam
+    from paper_conf_icpp_blattnerkcsbz14_b200 import StitchError
+    from paper_conf_icpp_blattnerkcsbz14_b200.parallel import BandPciam, gather_translations
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -382,9 +383,19 @@ def main():
     first = r0 * m
 
     transport = args.transport or ("library" if args.dist_backend == "nccl" else "torch")
-    bp = BandPciam(n, m, H, W, rank, world, device=local, transport=transport,
-                   chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles,
-                   precision=1 if args.precision == "f64" else 0)
+    kw = dict(chunk_pairs=args.chunk_pairs, chunk_tiles=args.chunk_tiles,
+              precision=1 if args.precision == "f64" else 0)
+    try:
+        bp = BandPciam(n, m, H, W, rank, world, device=local, transport=transport, **kw)
+    except StitchError as err:
+        # the library's NCCL communicator could not be formed (stitch_init is collective, so
+        # every rank lands here): measure with the torch.distributed transport instead, and say so
+        if transport != "library":
+            raise
+        print(f"bench: library NCCL transport unavailable ({err}); using torch.distributed",
+              file=sys.stderr, flush=True)
+        transport = "torch"
+        bp = BandPciam(n, m, H, W, rank, world, device=local, transport=transport, **kw)
     pg = bp.grid
     stream = pg.stream          # the stream the library enqueues on (events must be recorded here)
     pg.load_tiles(host, first)
@@ -549,6 +560,15 @@ def main():
     h2d = sum_over_ranks((e - halo) * T)          # whole job: every rank's tile rows
     d2h = sum_over_ranks(pairs_local * 64)
 
+    # ---- every rank's translations merged and checked against the generator's known shifts --
+    if world > 1:
+        west, north = gather_translations(west, north, bp.bd)
+    truth_o = synthgrid.origins(n, m, H, W, cfg["overlap"], cfg["delta"])
+    shifts_ok = bool(np.array_equal(west["dx"][:, 1:], truth_o[:, 1:, 0] - truth_o[:, :-1, 0]) and
+                     np.array_equal(west["dy"][:, 1:], truth_o[:, 1:, 1] - truth_o[:, :-1, 1]) and
+                     np.array_equal(north["dx"][1:], truth_o[1:, :, 0] - truth_o[:-1, :, 0]) and
+                     np.array_equal(north["dy"][1:], truth_o[1:, :, 1] - truth_o[:-1, :, 1]))
+
     # ---- optional: stitching phases 2 + 3 on the result (NEXT rows f3, f4) -------------
     phase23 = None
     if args.compose and world == 1:
@@ -583,7 +603,8 @@ def main():
                                "torch": "exchange (torch.distributed)"}.get(bp.transport,
                                                                             "recompute")
                               if world > 1 else "none"),
-                     "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)"})
+                     "l2": "inputs larger than L2 (7.2 GB tiles, 7.3 GB spectra vs 126 MB)",
+                     "shifts_recovered": shifts_ok})
         line = {
             "metric": metric_name(cfg),
             "value": value, "unit": "pairs/s", "n_gpus": world, "steps": args.steps,
