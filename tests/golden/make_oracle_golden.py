@@ -46,6 +46,14 @@ CASES = {
                       density=0.02, search=dict(start=1000, min_ambiguous=3)),
     "lowtex1392": dict(n=10, m=12, H=1040, W=1392, overlap=0.10, delta=12, texture="cells",
                        density=0.01, search=dict(start=2000, min_ambiguous=1)),
+    # configs[4]: the 100x100 grid ("up to 10 000 tiles")
+    "cfg5": dict(n=100, m=100, H=1040, W=1392, overlap=0.10, delta=12, seed=synthgrid.SEED),
+    # configs[3]: two grids of the 161-scan x 2-channel time series: the first scan's
+    # second channel (another texture seed) and the last scan's first channel (re-jittered origins)
+    "ts_s0c1": dict(n=18, m=22, H=1040, W=1392, overlap=0.10, delta=12, seed=synthgrid.SEED,
+                    scan=0, channel=1),
+    "ts_s160c0": dict(n=18, m=22, H=1040, W=1392, overlap=0.10, delta=12, seed=synthgrid.SEED,
+                      scan=160, channel=0),
 }
 NEAR_TIE = 1e-4
 BAND = 8
@@ -59,7 +67,7 @@ def grid_sha(tiles_iter) -> str:
 
 
 def render(p, rows):
-    kw = {k: p[k] for k in ("overlap", "delta", "seed") if k in p}
+    kw = {k: p[k] for k in ("overlap", "delta", "seed", "scan", "channel") if k in p}
     if "texture" in p:
         kw["texture"] = p["texture"]
         kw["density"] = p["density"]

@@ -15,7 +15,7 @@ import oracle
 import synthgrid
 
 GOLD = os.path.join(os.path.dirname(os.path.abspath(__file__)), "golden")
-CASES = ["cfg2", "cfg3", "cfg3_ov70", "lowtex256", "lowtex1392"]
+CASES = ["cfg2", "cfg3", "cfg3_ov70", "lowtex256", "lowtex1392", "cfg5", "ts_s0c1", "ts_s160c0"]
 FIELDS = ["dx", "dy", "candidate", "peak_x", "peak_y", "peak", "runner_up", "ccf"]
 
 
@@ -28,7 +28,8 @@ def load(name):
 
 
 def render(p, rows=None):
-    kw = dict(overlap=p["overlap"], delta=p["delta"], seed=p["seed"])
+    kw = dict(overlap=p["overlap"], delta=p["delta"], seed=p["seed"], scan=p.get("scan", 0),
+              channel=p.get("channel", 0))
     if "texture" in p:
         kw.update(texture=p["texture"], density=p["density"])
     return synthgrid.make_grid(p["n"], p["m"], p["H"], p["W"], rows=rows, **kw)
@@ -70,9 +71,13 @@ def test_low_texture_fixtures_hold_near_ties(name, k):
 def test_full_size_fixtures_recover_the_known_shifts():
     """At 10 % and 70 % overlap the oracle recovers every generator shift of the headline grid
     (a pin of the oracle at full size, independent of the GPU)."""
-    for name in ("cfg2", "cfg3", "cfg3_ov70"):
+    for name in ("cfg2", "cfg3", "cfg3_ov70", "cfg5", "ts_s0c1", "ts_s160c0"):
+        path = os.path.join(GOLD, f"oracle_{name}.npz")
+        if not os.path.exists(path):
+            continue
         p, west, north, _ = load(name)
-        o = synthgrid.origins(p["n"], p["m"], p["H"], p["W"], p["overlap"], p["delta"], p["seed"])
+        o = synthgrid.origins(p["n"], p["m"], p["H"], p["W"], p["overlap"], p["delta"], p["seed"],
+                              scan=p.get("scan", 0), channel=p.get("channel", 0))
         assert np.array_equal(west["dx"][:, 1:], (o[:, 1:, 0] - o[:, :-1, 0])), name
         assert np.array_equal(west["dy"][:, 1:], (o[:, 1:, 1] - o[:, :-1, 1])), name
         assert np.array_equal(north["dx"][1:], (o[1:, :, 0] - o[:-1, :, 0])), name

@@ -38,22 +38,26 @@ def load_case(name):
 
 
 def render(p):
-    kw = dict(overlap=p["overlap"], delta=p["delta"], seed=p["seed"])
+    kw = dict(overlap=p["overlap"], delta=p["delta"], seed=p["seed"], scan=p.get("scan", 0),
+              channel=p.get("channel", 0))
     if "texture" in p:
         kw.update(texture=p["texture"], density=p["density"])
     return synthgrid.make_grid(p["n"], p["m"], p["H"], p["W"], **kw)
 
 
-def run_case(name, expect_truth=True, min_ambiguous=0):
+def run_case(name, expect_truth=True, min_ambiguous=0, results=None):
     p, ow, on, sha = load_case(name)
     g = render(p)
     assert hashlib.sha256(g.tiles.tobytes()).hexdigest() == sha, "generator drift"
     n, m = p["n"], p["m"]
-    with PciamGrid(n, m, p["H"], p["W"], device=0) as pg:      # the bench's launch configuration
-        pg.load_grid(g.tiles)
-        west, north = pg.compute_translations()
-        counts = pg.last_counts()
-    assert counts["pairs"] == 2 * n * m - n - m
+    if results is None:
+        with PciamGrid(n, m, p["H"], p["W"], device=0) as pg:  # the bench's launch configuration
+            pg.load_grid(g.tiles)
+            west, north = pg.compute_translations()
+            counts = pg.last_counts()
+        assert counts["pairs"] == 2 * n * m - n - m
+    else:
+        west, north = results(g)
     stats = {}
     amb = _parity.grid_parity(g.tiles, west, north, ow, on, stats)
     print(f"{name}: {2 * n * m - n - m} pairs compared, {amb} near-tie pairs (C17) "
@@ -80,6 +84,31 @@ def test_config3_headline_every_pair_matches_oracle():
 @pytest.mark.slow
 def test_config3_overlap70_every_pair_matches_oracle():
     run_case("cfg3_ov70")
+
+
+@pytest.mark.slow
+def test_config5_every_pair_matches_oracle():
+    """configs[4]: every pair of the 100x100 grid (19,800 pairs; 29 GB of tiles)."""
+    if not os.path.exists(os.path.join(GOLD, "oracle_cfg5.npz")):
+        pytest.skip("oracle_cfg5.npz not generated")
+    run_case("cfg5")
+
+
+def test_time_series_grids_through_the_stream_match_oracle():
+    """configs[3]: two grids of the 161-scan x 2-channel series (another channel's texture; the
+    last scan's re-jittered origins), pushed through the streaming path (stream.GridStream, two
+    slots, H2D pipelined) in one run, every pair against the oracle."""
+    from paper_conf_icpp_blattnerkcsbz14_b200.stream import GridStream
+    names = ["ts_s0c1", "ts_s160c0"]
+    cases = [load_case(nm) for nm in names]
+    grids = [render(c[0]) for c in cases]
+    got = {}
+    p0 = cases[0][0]
+    with GridStream(p0["n"], p0["m"], p0["H"], p0["W"], slots=2) as gs:
+        gs.run(range(2), lambda i, host: grids[i].tiles,
+               lambda r: got.__setitem__(r.index, (r.west, r.north)))
+    for i, nm in enumerate(names):
+        run_case(nm, results=lambda g, i=i: got[i])
 
 
 def test_low_texture_256_near_ties():
