@@ -560,7 +560,7 @@ __device__ __forceinline__ void row_moments_pk(MomentsPk& m, Moments& mt, const 
     const uint32_t* b32 = reinterpret_cast<const uint32_t*>(br);
     const uint32_t* a32 = reinterpret_cast<const uint32_t*>(ar + off - (ODD ? 1 : 0));
     const int npk = w >> 1;
-#pragma unroll 2
+#pragma unroll 4
     for (int q = lane; q < npk; q += 32) {
         uint32_t wa;
         if constexpr (ODD) wa = __funnelshift_r(a32[q], a32[q + 1], 16);
