@@ -117,9 +117,15 @@ def band(rank: int, world: int, n: int, m: int):
 
 
 # The oracle's bounded sample (cpu_baseline and the reference arm time the same one): the
-# top-left SUB corner of the workload's grid -- the same tiles and pair kinds as the GPU
-# step -- through oracle.grid (fp64, Fig. 4 over Fig. 2) on every host core.
-SUB = (4, 5)
+# top-left 4 x c corner of the workload's grid -- the same tiles and pair kinds as the GPU
+# step -- through oracle.grid (fp64, Fig. 4 over Fig. 2) on every host core; c is chosen so the
+# corner holds about two tiles per core (the oracle's forward phase spreads tiles over threads),
+# i.e. a few seconds of work per sample.
+
+
+def sub_grid():
+    cores = os.cpu_count() or 1
+    return 4, max(3, round(2 * cores / 4))
 
 
 def metric_name(cfg: dict) -> str:
@@ -135,11 +141,12 @@ def workload_config(cfg: dict, config_index: int) -> dict:
 
 
 def oracle_sample(cfg: dict):
-    g = synthgrid.make_grid(SUB[0], SUB[1], cfg["H"], cfg["W"], overlap=cfg["overlap"],
+    r, c = sub_grid()
+    g = synthgrid.make_grid(r, c, cfg["H"], cfg["W"], overlap=cfg["overlap"],
                             delta=cfg["delta"])
-    pairs = 2 * SUB[0] * SUB[1] - SUB[0] - SUB[1]
-    desc = (f"{SUB[0]}x{SUB[1]} corner of the {cfg['name']} grid ({pairs} pairs, "
-            f"{SUB[0] * SUB[1]} forward transforms) per sample, oracle.grid fp64")
+    pairs = 2 * r * c - r - c
+    desc = (f"{r}x{c} corner of the {cfg['name']} grid ({pairs} pairs, "
+            f"{r * c} forward transforms) per sample, oracle.grid fp64")
     return g, pairs, desc
 
 

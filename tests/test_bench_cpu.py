@@ -26,4 +26,5 @@ def test_reference_arm_json_line():
     assert line["e2e"]["h2d_bytes_per_step"] == 0 and line["e2e"]["d2h_bytes_per_step"] == 0
     cb = line["cpu_baseline"]
     assert cb["kind"] == "oracle" and cb["cores"] >= 1 and cb["value"] == line["value"]
-    assert "4x5 corner" in cb["sample"]
+    r, c = bench.sub_grid()
+    assert f"{r}x{c} corner" in cb["sample"] and f"{2 * r * c - r - c} pairs" in cb["sample"]
