@@ -83,31 +83,3 @@ __device__ __forceinline__ void bulk_wait_read_all() {
 }
 
 }  // namespace stitch
-
-namespace stitch {
-
-// 2-D TMA tile load (cp.async.bulk.tensor, SASS UTMALDG): box at element coordinates
-// (x = innermost, y) of the tensor described by `map` (a __grid_constant__ CUtensorMap
-// kernel parameter) into shared memory, completing its bytes on `bar`.
-__device__ __forceinline__ void tma_load_2d(void* dst_smem, const void* map, int x, int y,
-                                            uint64_t* bar) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes"
-        " [%0], [%1, {%2, %3}], [%4];" ::"r"(smem_u32(dst_smem)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(x), "r"(y), "r"(smem_u32(bar))
-        : "memory");
-}
-
-// 2-D TMA prefetch of a box into L2 only (no shared memory, no completion tracking).
-__device__ __forceinline__ void tma_prefetch_l2_2d(const void* map, int x, int y) {
-    asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(
-                     reinterpret_cast<uint64_t>(map)),
-                 "r"(x), "r"(y)
-                 : "memory");
-}
-
-__device__ __forceinline__ void prefetch_tensormap(const void* map) {
-    asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(map)) : "memory");
-}
-
-}  // namespace stitch

@@ -31,7 +31,6 @@
 //   K5 ccf_mom    raw -> mom    integer moments of the 4 candidate overlaps (step 6, Fig. 3)
 //   K6 finalize   mom -> pairs  CCF in fp64 from exact int128 moments, candidate selection (step 7)
 #pragma once
-#include <cuda.h>
 #include <cuda_runtime.h>
 #include <math.h>
 #include <stdint.h>

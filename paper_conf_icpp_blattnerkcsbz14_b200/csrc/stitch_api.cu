@@ -13,9 +13,7 @@
 //     two kinds so that slots are recycled by reference count (the paper's pool);
 //   * multi-rank: an optional in-library NCCL halo exchange (libnccl.so.2 loaded at run time) on
 //     its own stream, overlapped with the interior pairs.
-#include <cuda.h>
 #include <cuda_runtime.h>
-#include <cudaTypedefs.h>
 #include <dlfcn.h>
 #include <nccl.h>   // types only: the functions are resolved with dlsym (no link-time NCCL)
 
