@@ -18,6 +18,8 @@ timeout 900 python bench.py --pool 160 --steps 5 --warmup 2 --no-cpu-baseline > 
 timeout 900 python bench.py --config 4 --ts-grids 24 --warmup 2 > gpurun_out/${TAG}_config4.json 2>&1
 timeout 900 python bench.py --config 2 --steps 20 --warmup 5 --no-cpu-baseline > gpurun_out/${TAG}_config2.json 2>&1
 timeout 900 python bench.py --compose --steps 5 --warmup 2 --no-cpu-baseline > gpurun_out/${TAG}_compose.json 2>&1
+timeout 900 python bench.py --config 5 --steps 5 --warmup 2 --no-cpu-baseline --e2e-steps 1 > gpurun_out/${TAG}_config5.json 2>&1
+timeout 900 python bench.py --config 5 --pool 480 --steps 3 --warmup 1 --no-cpu-baseline --e2e-steps 1 > gpurun_out/${TAG}_config5_pool.json 2>&1
 LAUNCHES=1 WARM=1 TAG=$TAG KERNELS="$KS" bash tools/ncu_profile.sh > /dev/null 2>&1
 python tools/launch_shares.py gpurun_out/${TAG}_launches.csv > gpurun_out/${TAG}_launch_shares.txt 2>&1
 for k in $KS; do
