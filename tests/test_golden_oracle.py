@@ -47,7 +47,8 @@ def test_golden_is_complete_and_reproduced_by_the_oracle(name):
     rng = np.random.default_rng(len(name))
     r = int(rng.integers(1, n))
     g = render(p, rows=(r - 1, r + 1))           # rows r-1, r only
-    for c in sorted({1, int(rng.integers(1, m)), m - 1}):
+    cols = {1, int(rng.integers(1, m)), m - 1} if p["H"] * p["W"] < 500_000 else {int(rng.integers(1, m))}
+    for c in sorted(cols):
         for kind, gold in (("w", west), ("n", north)):
             A = g.tiles[1, c - 1] if kind == "w" else g.tiles[0, c]
             got = oracle.pciam(A, g.tiles[1, c])
