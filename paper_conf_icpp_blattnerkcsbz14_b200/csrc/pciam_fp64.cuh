@@ -78,6 +78,84 @@ struct Plan64 {
                   "fp64 shared memory");
 };
 
+// Prime-factor (Good-Thomas) two-stage transform of L lines of length N = R0 R1 (coprime) by a
+// CTA, for D4's rows (696 = 29 x 24): no stage-2 twiddles (in double each was a complex multiply
+// plus a 16-byte twiddle load), only index maps --
+//   stage 1 (radix R0, butterfly b < R1):  element a at n = (R0 b + R1 a) mod N -> exchange (a, b)
+//   stage 2 (radix R1, butterfly k1 < R0): reads (k1, j), output j at n = (C1 k1 + C2 j) mod N.
+// IN_PLACE: the source is the exchange buffer (every stage-1 input is loaded before a barrier).
+// SLOT_OUT: stage 2 writes its outputs back into the slots it read (conflict-free, in place);
+// Z[q] is then at exchange (q mod R0, q mod R1) (CRT) -- D1's R2C post-pass reads it there.
+template <class RX, int SIGN, int L, int T, class C = double2>
+struct FftRunPfa;
+template <int N, int R0, int R1, int SIGN, int L, int T, class C>
+struct FftRunPfa<Radix<N, R0, R1>, SIGN, L, T, C> {
+    static constexpr bool OK = gcd_c(R0, R1) == 1;
+    static constexpr int C1 = (R1 * modinv(R1 % R0, R0)) % N;
+    static constexpr int C2 = (R0 * modinv(R0 % R1, R1)) % N;
+    template <bool IN_PLACE, bool SLOT_OUT = false, class Src, class Xc, class Dst>
+    static __device__ __forceinline__ void run(const Src& src, const Xc& xc, Dst& dst) {
+        {
+            constexpr int TOTAL = L * R1;
+            constexpr int ITER = (TOTAL + T - 1) / T;
+            C v[ITER][R0];
+#pragma unroll
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    const int line = g / R1, b = g - line * R1;
+                    int n = R0 * b;
+#pragma unroll
+                    for (int a = 0; a < R0; ++a) {
+                        v[it][a] = src.load(line, n);
+                        n += R1;
+                        if (n >= N) n -= N;
+                    }
+                }
+            }
+            if constexpr (IN_PLACE) __syncthreads();
+#pragma unroll
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    const int line = g / R1, b = g - line * R1;
+                    Dft<R0, SIGN>::run(v[it]);
+#pragma unroll
+                    for (int a = 0; a < R0; ++a) xc.at(line, a, b) = v[it][a];
+                }
+            }
+        }
+        __syncthreads();
+        {
+            constexpr int TOTAL = L * R0;
+            constexpr int ITER = (TOTAL + T - 1) / T;
+#pragma unroll 1
+            for (int it = 0; it < ITER; ++it) {
+                const int g = threadIdx.x + it * T;
+                if (TOTAL % T == 0 || g < TOTAL) {
+                    const int line = g / R0, k1 = g - line * R0;
+                    C v[R1];
+#pragma unroll
+                    for (int j = 0; j < R1; ++j) v[j] = xc.at(line, k1, j);
+                    Dft<R1, SIGN>::run(v);
+                    if constexpr (SLOT_OUT) {
+#pragma unroll
+                        for (int j = 0; j < R1; ++j) xc.at(line, k1, j) = v[j];
+                    } else {
+                        int n = (C1 * k1) % N;
+#pragma unroll
+                        for (int j = 0; j < R1; ++j) {
+                            dst.store(line, n, v[j]);
+                            n += C2;
+                            if (n >= N) n -= N;
+                        }
+                    }
+                }
+            }
+        }
+    }
+};
+
 // ------------------------------------------------------------------ D1 ----
 template <class PL>
 struct U16RowSrcD {  // z[n] = x[2n] + i x[2n+1] (exact in double)
@@ -130,12 +208,30 @@ __global__ void __launch_bounds__(PL::ROW_T) d1_fwd_rows(const uint16_t* __restr
     const int y0 = blockIdx.x * L;
     U16RowSrcD<PL> src{reinterpret_cast<const uint32_t*>(raw + (t * PL::H + y0) * PL::W)};
     typename P64::RowX xc{reinterpret_cast<double2*>(smem64)};
-    FftRun<typename P64::Row, -1, L, T, RowMap, false, double2>::run(src, xc, xc, tw2);
-    __syncthreads();
+    using RI = typename P64::RI;
+    if constexpr (RI::STAGES == 2 && gcd_c(RI::R0, RI::R1) == 1) {
+        // prime-factor transform, outputs left in their slots: Z[q] at (q mod R0, q mod R1)
+        FftRunPfa<typename P64::Row, -1, L, T>::template run<false, true>(src, xc, xc);
+        __syncthreads();
+        struct {
+            typename P64::RowX x;
+            __device__ __forceinline__ double2 nat(int line, int q) const {
+                return x.at(line, q % RI::R0, q % RI::R1);
+            }
+        } z{xc};
 #pragma unroll 1
-    for (int line = 0; line < L; ++line)
-        r2c_post_line_d<PL>(xc, line, GRowD<PL>{G + (size_t)blockIdx.y * PL::H * PL::WP, y0 + line},
-                            twW);
+        for (int line = 0; line < L; ++line)
+            r2c_post_line_d<PL>(z, line, GRowD<PL>{G + (size_t)blockIdx.y * PL::H * PL::WP, y0 + line},
+                                twW);
+    } else {
+        FftRun<typename P64::Row, -1, L, T, RowMap, false, double2>::run(src, xc, xc, tw2);
+        __syncthreads();
+#pragma unroll 1
+        for (int line = 0; line < L; ++line)
+            r2c_post_line_d<PL>(xc, line, GRowD<PL>{G + (size_t)blockIdx.y * PL::H * PL::WP,
+                                                    y0 + line},
+                                twW);
+    }
 }
 
 // ------------------------------------------------------------------ D2 ----
@@ -276,77 +372,6 @@ struct ArgmaxDstD {  // step 5 in double: running (max |x|, smallest index at th
         const uint32_t idx = (uint32_t)((row_base + line) * W + 2 * n);
         take(fabs(v.x), idx);
         take(fabs(v.y), idx + 1);
-    }
-};
-
-// Prime-factor (Good-Thomas) two-stage transform of L lines of length N = R0 R1 (coprime) by a
-// CTA, for D4's rows (696 = 29 x 24): no stage-2 twiddles (in double each was a complex multiply
-// plus a 16-byte twiddle load), only index maps --
-//   stage 1 (radix R0, butterfly b < R1):  element a at n = (R0 b + R1 a) mod N -> exchange (a, b)
-//   stage 2 (radix R1, butterfly k1 < R0): reads (k1, j), output j at n = (C1 k1 + C2 j) mod N.
-// IN_PLACE: the source is the exchange buffer (every stage-1 input is loaded before a barrier).
-template <class RX, int SIGN, int L, int T, class C = double2>
-struct FftRunPfa;
-template <int N, int R0, int R1, int SIGN, int L, int T, class C>
-struct FftRunPfa<Radix<N, R0, R1>, SIGN, L, T, C> {
-    static constexpr bool OK = gcd_c(R0, R1) == 1;
-    static constexpr int C1 = (R1 * modinv(R1 % R0, R0)) % N;
-    static constexpr int C2 = (R0 * modinv(R0 % R1, R1)) % N;
-    template <bool IN_PLACE, class Src, class Xc, class Dst>
-    static __device__ __forceinline__ void run(const Src& src, const Xc& xc, Dst& dst) {
-        {
-            constexpr int TOTAL = L * R1;
-            constexpr int ITER = (TOTAL + T - 1) / T;
-            C v[ITER][R0];
-#pragma unroll
-            for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
-                if (TOTAL % T == 0 || g < TOTAL) {
-                    const int line = g / R1, b = g - line * R1;
-                    int n = R0 * b;
-#pragma unroll
-                    for (int a = 0; a < R0; ++a) {
-                        v[it][a] = src.load(line, n);
-                        n += R1;
-                        if (n >= N) n -= N;
-                    }
-                }
-            }
-            if constexpr (IN_PLACE) __syncthreads();
-#pragma unroll
-            for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
-                if (TOTAL % T == 0 || g < TOTAL) {
-                    const int line = g / R1, b = g - line * R1;
-                    Dft<R0, SIGN>::run(v[it]);
-#pragma unroll
-                    for (int a = 0; a < R0; ++a) xc.at(line, a, b) = v[it][a];
-                }
-            }
-        }
-        __syncthreads();
-        {
-            constexpr int TOTAL = L * R0;
-            constexpr int ITER = (TOTAL + T - 1) / T;
-#pragma unroll 1
-            for (int it = 0; it < ITER; ++it) {
-                const int g = threadIdx.x + it * T;
-                if (TOTAL % T == 0 || g < TOTAL) {
-                    const int line = g / R0, k1 = g - line * R0;
-                    C v[R1];
-#pragma unroll
-                    for (int j = 0; j < R1; ++j) v[j] = xc.at(line, k1, j);
-                    Dft<R1, SIGN>::run(v);
-                    int n = (C1 * k1) % N;
-#pragma unroll
-                    for (int j = 0; j < R1; ++j) {
-                        dst.store(line, n, v[j]);
-                        n += C2;
-                        if (n >= N) n -= N;
-                    }
-                }
-            }
-        }
     }
 };
 
