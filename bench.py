@@ -474,10 +474,10 @@ def main():
         "k5_ccf_moments": 2 * T,       # the four candidate overlaps of A and B (HW pixels each)
         "k6_finalize": 8 + 160 + 64}
     if args.precision == "f64":
-        # fp64 path (D1..D4, pciam_fp64.cuh): complex intermediates are 2S, the resident
-        # unit phasor is 2S (double2 per bin); D4's per-block argmax partials are ~0
-        alg_bytes_per_unit.update({"k1_fwd_rows": T + 2 * S, "k2_fwd_cols": 4 * S,
-                                   "k3_pair_cols": 6 * S, "k4_pair_rows": 2 * S})
+        # fp64 path (D1..D4, pciam_fp64.cuh): complex intermediates are 2S (complex128), the
+        # resident unit phasor is S (Q31, 8 B per bin); D4's per-block argmax partials are ~0
+        alg_bytes_per_unit.update({"k1_fwd_rows": T + 2 * S, "k2_fwd_cols": 3 * S,
+                                   "k3_pair_cols": 4 * S, "k4_pair_rows": 2 * S})
     kd = kt_sum[dom]
     nsteps_k = max(1, min(args.steps, 5))
     fwd_tiles = (e - b) if bp.use_exchange else (e - halo)   # halo received or recomputed
@@ -621,7 +621,8 @@ def main():
             "vs_baseline_ref": "BASELINE.md: paper Pipelined-GPU 1x C2070, 42x59 in 49.7 s "
                                "(Table II, P:L1208) = 97.7 pairs/s; other hardware, end to end "
                                "incl. TIFF reads",
-            "dtype": ("f64" if args.precision == "f64" else "f32 (Q15 resident phasor)"),
+            "dtype": ("f64 (Q31 resident phasor)" if args.precision == "f64"
+                      else "f32 (Q15 resident phasor)"),
             "data": "synthetic",
             "config": conf,
             "roofline": roofline,

@@ -238,7 +238,7 @@ stitch_status stitch_debug_spectrum(stitch_ctx* ctx, int32_t tile, float* host_o
  * Test hook of the fp64 path (precision = 1): tile t's complex
  * half spectrum F(ky, kx) (step 2; "double complex") as
  * [H][W/2+1][2] doubles, recomputed by the same fp64 forward kernels.  The
- * context's resident store holds F/|F| (the only part step 3 uses).
+ * context's resident store holds F/|F| in Q31 fixed point (the only part step 3 uses).
  * Synchronous.  STITCH_ERR_STATE on an fp32 context.
  */
 stitch_status stitch_debug_spectrum_f64(stitch_ctx* ctx, int32_t tile, double* host_out);

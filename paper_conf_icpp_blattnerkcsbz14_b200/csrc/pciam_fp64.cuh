@@ -48,10 +48,10 @@ struct Plan64 {
     using ColX = ColXchg<CI::R0, CI::R1, PL::COL_PAD, COL_P, double2>;
     static constexpr size_t COL_XCH =
         CI::STAGES == 1 ? 16 : sizeof(double2) * COL_P * CI::R1 * (CI::R0 + PL::COL_PAD);
-    // column pitch of the column-major unit phasor U (double2): >= H, 2 mod 8, so the 16-byte
-    // loads of a landed 4-column panel (8 lanes per wavefront: 4 columns x 2 rows) are
-    // bank-conflict-free
-    static constexpr int HP64 = H % 8 <= 2 ? H + (2 - H % 8) : H + (10 - H % 8);
+    // column pitch of the column-major Q31 unit phasor U (int2, 8 bytes per bin): >= H and
+    // 8 mod 16, so the 8-byte loads of a landed 2-column panel (16 lanes per wavefront: 2
+    // columns x 8 rows) are bank-conflict-free (and every column run is 16-byte aligned)
+    static constexpr int HP64 = H % 16 <= 8 ? H + (8 - H % 16) : H + (24 - H % 16);
     static constexpr size_t PANEL_G = sizeof(double2) * COL_P * H;      // D2's landed Gd panel
     static constexpr size_t D2_SMEM = (PANEL_G > COL_XCH ? PANEL_G : COL_XCH);
     // D3 takes 2-column panels of U (any column run of the column-major U is contiguous): two
@@ -66,7 +66,7 @@ struct Plan64 {
     using ColX3 = ColXchg<CI::R0, CI::R1, PL::COL_PAD, COL_P3, double2>;
     static constexpr size_t COL_XCH3 =
         CI::STAGES == 1 ? 16 : sizeof(double2) * COL_P3 * CI::R1 * (CI::R0 + PL::COL_PAD);
-    static constexpr size_t PANEL_U = sizeof(double2) * COL_P3 * HP64;  // one tile's U panel
+    static constexpr size_t PANEL_U = sizeof(int2) * COL_P3 * HP64;     // one tile's U panel
     static constexpr size_t U_B_OFF = (PANEL_U + 127) / 128 * 128;      // D3's second panel
     static constexpr size_t D3_SMEM =
         (U_B_OFF + PANEL_U > COL_XCH3 ? U_B_OFF + PANEL_U : COL_XCH3);
@@ -246,13 +246,18 @@ struct PanelIOD {  // a panel of columns of one [H][WP] double2 array
     }
 };
 
+// The fp64 path's resident spectrum: the unit phasor U = F/|F| (0 where F = 0, reading C4) in
+// Q31 fixed point, round(S Re U), round(S Im U) with S = 2^31 - 1 (per-component error <= 2^-32 of
+// the unit circle, reading C11-f2), column-major.  D3 forms U_A conj(U_B) exactly in int64.
+constexpr double Q31_S = 2147483647.0;
 template <class PL>
-struct UnitDst {  // spectrum: U = F/|F|, 0 where F = 0 (reading C4), column-major panel
-    double2* p;
+struct UnitDst {
+    int2* p;
     __device__ __forceinline__ void store(int line, int n, double2 v) const {
         const double m2 = fma(v.x, v.x, v.y * v.y);
-        const double r = m2 > 0.0 ? rsqrt(m2) : 0.0;
-        p[(size_t)line * Plan64<PL>::HP64 + n] = make_double2(v.x * r, v.y * r);
+        const double r = m2 > 0.0 ? rsqrt(m2) * Q31_S : 0.0;
+        p[(size_t)line * Plan64<PL>::HP64 + n] =
+            make_int2(__double2int_rn(v.x * r), __double2int_rn(v.y * r));
     }
 };
 
@@ -270,7 +275,7 @@ struct LandSrcD {  // a landed Gd panel [H][COL_P] in shared memory
 // two 5-warp CTAs per SM (register-budgeted by the launch bounds)
 template <class PL, bool UNIT_OUT>
 __global__ void __launch_bounds__(Plan64<PL>::COL_T, 2) d2_fwd_cols(const double2* __restrict__ G,
-                                                                 double2* __restrict__ U,
+                                                                 int2* __restrict__ U,
                                                                  double2* __restrict__ out,
                                                                  int tile0,
                                                                  const double2* __restrict__ tw2) {
@@ -302,17 +307,21 @@ __global__ void __launch_bounds__(Plan64<PL>::COL_T, 2) d2_fwd_cols(const double
 
 // ------------------------------------------------------------------ D3 ----
 template <class PL>
-struct NcpsUnitSrc {  // step 3: U_A conj(U_B) = F_A conj(F_B) / |F_A conj(F_B)| (0 if either is 0)
-    const double2* a;  // landed column-major panels [COL_P][HP64]
-    const double2* b;
+struct NcpsUnitSrc {  // step 3: U_A conj(U_B) = F_A conj(F_B) / |F_A conj(F_B)| (x S^2; 0 if either is 0)
+    const int2* a;     // landed column-major Q31 panels [COL_P3][HP64]
+    const int2* b;
     __device__ __forceinline__ double2 load(int line, int n) const {
         const int o = line * Plan64<PL>::HP64 + n;
-        return cmulc(a[o], b[o]);
+        const int2 ua = a[o], ub = b[o];
+        // exact in int64: |.| <= |U_A| |U_B| S^2 < 2^62
+        const long long re = (long long)ua.x * ub.x + (long long)ua.y * ub.y;
+        const long long im = (long long)ua.y * ub.x - (long long)ua.x * ub.y;
+        return make_double2((double)re, (double)im);
     }
 };
 
 template <class PL>
-__global__ void __launch_bounds__(Plan64<PL>::COL_T3, 2) d3_pair_cols(const double2* __restrict__ U,
+__global__ void __launch_bounds__(Plan64<PL>::COL_T3, 3) d3_pair_cols(const int2* __restrict__ U,
                                                                   double2* __restrict__ Q,
                                                                   const PairIdx* __restrict__ pairs,
                                                                   int pair0,
@@ -322,8 +331,8 @@ __global__ void __launch_bounds__(Plan64<PL>::COL_T3, 2) d3_pair_cols(const doub
     __shared__ uint64_t bar;
     const PairIdx pr = pairs[pair0 + blockIdx.y];
     const int c0 = blockIdx.x * P64::COL_P3;
-    double2* la = reinterpret_cast<double2*>(smem64);
-    double2* lb = reinterpret_cast<double2*>(smem64 + P64::U_B_OFF);
+    int2* la = reinterpret_cast<int2*>(smem64);
+    int2* lb = reinterpret_cast<int2*>(smem64 + P64::U_B_OFF);
     if (threadIdx.x == 0) {
         mbar_init(&bar, 1);
         fence_mbar_init();

@@ -68,8 +68,8 @@ struct PlanOps {
     int nblk64;
     cudaError_t (*d_setup)();
     void (*d1)(const uint16_t*, double2*, int, int, const double2*, const double2*, cudaStream_t);
-    void (*d2)(const double2*, double2*, double2*, int, int, const double2*, bool, cudaStream_t);
-    void (*d3)(const double2*, double2*, const PairIdx*, int, int, const double2*, cudaStream_t);
+    void (*d2)(const double2*, int2*, double2*, int, int, const double2*, bool, cudaStream_t);
+    void (*d3)(const int2*, double2*, const PairIdx*, int, int, const double2*, cudaStream_t);
     void (*d4)(const double2*, double*, uint32_t*, int, int, const double2*, const double2*,
                cudaStream_t);
 };
@@ -210,7 +210,7 @@ void launch_d1(const uint16_t* raw, double2* G, int t0, int nt, const double2* t
     d1_fwd_rows<PL><<<dim3(P64::NBLK, nt), P64::ROW_T, P64::ROW_SMEM, s>>>(raw, G, t0, tw2, twW);
 }
 template <class PL>
-void launch_d2(const double2* G, double2* U, double2* out, int t0, int nt, const double2* tw2,
+void launch_d2(const double2* G, int2* U, double2* out, int t0, int nt, const double2* tw2,
                bool unit_out, cudaStream_t s) {
     using P64 = Plan64<PL>;
     const dim3 grid(PL::WP / P64::COL_P, nt);
@@ -220,7 +220,7 @@ void launch_d2(const double2* G, double2* U, double2* out, int t0, int nt, const
         d2_fwd_cols<PL, false><<<grid, P64::COL_T, P64::D2_SMEM, s>>>(G, U, out, t0, tw2);
 }
 template <class PL>
-void launch_d3(const double2* U, double2* Q, const PairIdx* pairs, int p0, int np,
+void launch_d3(const int2* U, double2* Q, const PairIdx* pairs, int p0, int np,
                const double2* tw2, cudaStream_t s) {
     using P64 = Plan64<PL>;
     d3_pair_cols<PL><<<dim3(PL::WP / P64::COL_P3, np), P64::COL_T3, P64::D3_SMEM, s>>>(U, Q, pairs,
@@ -379,7 +379,7 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     // spectrum by slot: u32 Q15 unit phasor [WP][HP] (fp32) or double2 unit phasor [H][WP] (fp64)
-    L->spec_tile_bytes = L->prec ? (size_t)ops->HP64 * WP * sizeof(double2)
+    L->spec_tile_bytes = L->prec ? (size_t)ops->HP64 * WP * sizeof(int2)
                                  : (size_t)ops->HP * WP * sizeof(uint32_t);
     const size_t cplx = L->prec ? sizeof(double2) : sizeof(float2);
     const size_t np1 = (size_t)(np > 0 ? np : 1);
@@ -462,7 +462,8 @@ struct stitch_ctx {
     float2 *G, *Q, *twM, *twH, *twW;  // chunk intermediates, twiddles
     int32_t* fslot;                   // slot of each local tile
     int prec = 0;                     // 1: fp64 path (f2): the buffers below are used instead
-    double2 *Gd = nullptr, *Qd = nullptr, *Ud = nullptr;   // Ud: resident unit phasors
+    double2 *Gd = nullptr, *Qd = nullptr;
+    int2* Ud = nullptr;               // resident Q31 unit phasors (fp64 path)
     double2 *twMd = nullptr, *twHd = nullptr, *twWd = nullptr;
     double* part_v = nullptr;         // fp64 argmax partials [pairs][nblk64]
     uint32_t* part_i = nullptr;
@@ -958,7 +959,7 @@ static stitch_status enqueue_ops(stitch_ctx* ctx, const std::vector<Op>& ops, co
             // the key's value is max |c| (fp64 path) or max |c| x 32767^2 (Q15 phasor NCPS)
             k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
                 ctx->keys + pa, ctx->mom + pa * 20, ctx->res + pa, ctx->H, ctx->W, (int)np,
-                (double)ctx->W * ctx->H * (ctx->prec ? 1.0 : NCPS_Q15_SCALE));
+                (double)ctx->W * ctx->H * (ctx->prec ? Q31_S * Q31_S : NCPS_Q15_SCALE));
         });
         mark(ctx, 5);
         ctx->launches += 1;
@@ -1294,7 +1295,7 @@ stitch_status stitch_init(const stitch_config* cfg, stitch_ctx** out) {
     ctx->twW = ctx->twH + tw_col(ops);
     ctx->fslot = (int32_t*)(b + L.off_fslot);
     if (ctx->prec) {
-        ctx->Ud = (double2*)(b + L.off_spec);
+        ctx->Ud = (int2*)(b + L.off_spec);
         ctx->Gd = (double2*)(b + L.off_g);
         ctx->Qd = (double2*)(b + L.off_q);
         ctx->twMd = (double2*)(b + L.off_tw);

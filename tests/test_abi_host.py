@@ -92,7 +92,7 @@ def test_fp64_workspace_and_precision_validation(lib):
     ws = pkg.workspace_size(cfg)
     H, W, WP = 1040, 1392, 704
     raw = 2478 * H * W * 2
-    spec = 2478 * WP * 1042 * 16      # resident unit phasors (double2), column pitch 1042
+    spec = 2478 * WP * 1048 * 8       # resident Q31 unit phasors (int2), column pitch 1048
     chunks = 2 * 8 * H * WP * 16      # Gd + Qd
     part = 4855 * (H // 4) * 12       # (double, u32) per pair and 4-row block
     assert raw + spec + chunks + part < ws < raw + spec + chunks + part + 5 * 2**20
