@@ -351,6 +351,121 @@ __global__ void __launch_bounds__(Plan64<PL>::COL_T3, 3) d3_pair_cols(const int2
         true>(src, xc, dst, tw2);
 }
 
+// D3 as a three-factor prime-factor (Good-Thomas) column transform where H splits into three
+// pairwise coprime radices with codelets (1040 = 16 x 5 x 13): no twiddles at all, and butterflies
+// of at most 16 points -- ~90 registers instead of the radix-40 butterfly's 168-222 -- so four
+// 5-warp CTAs share an SM.  With N = A B C, element (a, b, c) of the 3-D array is
+//   input  n = (a N/A + b N/B + c N/C) mod N          (the Ruritanian map)
+//   output k = (ka e_A + kb e_B + kc e_C) mod N,  e_X = (N/X) ((N/X)^-1 mod X)   (CRT)
+// and the transform is three passes of 1-D DFTs along c (radix C), a (radix A), b (radix B).
+// Pass 1 reads U_A conj(U_B) straight from the landed Q31 panels (lanes walk a: input stride
+// N/A = 65 = 1 mod 16 banks) into registers, then -- after a barrier -- writes the work buffer,
+// which reuses the landing; passes 2-3 work in place; pass 3 writes Q at the CRT index.
+template <int H> struct Pfa3 {   // no three-factor split with codelets: the two-stage D3 runs
+    static constexpr bool OK = false;
+    static constexpr int A = 1, B = 1, C = 1;
+};
+template <> struct Pfa3<1040> {
+    static constexpr bool OK = true;
+    static constexpr int A = 16, B = 5, C = 13;
+};
+
+template <class PL>
+struct D3P {
+    using F = Pfa3<PL::H>;
+    static constexpr int A = F::A, B = F::B, C = F::C, N = PL::H;
+    static constexpr int P = 2;                                   // columns per CTA
+    static constexpr int T = 160;
+    static constexpr int SA = N / A, SB = N / B, SC = N / C;      // input-map strides
+    static constexpr int EA = SA * modinv(SA % A, A) % N;         // CRT output weights
+    static constexpr int EB = SB * modinv(SB % B, B) % N;
+    static constexpr int EC = SC * modinv(SC % C, C) % N;
+    static constexpr int CS = N + 4;                              // work-buffer column stride (16 B units)
+    static constexpr size_t WORK = sizeof(double2) * P * CS;
+    static constexpr size_t PANEL_U = sizeof(int2) * P * Plan64<PL>::HP64;
+    static constexpr size_t U_B_OFF = (PANEL_U + 127) / 128 * 128;
+    static constexpr size_t SMEM = U_B_OFF + PANEL_U > WORK ? U_B_OFF + PANEL_U : WORK;
+    static_assert(!F::OK || (A * B * C == N && P * A * B == T), "pass 1: one butterfly per thread");
+    // work element (col, a, b, c)
+    static __device__ __forceinline__ int w(int col, int a, int b, int c) {
+        return col * CS + (a * B + b) * C + c;
+    }
+};
+
+template <class PL>
+__global__ void __launch_bounds__(D3P<PL>::T, 4) d3p_pair_cols(const int2* __restrict__ U,
+                                                               double2* __restrict__ Q,
+                                                               const PairIdx* __restrict__ pairs,
+                                                               int pair0) {
+    using S = D3P<PL>;
+    using P64 = Plan64<PL>;
+    constexpr int A = S::A, B = S::B, C = S::C, N = S::N;
+    extern __shared__ __align__(128) unsigned char smem64[];
+    __shared__ uint64_t bar;
+    const PairIdx pr = pairs[pair0 + blockIdx.y];
+    const int c0 = blockIdx.x * S::P;
+    int2* la = reinterpret_cast<int2*>(smem64);
+    int2* lb = reinterpret_cast<int2*>(smem64 + S::U_B_OFF);
+    double2* wk = reinterpret_cast<double2*>(smem64);   // reuses the landing after pass 1's loads
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {   // each tile's 2-column run of the column-major U: one bulk copy each
+        mbar_arrive_expect_tx(&bar, 2 * (uint32_t)S::PANEL_U);
+        bulk_g2s(la, U + ((size_t)pr.a * PL::WP + c0) * P64::HP64, (uint32_t)S::PANEL_U, &bar);
+        bulk_g2s(lb, U + ((size_t)pr.b * PL::WP + c0) * P64::HP64, (uint32_t)S::PANEL_U, &bar);
+    }
+    mbar_wait(&bar, 0);
+    const int t = threadIdx.x;
+    {   // pass 1: radix C along c; butterfly (col, a, b) = thread, lanes walk a
+        const int a = t % A, col = (t / A) % S::P, b = t / (A * S::P);
+        NcpsUnitSrc<PL> src{la, lb};
+        double2 v[C];
+        int n = (a * S::SA + b * S::SB) % N;
+#pragma unroll
+        for (int c = 0; c < C; ++c) {
+            v[c] = src.load(col, n);
+            n += S::SC;
+            if (n >= N) n -= N;
+        }
+        __syncthreads();   // every landed value is in registers: the buffer becomes the work array
+        Dft<C, +1>::run(v);
+#pragma unroll
+        for (int c = 0; c < C; ++c) wk[S::w(col, a, b, c)] = v[c];
+    }
+    __syncthreads();
+    // pass 2: radix A along a; butterflies (col, b, kc), lanes walk kc
+    for (int g = t; g < S::P * B * C; g += S::T) {
+        const int kc = g % C, b = (g / C) % B, col = g / (B * C);
+        double2 v[A];
+#pragma unroll
+        for (int a = 0; a < A; ++a) v[a] = wk[S::w(col, a, b, kc)];
+        Dft<A, +1>::run(v);
+#pragma unroll
+        for (int a = 0; a < A; ++a) wk[S::w(col, a, b, kc)] = v[a];
+    }
+    __syncthreads();
+    // pass 3: radix B along b; butterflies (col, ka, kc), lanes walk col then kc; output at the
+    // CRT index k of column c0 + col of this pair's Q (two adjacent lanes fill one 32-byte row run)
+    double2* q = Q + (size_t)blockIdx.y * PL::H * PL::WP + c0;
+    for (int g = t; g < S::P * A * C; g += S::T) {
+        const int col = g % S::P, kc = (g / S::P) % C, ka = g / (S::P * C);
+        double2 v[B];
+#pragma unroll
+        for (int b = 0; b < B; ++b) v[b] = wk[S::w(col, ka, b, kc)];
+        Dft<B, +1>::run(v);
+        int k = (ka * S::EA + kc * S::EC) % N;
+#pragma unroll
+        for (int kb = 0; kb < B; ++kb) {
+            q[(size_t)k * PL::WP + col] = v[kb];
+            k += S::EB;
+            if (k >= N) k -= N;
+        }
+    }
+}
+
 // ------------------------------------------------------------------ D4 ----
 template <class PL>
 struct C2RSrcD {  // complex-to-real pre-processing of row X[0..M] into Z[0..M) (as C2RSrc)

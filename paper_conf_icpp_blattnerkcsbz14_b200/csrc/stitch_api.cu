@@ -201,6 +201,7 @@ cudaError_t d_setup() {
     CKE(max_smem(d4_pair_rows<PL>, P64::D4_SMEM));
     CKE(max_smem(d2_fwd_cols<PL, true>, P64::D2_SMEM));
     CKE(max_smem(d2_fwd_cols<PL, false>, P64::D2_SMEM));
+    if constexpr (D3P<PL>::F::OK) CKE(max_smem(d3p_pair_cols<PL>, D3P<PL>::SMEM));
     return max_smem(d3_pair_cols<PL>, P64::D3_SMEM);
 }
 template <class PL>
@@ -223,6 +224,11 @@ template <class PL>
 void launch_d3(const int2* U, double2* Q, const PairIdx* pairs, int p0, int np,
                const double2* tw2, cudaStream_t s) {
     using P64 = Plan64<PL>;
+    if constexpr (D3P<PL>::F::OK) {   // three-factor prime-factor columns (1040 = 16 x 5 x 13)
+        using S3 = D3P<PL>;
+        d3p_pair_cols<PL><<<dim3(PL::WP / S3::P, np), S3::T, S3::SMEM, s>>>(U, Q, pairs, p0);
+        return;
+    }
     d3_pair_cols<PL><<<dim3(PL::WP / P64::COL_P3, np), P64::COL_T3, P64::D3_SMEM, s>>>(U, Q, pairs,
                                                                                       p0, tw2);
 }
