@@ -466,6 +466,119 @@ __global__ void __launch_bounds__(D3P<PL>::T, 4) d3p_pair_cols(const int2* __res
     }
 }
 
+// D2 on the same three-factor split (forward): a CTA takes one 4-column Gd panel (one bulk copy),
+// pass 1 (radix C) reads it with the Ruritanian input map into registers, passes 2-3 (radix A, B)
+// work in place on the work array that reuses the landing; pass 3 encodes the Q31 unit phasor at the
+// CRT index into a staging panel [4][HPS] (a conflict-free pitch), stored with one bulk copy per
+// column into the column-major U (or, UNIT_OUT = false, the complex spectrum row-major into `out`).
+template <class PL>
+struct D2P {
+    using F = Pfa3<PL::H>;
+    static constexpr int A = F::A, B = F::B, C = F::C, N = PL::H;
+    static constexpr int P = Plan64<PL>::COL_P;                  // 4 columns: one Gd panel
+    static constexpr int T = P * A * B;                           // pass 1: one butterfly each
+    static constexpr int SA = N / A, SB = N / B, SC = N / C;
+    static constexpr int EA = SA * modinv(SA % A, A) % N;
+    static constexpr int EB = SB * modinv(SB % B, B) % N;
+    static constexpr int EC = SC * modinv(SC % C, C) % N;
+    static constexpr int CS = N % 8 <= 2 ? N + (2 - N % 8) : N + (10 - N % 8);   // 2 mod 8
+    static constexpr int HPS = N % 16 <= 4 ? N + (4 - N % 16) : N + (20 - N % 16); // 4 mod 16
+    static constexpr size_t LAND = sizeof(double2) * P * N;
+    static constexpr size_t WORK = sizeof(double2) * P * CS;
+    static constexpr size_t STG_OFF = ((LAND > WORK ? LAND : WORK) + 127) / 128 * 128;
+    static constexpr size_t SMEM = STG_OFF + sizeof(int2) * P * HPS;
+    static __device__ __forceinline__ int w(int col, int a, int b, int c) {
+        return col * CS + (a * B + b) * C + c;
+    }
+};
+
+template <class PL, bool UNIT_OUT>
+__global__ void __launch_bounds__(D2P<PL>::T, 2) d2p_fwd_cols(const double2* __restrict__ G,
+                                                              int2* __restrict__ U,
+                                                              double2* __restrict__ out,
+                                                              int tile0) {
+    using S = D2P<PL>;
+    using P64 = Plan64<PL>;
+    constexpr int A = S::A, B = S::B, C = S::C, N = S::N, P = S::P;
+    extern __shared__ __align__(128) unsigned char smem64[];
+    __shared__ uint64_t bar;
+    const int tl = blockIdx.y, c0 = blockIdx.x * P;
+    const double2* land = reinterpret_cast<const double2*>(smem64);   // [n][P]
+    double2* wk = reinterpret_cast<double2*>(smem64);
+    int2* stage = reinterpret_cast<int2*>(smem64 + S::STG_OFF);
+    if (threadIdx.x == 0) {
+        mbar_init(&bar, 1);
+        fence_mbar_init();
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        mbar_arrive_expect_tx(&bar, (uint32_t)S::LAND);
+        bulk_g2s(smem64, G + ((size_t)tl * PL::WP + c0) * PL::H, (uint32_t)S::LAND, &bar);
+    }
+    mbar_wait(&bar, 0);
+    const int t = threadIdx.x;
+    {   // pass 1: radix C along c; butterfly (col, a, b) = thread, lanes walk col then a
+        const int col = t % P, a = (t / P) % A, b = t / (P * A);
+        double2 v[C];
+        int n = (a * S::SA + b * S::SB) % N;
+#pragma unroll
+        for (int c = 0; c < C; ++c) {
+            v[c] = land[n * P + col];
+            n += S::SC;
+            if (n >= N) n -= N;
+        }
+        __syncthreads();
+        Dft<C, -1>::run(v);
+#pragma unroll
+        for (int c = 0; c < C; ++c) wk[S::w(col, a, b, c)] = v[c];
+    }
+    __syncthreads();
+    for (int g = t; g < P * B * C; g += S::T) {   // pass 2: radix A along a
+        const int col = g % P, kc = (g / P) % C, b = g / (P * C);
+        double2 v[A];
+#pragma unroll
+        for (int a = 0; a < A; ++a) v[a] = wk[S::w(col, a, b, kc)];
+        Dft<A, -1>::run(v);
+#pragma unroll
+        for (int a = 0; a < A; ++a) wk[S::w(col, a, b, kc)] = v[a];
+    }
+    __syncthreads();
+    for (int g = t; g < P * A * C; g += S::T) {   // pass 3: radix B along b, CRT output
+        const int col = g % P, ka = (g / P) % A, kc = g / (P * A);
+        double2 v[B];
+#pragma unroll
+        for (int b = 0; b < B; ++b) v[b] = wk[S::w(col, ka, b, kc)];
+        Dft<B, -1>::run(v);
+        int k = (ka * S::EA + kc * S::EC) % N;
+#pragma unroll
+        for (int kb = 0; kb < B; ++kb) {
+            if constexpr (UNIT_OUT) {
+                const double2 x = v[kb];
+                const double m2 = fma(x.x, x.x, x.y * x.y);
+                const double r = m2 > 0.0 ? rsqrt(m2) * Q31_S : 0.0;
+                stage[col * S::HPS + k] = make_int2(__double2int_rn(x.x * r), __double2int_rn(x.y * r));
+            } else {
+                out[((size_t)tl * PL::H + k) * PL::WP + c0 + col] = v[kb];
+            }
+            k += S::EB;
+            if (k >= N) k -= N;
+        }
+    }
+    if constexpr (UNIT_OUT) {
+        fence_proxy_async();
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            int2* dst = U + ((size_t)(tile0 + tl) * PL::WP + c0) * P64::HP64;
+#pragma unroll
+            for (int col = 0; col < P; ++col)
+                bulk_s2g(dst + (size_t)col * P64::HP64, stage + col * S::HPS,
+                         (uint32_t)(sizeof(int2) * N));
+            bulk_commit();
+            bulk_wait_read_all();
+        }
+    }
+}
+
 // ------------------------------------------------------------------ D4 ----
 template <class PL>
 struct C2RSrcD {  // complex-to-real pre-processing of row X[0..M] into Z[0..M) (as C2RSrc)

@@ -201,7 +201,11 @@ cudaError_t d_setup() {
     CKE(max_smem(d4_pair_rows<PL>, P64::D4_SMEM));
     CKE(max_smem(d2_fwd_cols<PL, true>, P64::D2_SMEM));
     CKE(max_smem(d2_fwd_cols<PL, false>, P64::D2_SMEM));
-    if constexpr (D3P<PL>::F::OK) CKE(max_smem(d3p_pair_cols<PL>, D3P<PL>::SMEM));
+    if constexpr (D3P<PL>::F::OK) {
+        CKE(max_smem(d3p_pair_cols<PL>, D3P<PL>::SMEM));
+        CKE(max_smem(d2p_fwd_cols<PL, true>, D2P<PL>::SMEM));
+        CKE(max_smem(d2p_fwd_cols<PL, false>, D2P<PL>::SMEM));
+    }
     return max_smem(d3_pair_cols<PL>, P64::D3_SMEM);
 }
 template <class PL>
@@ -215,6 +219,14 @@ void launch_d2(const double2* G, int2* U, double2* out, int t0, int nt, const do
                bool unit_out, cudaStream_t s) {
     using P64 = Plan64<PL>;
     const dim3 grid(PL::WP / P64::COL_P, nt);
+    if constexpr (D2P<PL>::F::OK) {   // three-factor prime-factor columns (1040 = 16 x 5 x 13)
+        using S2 = D2P<PL>;
+        if (unit_out)
+            d2p_fwd_cols<PL, true><<<grid, S2::T, S2::SMEM, s>>>(G, U, out, t0);
+        else
+            d2p_fwd_cols<PL, false><<<grid, S2::T, S2::SMEM, s>>>(G, U, out, t0);
+        return;
+    }
     if (unit_out)
         d2_fwd_cols<PL, true><<<grid, P64::COL_T, P64::D2_SMEM, s>>>(G, U, out, t0, tw2);
     else
