@@ -37,6 +37,15 @@ __device__ __forceinline__ double2 cmulc(double2 a, double2 b) {
     return make_double2(fma(a.x, b.x, a.y * b.y), fma(a.y, b.x, -a.x * b.y));
 }
 
+// Modular inverse of a mod m and gcd, at compile time (prime-factor index maps).
+__host__ __device__ constexpr int modinv(int a, int m) {
+    int r = 1;
+    for (int x = 1; x < m; ++x)
+        if ((a * x) % m == 1) r = x;
+    return r;
+}
+__host__ __device__ constexpr int gcd_c(int a, int b) { return b == 0 ? a : gcd_c(b, a % b); }
+
 // Butterfly id g -> (line, b).  Row map: consecutive threads walk one line.
 struct RowMap {
     template <int NB, int L>

@@ -361,15 +361,6 @@ __global__ void __launch_bounds__(Plan64<PL>::COL_T3, 3) d3_pair_cols(const int2
 // Pass 1 reads U_A conj(U_B) straight from the landed Q31 panels (lanes walk a: input stride
 // N/A = 65 = 1 mod 16 banks) into registers, then -- after a barrier -- writes the work buffer,
 // which reuses the landing; passes 2-3 work in place; pass 3 writes Q at the CRT index.
-template <int H> struct Pfa3 {   // no three-factor split with codelets: the two-stage D3 runs
-    static constexpr bool OK = false;
-    static constexpr int A = 1, B = 1, C = 1;
-};
-template <> struct Pfa3<1040> {
-    static constexpr bool OK = true;
-    static constexpr int A = 16, B = 5, C = 13;
-};
-
 template <class PL>
 struct D3P {
     using F = Pfa3<PL::H>;

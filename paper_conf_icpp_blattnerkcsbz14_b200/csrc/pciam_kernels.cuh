@@ -354,6 +354,19 @@ __global__ void __launch_bounds__(PL::COL_T, PL::COL_MINB)
                                                                                          dst, tws);
 }
 
+// Column lengths with a three-factor prime-factor (Good-Thomas) split into pairwise coprime
+// radices that have codelets (1040 = 16 x 5 x 13): the fp64 three-pass column kernels (D2, D3)
+// need no twiddles and hold at most a 16-point butterfly in registers.
+template <int H> struct Pfa3 {   // no three-factor split with codelets: two-stage kernels run
+    static constexpr bool OK = false;
+    static constexpr int A = 1, B = 1, C = 1;
+};
+template <> struct Pfa3<1040> {
+    static constexpr bool OK = true;
+    static constexpr int A = 16, B = 5, C = 13;
+};
+
+
 // ------------------------------------------------------------------ K4 ----
 template <class PL>
 struct C2RSrc {  // complex-to-real pre-processing of row X[0..M] into Z[0..M)

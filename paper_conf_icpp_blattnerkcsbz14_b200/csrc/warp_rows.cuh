@@ -74,13 +74,6 @@ struct WarpFft2<Radix<N, R0, R1>, SIGN, PAD> {
 // (k1 < R0: the stage-2 butterfly, k2 < R1: its output).  The input map wraps once per
 // butterfly, at a lane-dependent a, so each load picks one of two base pointers; the
 // destination receives whole butterflies (store_pfa) and maps indices itself.
-__host__ __device__ constexpr int modinv(int a, int m) {
-    int r = 1;
-    for (int x = 1; x < m; ++x)
-        if ((a * x) % m == 1) r = x;
-    return r;
-}
-__host__ __device__ constexpr int gcd_c(int a, int b) { return b == 0 ? a : gcd_c(b, a % b); }
 
 template <class RX, int SIGN>
 struct WarpFftPfa;
