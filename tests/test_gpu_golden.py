@@ -45,13 +45,13 @@ def render(p):
     return synthgrid.make_grid(p["n"], p["m"], p["H"], p["W"], **kw)
 
 
-def run_case(name, expect_truth=True, min_ambiguous=0, results=None):
+def run_case(name, expect_truth=True, min_ambiguous=0, results=None, precision=0):
     p, ow, on, sha = load_case(name)
     g = render(p)
     assert hashlib.sha256(g.tiles.tobytes()).hexdigest() == sha, "generator drift"
     n, m = p["n"], p["m"]
     if results is None:
-        with PciamGrid(n, m, p["H"], p["W"], device=0) as pg:  # the bench's launch configuration
+        with PciamGrid(n, m, p["H"], p["W"], device=0, precision=precision) as pg:  # bench config
             pg.load_grid(g.tiles)
             west, north = pg.compute_translations()
             counts = pg.last_counts()
@@ -59,8 +59,8 @@ def run_case(name, expect_truth=True, min_ambiguous=0, results=None):
     else:
         west, north = results(g)
     stats = {}
-    amb = _parity.grid_parity(g.tiles, west, north, ow, on, stats)
-    print(f"{name}: {2 * n * m - n - m} pairs compared, {amb} near-tie pairs (C17) "
+    amb = _parity.grid_parity(g.tiles, west, north, ow, on, stats, fp64=precision == 1)
+    print(f"{name}{' fp64' if precision else ''}: {2 * n * m - n - m} pairs compared, {amb} near-tie pairs (C17) "
           f"{stats.get('near_tie', [])}, {stats.get('ccf_ties', 0)} CCF ties")
     assert amb >= min_ambiguous
     if expect_truth:   # property at any size: the generator's known shifts are recovered
@@ -117,3 +117,19 @@ def test_low_texture_256_near_ties():
 
 def test_low_texture_1392_near_ties():
     run_case("lowtex1392", expect_truth=False, min_ambiguous=1)
+
+
+# The fp64 path (row f2) on the same committed oracle results, with the fp64 bands
+# (_parity: near-tie margin 1e-9, peak height to float storage, CCF 1e-9).
+def test_fp64_config2_every_pair_matches_oracle():
+    run_case("cfg2", precision=1)
+
+
+@pytest.mark.slow
+def test_fp64_config3_headline_every_pair_matches_oracle():
+    run_case("cfg3", precision=1)
+
+
+def test_fp64_low_texture_near_ties():
+    run_case("lowtex256", expect_truth=False, precision=1)
+    run_case("lowtex1392", expect_truth=False, precision=1)
