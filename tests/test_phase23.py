@@ -1,15 +1,20 @@
 """NEXT rows f3 (phase 2: absolute positions) and f4 (phase 3: overlay composition).
 
-f3 is host code: pinned here on CPU against the generator's known tile origins, with the
-phase-1 translations taken from the oracle (reading C19: maximum
-spanning tree on CCF, positions = path sums).  f4 runs on the GPU and is compared with a
-plain numpy overlay (later tile on top, row-major order).
+f3 is host code (stitch_global_positions): checked here against the oracle's phase 2
+(oracle/phases.py: Prim's algorithm, where the product runs Kruskal's; PAPER.md L436-452,
+reading C19: maximum spanning tree on CCF, positions = path sums), which is itself pinned by
+brute-force enumeration of spanning forests on tiny grids, and against the generator's known
+tile origins.  f4 runs on the GPU (stitch_compose_overlay) and is compared with the oracle's
+overlay (later tile on top, row-major order), pinned per pixel.
 """
+import itertools
+
 import numpy as np
 import pytest
 
 import oracle
 import synthgrid
+from oracle import phases
 from paper_conf_icpp_blattnerkcsbz14_b200 import PAIR_DTYPE, global_positions
 
 
@@ -53,14 +58,116 @@ def test_global_positions_disconnected_components():
 
 
 def numpy_overlay(tiles, pos):
-    n, m, H, W = tiles.shape
     p = pos.reshape(-1, 2) - pos.reshape(-1, 2).min(axis=0)
-    cw, ch = p[:, 0].max() + W, p[:, 1].max() + H
-    canvas = np.zeros((ch, cw), np.uint16)
-    for t in range(n * m):
-        x, y = p[t]
-        canvas[y:y + H, x:x + W] = tiles.reshape(n * m, H, W)[t]
-    return canvas
+    return phases.overlay(tiles, p.reshape(pos.shape))
+
+
+# ---- pins of the oracle's phase 2 / phase 3 ------------------------------------------------
+def random_pairs(n, m, rng, ties=False, invalid=0.0):
+    """Random west/north records: translations, CCFs (optionally drawn from 3 values, so the
+    pair-id tie rule decides), a fraction of invalid pairs (candidate 0 / NaN CCF)."""
+    w = np.zeros((n, m), PAIR_DTYPE)
+    no = np.zeros((n, m), PAIR_DTYPE)
+    for rec, ok in ((w, np.arange(m)[None, :] >= 1), (no, np.arange(n)[:, None] >= 1)):
+        valid = np.broadcast_to(ok, (n, m)) & (rng.random((n, m)) >= invalid)
+        rec["dx"] = rng.integers(-40, 300, (n, m))
+        rec["dy"] = rng.integers(-40, 300, (n, m))
+        rec["ccf"] = (rng.choice([0.5, 0.7, 0.9], (n, m)) if ties else rng.random((n, m)))
+        rec["candidate"] = np.where(valid, rng.integers(1, 5, (n, m)), 0)
+        rec["ccf"] = np.where(valid, rec["ccf"], np.nan)
+    return w, no
+
+
+def brute_force_forest(nt, es):
+    """The best spanning forest by definition: among all acyclic edge sets with as many edges
+    as a spanning forest has, the one whose edge keys, sorted, are lexicographically smallest
+    (the greedy optimum of a matroid under a strict total order on its elements)."""
+    parent = list(range(nt))
+
+    def find(u, par):
+        while par[u] != u:
+            u = par[u]
+        return u
+    for _, a, b, _, _ in es:
+        ra, rb = find(a, parent), find(b, parent)
+        if ra != rb:
+            parent[ra] = rb
+    k = nt - len({find(u, parent) for u in range(nt)})
+    best = None
+    for sub in itertools.combinations(es, k):
+        par = list(range(nt))
+        acyclic = True
+        for _, a, b, _, _ in sub:
+            ra, rb = find(a, par), find(b, par)
+            if ra == rb:
+                acyclic = False
+                break
+            par[ra] = rb
+        if acyclic:
+            keys = sorted(e[0] for e in sub)
+            if best is None or keys < best[0]:
+                best = (keys, sub)
+    return sorted(best[1])
+
+
+@pytest.mark.parametrize("shape,ties,invalid", [((2, 2), False, 0.0), ((2, 3), False, 0.0),
+                                                ((3, 3), False, 0.0), ((2, 3), True, 0.0),
+                                                ((3, 3), True, 0.0), ((3, 3), False, 0.3),
+                                                ((2, 4), True, 0.4)])
+def test_oracle_spanning_tree_is_the_brute_force_optimum(shape, ties, invalid):
+    rng = np.random.default_rng(hash((shape, ties, invalid)) % 2**32)
+    for _ in range(5):
+        w, n = random_pairs(*shape, rng, ties, invalid)
+        es = phases.edges(w, n)
+        nt = shape[0] * shape[1]
+        assert sorted(phases.spanning_tree(nt, es)) == brute_force_forest(nt, es)
+
+
+def test_oracle_positions_are_path_sums():
+    """Exact translations of known origins: any tree gives the origins back (path invariance),
+    and every tile's position is its parent's plus the connecting translation."""
+    rng = np.random.default_rng(3)
+    n, m = 4, 6
+    org = np.stack(np.meshgrid(np.arange(m) * 200, np.arange(n) * 150), -1)
+    org = org + rng.integers(0, 9, (n, m, 2))
+    w, no = random_pairs(n, m, rng)
+    w["dx"][:, 1:] = org[:, 1:, 0] - org[:, :-1, 0]
+    w["dy"][:, 1:] = org[:, 1:, 1] - org[:, :-1, 1]
+    no["dx"][1:] = org[1:, :, 0] - org[:-1, :, 0]
+    no["dy"][1:] = org[1:, :, 1] - org[:-1, :, 1]
+    pos, parent = phases.global_positions(w, no)
+    assert np.array_equal(pos, org - org[0, 0])
+    assert parent[0, 0] == -1 and (parent.reshape(-1)[1:] >= 0).all()
+
+
+def test_oracle_overlay_per_pixel():
+    """Each canvas pixel is the pixel of the LAST tile (row-major) covering it, 0 if none."""
+    rng = np.random.default_rng(4)
+    tiles = rng.integers(1, 60000, (2, 3, 5, 7)).astype(np.uint16)
+    pos = np.array([[[0, 0], [5, 1], [11, 0]], [[1, 4], [6, 3], [12, 5]]])
+    canvas = phases.overlay(tiles, pos)
+    for y in range(canvas.shape[0]):
+        for x in range(canvas.shape[1]):
+            want = 0
+            for t in range(6):
+                px, py = pos.reshape(-1, 2)[t]
+                if px <= x < px + 7 and py <= y < py + 5:
+                    want = tiles.reshape(6, 5, 7)[t, y - py, x - px]
+            assert canvas[y, x] == want, (x, y)
+
+
+# ---- the product's phase 2 against the oracle's ---------------------------------------------
+@pytest.mark.parametrize("shape,ties,invalid", [((6, 7), False, 0.0), ((6, 7), True, 0.0),
+                                                ((9, 5), False, 0.25), ((8, 8), True, 0.35),
+                                                ((1, 9), False, 0.0), ((7, 1), True, 0.2)])
+def test_global_positions_match_oracle(shape, ties, invalid):
+    rng = np.random.default_rng(sum(shape) * 7 + int(ties) + int(invalid * 100))
+    for _ in range(4):
+        w, n = random_pairs(*shape, rng, ties, invalid)
+        pos, parent = global_positions(w, n)
+        opos, oparent = phases.global_positions(w, n)
+        assert np.array_equal(pos, opos)
+        assert np.array_equal(parent, oparent)
 
 
 @pytest.mark.gpu
