@@ -314,6 +314,16 @@ stitch_status stitch_compose_overlay(const uint16_t* dev_tiles, int32_t n, int32
                                      int32_t W, const int64_t* host_pos_xy, int64_t canvas_w,
                                      int64_t canvas_h, uint16_t* dev_canvas, void* stream);
 
+/*
+ * Phase 3, stream-ordered: as stitch_compose_overlay, but returns once the work is enqueued
+ * on `stream` (host_pos_xy is consumed before the call returns; dev_tiles and dev_canvas
+ * must stay valid until the stream reaches that point).  Errors: as above.
+ */
+stitch_status stitch_compose_overlay_async(const uint16_t* dev_tiles, int32_t n, int32_t m,
+                                           int32_t H, int32_t W, const int64_t* host_pos_xy,
+                                           int64_t canvas_w, int64_t canvas_h,
+                                           uint16_t* dev_canvas, void* stream);
+
 /* Message for the last error on ctx (valid until the next call on ctx). */
 const char* stitch_last_error(stitch_ctx* ctx);
 

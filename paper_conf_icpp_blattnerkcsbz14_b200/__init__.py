@@ -66,7 +66,8 @@ EXPORTS = ["stitch_status_string", "stitch_workspace_size", "stitch_pair_count",
            "stitch_forward_range_async", "stitch_spectra_range", "stitch_pairs_async",
            "stitch_global_positions", "stitch_compose_overlay", "stitch_debug_spectrum_f64",
            "stitch_compute_translations_from_host_async", "stitch_timeline",
-           "stitch_nccl_unique_id", "stitch_pairs_part_async", "stitch_debug_surface"]
+           "stitch_nccl_unique_id", "stitch_pairs_part_async", "stitch_debug_surface",
+           "stitch_compose_overlay_async"]
 
 _lib = None
 
@@ -114,6 +115,8 @@ def load_library():
         "stitch_pairs_async": (ctypes.c_int, [vp]),
         "stitch_global_positions": (ctypes.c_int, [i32, i32, vp, vp, vp, vp]),
         "stitch_compose_overlay": (ctypes.c_int, [vp, i32, i32, i32, i32, vp, i64, i64, vp, vp]),
+        "stitch_compose_overlay_async": (ctypes.c_int,
+                                         [vp, i32, i32, i32, i32, vp, i64, i64, vp, vp]),
     }
     for name, (res, args) in sig.items():
         f = getattr(lib, name)
@@ -172,9 +175,10 @@ def global_positions(west: np.ndarray, north: np.ndarray):
     return pos.reshape(n, m, 2), parent.reshape(n, m)
 
 
-def compose_overlay(tiles, pos_xy: np.ndarray, canvas=None):
+def compose_overlay(tiles, pos_xy: np.ndarray, canvas=None, sync: bool = True):
     """Phase 3 (f4): overlay-blend composite of a device tile grid (torch CUDA uint16
-    [n, m, H, W]) at integer origins pos_xy [n, m, 2]; returns the torch canvas."""
+    [n, m, H, W]) at integer origins pos_xy [n, m, 2]; returns the torch canvas.
+    sync=False: stream-ordered on torch's current stream (stitch_compose_overlay_async)."""
     import torch
     n, m, H, W = tiles.shape
     p = np.ascontiguousarray(pos_xy.reshape(-1, 2), dtype=np.int64)
@@ -182,11 +186,12 @@ def compose_overlay(tiles, pos_xy: np.ndarray, canvas=None):
     cw, ch = int(p[:, 0].max()) + W, int(p[:, 1].max()) + H
     if canvas is None:
         canvas = torch.zeros((ch, cw), dtype=torch.uint16, device=tiles.device)
-    st = load_library().stitch_compose_overlay(
+    name = "stitch_compose_overlay" if sync else "stitch_compose_overlay_async"
+    st = getattr(load_library(), name)(
         tiles.data_ptr(), n, m, H, W, p.ctypes.data, cw, ch, canvas.data_ptr(),
         torch.cuda.current_stream(tiles.device).cuda_stream)
     if st:
-        raise StitchError(st, "stitch_compose_overlay")
+        raise StitchError(st, name)
     return canvas
 
 

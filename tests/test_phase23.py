@@ -171,13 +171,17 @@ def test_global_positions_match_oracle(shape, ties, invalid):
 
 
 @pytest.mark.gpu
-@pytest.mark.parametrize("ov", [0.1, 0.7])
-def test_compose_overlay_matches_numpy(ov):
+@pytest.mark.parametrize("shape,ov", [((4, 5, 192, 256), 0.1), ((4, 5, 192, 256), 0.7),
+                                      ((3, 4, 26, 58), 0.3), ((2, 3, 1040, 1392), 0.1)])
+def test_compose_overlay_matches_numpy(shape, ov):
+    """The 16-byte vector path (W a multiple of 8: every source misalignment and canvas row
+    phase occurs) and the pixel path (W = 58)."""
     torch = pytest.importorskip("torch")
     if not torch.cuda.is_available():
         pytest.skip("needs a CUDA device")
     from paper_conf_icpp_blattnerkcsbz14_b200 import compose_overlay
-    g = synthgrid.make_grid(4, 5, 192, 256, overlap=ov, delta=4, seed=52)
+    n, m, H, W = shape
+    g = synthgrid.make_grid(n, m, H, W, overlap=ov, delta=4, seed=52)
     dev = torch.from_numpy(g.tiles.view(np.int16)).view(torch.uint16).cuda()
     canvas = compose_overlay(dev, g.origins)
     torch.cuda.synchronize()
