@@ -21,3 +21,13 @@ for tool in memcheck racecheck; do
   echo "== $tool (2x2 @ 1392x1040)"
   timeout 1200 compute-sanitizer --tool $tool --print-limit 20 python -c "$BIG" 2>&1 | tail -6
 done
+COMPOSE='import numpy as np, torch, synthgrid; from paper_conf_icpp_blattnerkcsbz14_b200 import compose_overlay
+for (n, m, H, W, ov) in ((3, 4, 192, 256, 0.1), (3, 4, 26, 58, 0.3)):
+    g = synthgrid.make_grid(n, m, H, W, overlap=ov, delta=4, seed=52)
+    dev = torch.from_numpy(g.tiles.view(np.int16)).view(torch.uint16).cuda()
+    c = compose_overlay(dev, g.origins); torch.cuda.synchronize()
+print("compose ok (16-byte and pixel paths)")'
+for tool in memcheck initcheck; do
+  echo "== $tool (phase 3 overlay)"
+  timeout 600 compute-sanitizer --tool $tool --print-limit 20 python -c "$COMPOSE" 2>&1 | tail -4
+done
