@@ -187,3 +187,29 @@ def test_compose_overlay_matches_numpy(shape, ov):
     torch.cuda.synchronize()
     got = canvas.cpu().view(torch.int16).numpy().view(np.uint16)
     assert np.array_equal(got, numpy_overlay(g.tiles, g.origins))
+
+
+@pytest.mark.gpu
+def test_compose_overlay_stays_inside_the_canvas():
+    """compute-sanitizer is unavailable on the GPU pool: the canvas is a view into a larger
+    buffer at an odd element offset (so its rows start at every 16-byte phase), the bytes
+    around it hold a sentinel, and the overlay must leave them untouched."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_icpp_blattnerkcsbz14_b200 import compose_overlay
+    for n, m, H, W, ov in ((3, 4, 192, 256, 0.1), (3, 4, 26, 58, 0.3), (2, 2, 1040, 1392, 0.1)):
+        g = synthgrid.make_grid(n, m, H, W, overlap=ov, delta=4, seed=53)
+        p = g.origins.reshape(-1, 2) - g.origins.reshape(-1, 2).min(axis=0)
+        cw, ch = int(p[:, 0].max()) + W, int(p[:, 1].max()) + H
+        pad = 4099
+        big = torch.full((2 * pad + ch * cw,), 0xBEEF - 65536, dtype=torch.int16, device="cuda")
+        big[pad:pad + ch * cw] = 0
+        canvas = big[pad:pad + ch * cw].view(torch.uint16).view(ch, cw)
+        dev = torch.from_numpy(g.tiles.view(np.int16)).view(torch.uint16).cuda()
+        compose_overlay(dev, g.origins, canvas)
+        torch.cuda.synchronize()
+        b = big.cpu().numpy().view(np.uint16)
+        assert (b[:pad] == 0xBEEF).all() and (b[pad + ch * cw:] == 0xBEEF).all(), (n, m, H, W)
+        got = b[pad:pad + ch * cw].reshape(ch, cw)
+        assert np.array_equal(got, numpy_overlay(g.tiles, g.origins)), (n, m, H, W)
