@@ -16,6 +16,7 @@
 // result is deterministic without atomics.  Each row of a tile writes one clear span with
 // 16-byte loads and stores (bandwidth-bound: ~2 x 2 bytes per canvas pixel).
 #include <cuda_runtime.h>
+#include <nvtx3/nvToolsExt.h>
 
 #include <algorithm>
 #include <climits>
@@ -226,6 +227,10 @@ stitch_status stitch_compose_overlay_async(const uint16_t* dev_tiles, int32_t n,
                                            int32_t H, int32_t W, const int64_t* host_pos_xy,
                                            int64_t canvas_w, int64_t canvas_h,
                                            uint16_t* dev_canvas, void* stream) {
+    nvtxRangePushA("stitch_compose_overlay_async");
+    struct Pop {
+        ~Pop() { nvtxRangePop(); }
+    } pop_;
     if (!dev_tiles || !host_pos_xy || !dev_canvas || n < 1 || m < 1 || H < 1 || W < 1 ||
         canvas_w < 1 || canvas_h < 1)
         return STITCH_ERR_INVALID_ARG;

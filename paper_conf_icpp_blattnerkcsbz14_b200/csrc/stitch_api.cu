@@ -16,6 +16,7 @@
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>   // types only: the functions are resolved with dlsym (no link-time NCCL)
+#include <nvtx3/nvToolsExt.h>   // header-only NVTX v3: a no-op unless a tool (ncu / nsys) attaches
 
 #include <algorithm>
 #include <cmath>
@@ -607,7 +608,17 @@ static stitch_status nccl_fail(stitch_ctx* ctx, ncclResult_t r, const char* wher
         if (e_ != cudaSuccess) return cuda_fail(ctx, e_, where); \
     } while (0)
 
+// Tracing: every device-touching entry point is an NVTX range named after
+// it, so a profiler can scope captures to a call (ncu --nvtx --nvtx-include "stitch_.../").
+struct NvtxRange {
+    explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+    ~NvtxRange() { nvtxRangePop(); }
+    NvtxRange(const NvtxRange&) = delete;
+    NvtxRange& operator=(const NvtxRange&) = delete;
+};
+
 #define GUARD(ctx)                                                          \
+    NvtxRange nvtx_(__func__);                                              \
     DevGuard guard_((ctx)->cfg.device);                                     \
     if (guard_.err != cudaSuccess) return cuda_fail(ctx, guard_.err, "set device")
 

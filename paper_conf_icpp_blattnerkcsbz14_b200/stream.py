@@ -16,6 +16,7 @@ are dealt round-robin to the ranks (independent problems, no data-path collectiv
 """
 from __future__ import annotations
 
+import os
 from dataclasses import dataclass
 from typing import Callable, Iterable
 
@@ -29,6 +30,54 @@ class GridResult:
     index: int
     west: np.ndarray
     north: np.ndarray
+
+
+class ResultStore:
+    """Per-scan resumability of a time series: each finished
+    grid's (west, north) records go to their own file `grid_<index>.npz` in `directory`,
+    written to a temporary name and renamed into place, so a file present is a complete
+    result and a run that stops (crash, preemption) loses at most the grids in flight.
+    A restarted stream skips every index already stored."""
+
+    PREFIX, SUFFIX = "grid_", ".npz"
+
+    def __init__(self, directory: str):
+        self.dir = directory
+        os.makedirs(directory, exist_ok=True)
+
+    def path(self, index: int) -> str:
+        return os.path.join(self.dir, f"{self.PREFIX}{index:07d}{self.SUFFIX}")
+
+    def done(self) -> set[int]:
+        out = set()
+        for f in os.listdir(self.dir):
+            if f.startswith(self.PREFIX) and f.endswith(self.SUFFIX):
+                try:
+                    out.add(int(f[len(self.PREFIX):-len(self.SUFFIX)]))
+                except ValueError:
+                    pass
+        return out
+
+    def save(self, r: GridResult) -> None:
+        tmp = os.path.join(self.dir, f".tmp_{r.index}_{os.getpid()}.npz")
+        with open(tmp, "wb") as f:
+            np.savez(f, west=r.west, north=r.north)
+            f.flush()
+            os.fsync(f.fileno())
+        os.replace(tmp, self.path(r.index))
+
+    def load(self, index: int) -> GridResult:
+        with np.load(self.path(index)) as z:
+            return GridResult(index, z["west"], z["north"])
+
+
+def pending(indices: Iterable[int], store: ResultStore | None) -> list[int]:
+    """The indices still to run (in order): all of them, or those the store lacks."""
+    indices = list(indices)
+    if store is None:
+        return indices
+    done = store.done()
+    return [i for i in indices if i not in done]
 
 
 class GridStream:
@@ -47,15 +96,18 @@ class GridStream:
         self.pairs_per_grid = self.slots[0]["grid"].npairs
 
     def run(self, indices: Iterable[int], fill: Callable[[int, np.ndarray], object],
-            sink: Callable[[GridResult], None] | None = None) -> int:
+            sink: Callable[[GridResult], None] | None = None,
+            store: ResultStore | None = None) -> int:
         """For each grid index: fill(index, host_array) either writes its tiles into the
         slot's pinned buffer (returning None) or returns a pinned host tensor / array that
         already holds them; then H2D + steps 2-7 are enqueued on the slot's stream.
-        Results are collected (and passed to `sink`) when the slot comes round again.
+        Results are collected (saved to `store`, then passed to `sink`) when the slot comes
+        round again; with a store, indices it already holds are skipped (resume).
         Returns the number of grids processed."""
         count = 0
         S = len(self.slots)
-        for k, idx in enumerate(indices):
+        self._store = store
+        for k, idx in enumerate(pending(indices, store)):
             sl = self.slots[k % S]
             if sl["pending"] is not None:
                 self._collect(sl, sink)
@@ -72,8 +124,11 @@ class GridStream:
 
     def _collect(self, sl, sink):
         w, n = sl["grid"].get_translations()          # D2H of the results, synchronous
+        r = GridResult(sl["pending"], w.copy(), n.copy())
+        if getattr(self, "_store", None) is not None:
+            self._store.save(r)
         if sink is not None:
-            sink(GridResult(sl["pending"], w.copy(), n.copy()))
+            sink(r)
         sl["pending"] = None
 
     def close(self) -> None:

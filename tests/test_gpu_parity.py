@@ -10,6 +10,8 @@ Tolerances (BASELINE.json north_star):
     1e-4 of its max, any GPU peak in that near-tie set is accepted, and the
     GPU's (dx, dy, candidate, ccf) must equal oracle.eval_peak at the GPU peak.
 """
+import os
+
 import numpy as np
 import pytest
 
@@ -218,6 +220,33 @@ def test_stream_time_series_matches_per_grid():
     ow, on = oracle.grid(grids[3])
     assert np.array_equal(got[3].west["dx"][:, 1:], ow["dx"][:, 1:])
     assert np.array_equal(got[3].north["dy"][1:], on["dy"][1:])
+
+
+def test_stream_resumes_from_its_result_store(tmp_path):
+    """Per-scan resumability: a run interrupted after some grids (here:
+    the first run covers 3 of 6, then one stored result is lost) is restarted with the same
+    store; only the missing grids run, and every stored result equals an uninterrupted run's."""
+    from paper_conf_icpp_blattnerkcsbz14_b200.stream import GridStream, ResultStore
+    n, m, H, W = 3, 4, 192, 256
+    grids = {i: synthgrid.make_grid(n, m, H, W, scan=i, seed=43).tiles for i in range(6)}
+    ran = []
+
+    def fill(i, host):
+        ran.append(i)
+        host[...] = grids[i]
+
+    store = ResultStore(str(tmp_path / "series"))
+    with GridStream(n, m, H, W, slots=2) as gs:
+        assert gs.run([0, 1, 2], fill, store=store) == 3
+        os.remove(store.path(1))
+        ran.clear()
+        assert gs.run(range(6), fill, store=store) == 4
+    assert ran == [1, 3, 4, 5] and store.done() == set(range(6))
+    for i, tiles in grids.items():
+        w, nn, _ = run_gpu(tiles)
+        r = store.load(i)
+        assert r.west.tobytes() == w.reshape(n, m).tobytes() and \
+            r.north.tobytes() == nn.reshape(n, m).tobytes()
 
 
 def test_compute_from_host_pipelined_matches_load_then_compute():
