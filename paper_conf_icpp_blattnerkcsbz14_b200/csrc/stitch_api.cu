@@ -390,11 +390,13 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     L->pool = c->pool_tiles > 0;
     if (L->pool && (L->prec || c->nccl_id)) return STITCH_ERR_UNSUPPORTED;
     L->nslots = L->pool ? std::min(c->pool_tiles, L->nlocal) : L->nlocal;
-    // fp64 chunks of 8 keep the 94 MB intermediate (8 x H x WP x 16 B at 1392x1040) in L2
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : (L->prec ? 8 : 160);
+    // default chunks (both precisions): 160 pairs / 64 tiles -- the intermediates round-trip
+    // HBM either way, and larger launches lose less to their tail wave (fp64 sweep: 8/8 75.7 ms,
+    // 32/16 68.5 ms, 160/64 67.8 ms per 42x59 step, DESIGN.md variant 40)
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 160;
     L->chunk_tiles = c->chunk_tiles > 0
                          ? c->chunk_tiles
-                         : (L->prec ? 8 : (L->pool ? std::max(1, std::min(64, L->nslots / 4)) : 64));
+                         : (L->pool ? std::max(1, std::min(64, L->nslots / 4)) : 64);
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     // spectrum by slot: u32 Q15 unit phasor [WP][HP] (fp32) or double2 unit phasor [H][WP] (fp64)
