@@ -14,7 +14,7 @@ CSRC = os.path.join(PKG, "csrc")
 LIB = os.path.join(PKG, "libstitch_b200.so")
 SOURCES = ["stitch_api.cu", "phase23.cu"]
 HEADERS = ["fft_engine.cuh", "pciam_kernels.cuh", "pciam_fp64.cuh", "warp_rows.cuh",
-           "async_copy.cuh", "codelets.cuh", "gen_codelets.py"]
+           "async_copy.cuh", "codelets.cuh", "f32x2.cuh", "gen_codelets.py"]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 

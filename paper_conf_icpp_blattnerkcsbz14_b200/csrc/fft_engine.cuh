@@ -19,16 +19,13 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
-#include "codelets.cuh"
+#include "codelets.cuh"   // includes f32x2.cuh
 
 namespace stitch {
 
-__device__ __forceinline__ float2 cmul(float2 a, float2 b) {
-    return make_float2(fmaf(a.x, b.x, -a.y * b.y), fmaf(a.x, b.y, a.y * b.x));
-}
-__device__ __forceinline__ float2 cmulc(float2 a, float2 b) {  // a * conj(b)
-    return make_float2(fmaf(a.x, b.x, a.y * b.y), fmaf(a.y, b.x, -a.x * b.y));
-}
+// fp32 complex products on the packed f32x2 instructions (two instructions each, f32x2.cuh)
+__device__ __forceinline__ float2 cmul(float2 a, float2 b) { return cmul2(a, b); }
+__device__ __forceinline__ float2 cmulc(float2 a, float2 b) { return cmulc2(a, b); }  // a * conj(b)
 // fp64 twins (the f2 path instantiates the engine with C = double2)
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
     return make_double2(fma(a.x, b.x, -a.y * b.y), fma(a.x, b.y, a.y * b.x));

@@ -300,6 +300,235 @@ def pi4_twiddle(num, den):
     return den // g == 8
 
 
+# ---------------------------------------------------------------------------------------
+# Packed fp32 codelets (sm_100a FADD2 / FMUL2 / FFMA2, f32x2.cuh): the same algorithms at the
+# level of complex values.  Every complex add, complex x real constant, and complex fma with a
+# real constant is ONE packed instruction (the scalar codelets above spend two), and a
+# multiplication by a power of i is free: a value is (name, r) meaning i^r * name, emitted as
+# the operand view name / I(name) / NEG(name) / MI(name) that ptxas folds into the packed
+# instruction's source selectors.
+
+class PEm:
+    def __init__(self):
+        self.lines = []
+        self.n = 0
+
+    def new(self, expr: str):
+        self.n += 1
+        name = f"t{self.n}"
+        self.lines.append(f"    const float2 {name} = {expr};")
+        return (name, 0)
+
+
+def pop(v):
+    name, r = v
+    return (name, f"I({name})", f"NEG({name})", f"MI({name})")[r % 4]
+
+
+def prot(v, k):
+    """i^k * v (free)."""
+    return (v[0], (v[1] + k) % 4)
+
+
+def padd(e, a, b):
+    return e.new(f"f2add({pop(a)}, {pop(b)})")
+
+
+def psub(e, a, b):
+    return e.new(f"f2sub({pop(a)}, {pop(b)})")
+
+
+def pmul(e, a, c):
+    return e.new(f"f2mul({pop(a)}, K({flit(c)}))")
+
+
+def pfma(e, a, c, acc):
+    """a * c + acc, c real."""
+    return e.new(f"f2fma({pop(a)}, K({flit(c)}), {pop(acc)})")
+
+
+def ptwiddle(e, a, num, den, sign):
+    """a * exp(sign * 2 pi i num / den)."""
+    num %= den
+    if num == 0:
+        return a
+    g = math.gcd(num, den)
+    num //= g
+    den //= g
+    if den == 2:
+        return prot(a, 2)
+    if den == 4:
+        return prot(a, num if sign > 0 else (4 - num) % 4)
+    ang = sign * 2.0 * math.pi * num / den
+    c, s = math.cos(ang), math.sin(ang)
+    if den == 8:                       # sqrt(1/2) (+-a +- i a)
+        t = padd(e, prot(a, 0 if c > 0 else 2), prot(a, 1 if s > 0 else 3))
+        return pmul(e, t, math.sqrt(0.5))
+    return pfma(e, prot(a, 1), s, pmul(e, a, c))        # a c + (i a) s
+
+
+def pprime_rader(e, xs, sign):
+    """prime_rader on complex values (same Rader / CRT structure, one packed op per step)."""
+    n = len(xs)
+    h = (n - 1) // 2
+    g = primitive_root(n)
+    ja = [pow(g, a, n) for a in range(h)]
+    kb = [pow(g, (n - 1 - b) % (n - 1), n) for b in range(h)]
+    s = [padd(e, xs[j], xs[n - j]) for j in ja]
+    d = [psub(e, xs[j], xs[n - j]) for j in ja]
+    q = h // 2
+    up = [padd(e, s[a], s[a + q]) for a in range(q)]
+    um = [psub(e, s[a], s[a + q]) for a in range(q)]
+    out = [None] * n
+    acc = xs[0]
+    for a in range(q):
+        acc = padd(e, acc, up[a])
+    out[0] = acc
+    C = [math.cos(2.0 * math.pi * pow(g, m, n) / n) for m in range(h)]
+    P = [0.5 * (C[m] + C[(m + q) % h]) for m in range(q)]
+    Nm = [0.5 * (C[m] - C[(m + q) % h]) for m in range(h)]
+    A = [None] * h
+    for b in range(q):
+        pp = xs[0]
+        for a in range(q):
+            pp = pfma(e, up[a], P[(a - b) % q], pp)
+        ap = pp
+        for a in range(q):
+            m = a - b
+            ap = pfma(e, um[a], Nm[m] if m >= 0 else -Nm[m + q], ap)
+        A[b] = ap
+        A[b + q] = pfma(e, pp, 2.0, prot(ap, 2))          # pp - nn
+
+    def S(m):
+        return math.sin(2.0 * math.pi * pow(g, m % (n - 1), n) / n)
+    u = [d[a] for a in range(q)]
+    v = [d[a + q] for a in range(q)]
+    uv = [padd(e, u[a], v[a]) for a in range(q)]
+    Bv = [None] * h
+    for b in range(q):
+        t1 = None
+        for a in range(q):
+            t1 = pmul(e, u[a], S(a - b)) if t1 is None else pfma(e, u[a], S(a - b), t1)
+        y0 = t1
+        for a in range(q):
+            y0 = pfma(e, v[a], S(a - b + q), y0)
+        y1 = pfma(e, t1, -2.0, y0)
+        for a in range(q):
+            y1 = pfma(e, uv[a], S(a - b) - S(a - b + q), y1)
+        Bv[b] = y0
+        Bv[b + q] = y1
+    for b in range(h):                 # X_k = A - sign i B... as the scalar form:
+        k = kb[b]                      # sign < 0: X_k = A - i B, X_{n-k} = A + i B
+        lo, hi = (3, 1) if sign < 0 else (1, 3)
+        out[k] = padd(e, A[b], prot(Bv[b], lo))
+        out[n - k] = padd(e, A[b], prot(Bv[b], hi))
+    return out
+
+
+def pgen(e, xs, sign):
+    n = len(xs)
+    if n == 1:
+        return list(xs)
+    if n == 2:
+        return [padd(e, xs[0], xs[1]), psub(e, xs[0], xs[1])]
+    sp = psplit(n)
+    if sp is None and n >= RADER_MIN and ((n - 1) // 2) % 2 == 0:
+        return pprime_rader(e, xs, sign)
+    if sp is None:                     # prime: symmetric form
+        h = (n - 1) // 2
+        s = [None] + [padd(e, xs[j], xs[n - j]) for j in range(1, h + 1)]
+        d = [None] + [psub(e, xs[j], xs[n - j]) for j in range(1, h + 1)]
+        out = [None] * n
+        acc = xs[0]
+        for j in range(1, h + 1):
+            acc = padd(e, acc, s[j])
+        out[0] = acc
+        for k in range(1, h + 1):
+            if h == 1:                 # n = 3
+                c = math.cos(2.0 * math.pi * k / n)
+                sn = math.sin(2.0 * math.pi * k / n) * (1 if sign < 0 else -1)
+                A = pfma(e, s[1], c, xs[0])
+                out[k] = pfma(e, prot(d[1], 3), sn, A)          # A + sn (-i d)
+                out[n - k] = pfma(e, prot(d[1], 3), -sn, A)
+                continue
+            A = xs[0]
+            for j in range(1, h + 1):
+                A = pfma(e, s[j], math.cos(2.0 * math.pi * ((j * k) % n) / n), A)
+            sn = [None] + [math.sin(2.0 * math.pi * ((j * k) % n) / n) for j in range(1, h + 1)]
+            j0 = max(range(1, h + 1), key=lambda j: abs(sn[j]))
+            Iv = d[j0]
+            for j in range(1, h + 1):
+                if j != j0:
+                    Iv = pfma(e, d[j], sn[j] / sn[j0], Iv)
+            f = sn[j0] if sign < 0 else -sn[j0]
+            out[k] = pfma(e, prot(Iv, 3), f, A)                  # A + f (-i I)
+            out[n - k] = pfma(e, prot(Iv, 3), -f, A)
+        return out
+    n1, n2 = sp
+    if math.gcd(n1, n2) == 1:
+        u, w = pow(n2, -1, n1), pow(n1, -1, n2)
+        Y = [pgen(e, [xs[(n2 * a + n1 * b) % n] for a in range(n1)], sign) for b in range(n2)]
+        out = [None] * n
+        for k1 in range(n1):
+            X = pgen(e, [Y[b][k1] for b in range(n2)], sign)
+            for k2 in range(n2):
+                out[(n2 * u * k1 + n1 * w * k2) % n] = X[k2]
+        return out
+    Y = [pgen(e, [xs[n2 * a + b] for a in range(n1)], sign) for b in range(n2)]
+    out = [None] * n
+    for k1 in range(n1):
+        if n2 == 2 and pi4_twiddle(k1, n):
+            y0, y1 = Y[0][k1], Y[1][k1]
+            ang = sign * 2.0 * math.pi * k1 / n
+            cs, ss = (1 if math.cos(ang) > 0 else -1), (1 if math.sin(ang) > 0 else -1)
+            t = padd(e, prot(y1, 0 if cs > 0 else 2), prot(y1, 1 if ss > 0 else 3))
+            out[k1] = pfma(e, t, math.sqrt(0.5), y0)
+            out[k1 + n1] = pfma(e, t, -math.sqrt(0.5), y0)
+            continue
+        X = pgen(e, [ptwiddle(e, Y[b][k1], b * k1, n, sign) for b in range(n2)], sign)
+        for k2 in range(n2):
+            out[k1 + n1 * k2] = X[k2]
+    return out
+
+
+_PBEST = {}
+_PFORCE = {}
+
+
+def psplit(n):
+    """split() for the packed codelets (instruction count = emitted operations)."""
+    if n in _PFORCE:
+        return _PFORCE[n]
+    divs = [d for d in range(2, n) if n % d == 0]
+    if not divs:
+        return None
+    if n not in _PBEST:
+        def cost(sp):
+            e = PEm()
+            _PFORCE[n] = sp
+            try:
+                outs = pgen(e, [(f"x{j}", 0) for j in range(n)], -1)
+            finally:
+                del _PFORCE[n]
+            return len(e.lines) + sum(1 for o in outs if o[1] % 4)
+        _PBEST[n] = min(((d, n // d) for d in divs), key=lambda sp: (cost(sp), sp))
+    return _PBEST[n]
+
+
+def codelet_packed(n, sign):
+    e = PEm()
+    outs = pgen(e, [(f"x{j}", 0) for j in range(n)], sign)
+    tag = "m" if sign < 0 else "p"
+    lines = [f"__device__ __forceinline__ void dft{n}{tag}(float2* __restrict__ v) {{"]
+    for j in range(n):
+        lines.append(f"    const float2 x{j} = v[{j}];")
+    lines += e.lines
+    for k in range(n):
+        lines.append(f"    v[{k}] = {pop(outs[k])};")
+    lines.append("}")
+    return "\n".join(lines)
+
+
 def codelet(n, sign):
     e = Em()
     xs = []
@@ -333,13 +562,13 @@ def to_double(src: str) -> str:
 def main():
     out = ["// GENERATED by gen_codelets.py -- do not edit.",
            "// Straight-line fp32 / fp64 DFT codelets: v[k] <- sum_j v[j] exp(SIGN 2 pi i j k / R).",
-           "#pragma once", "", "namespace stitch {", "",
+           "// fp32: packed complex operations (f32x2.cuh); fp64: scalar double.",
+           "#pragma once", "", '#include "f32x2.cuh"', "", "namespace stitch {", "",
            "template <int R, int SIGN> struct Dft;", ""]
     for r in RADICES:
         for sign in (-1, 1):
-            c = codelet(r, sign)
-            out.append(c)
-            out.append(to_double(c))
+            out.append(codelet_packed(r, sign))         # fp32: packed f32x2
+            out.append(to_double(codelet(r, sign)))     # fp64 (f2): the scalar program in double
             tag = "m" if sign < 0 else "p"
             out.append(f"template <> struct Dft<{r}, {sign}> {{\n"
                        f"    static __device__ __forceinline__ void run(float2* v) {{ dft{r}{tag}(v); }}\n"

@@ -130,17 +130,47 @@ def _eval_codelet(body, x):
     return np.array([out[k] for k in range(len(x))])
 
 
+def _eval_packed_codelet(body, x):
+    """The fp32 codelets are packed complex programs (f32x2.cuh): every value is a complex
+    number, f2add / f2sub / f2mul / f2fma act component-wise, K(c) is a real constant, and the
+    views I / MI / NEG multiply by i, -i, -1."""
+    env = {"f2add": lambda a, b: a + b, "f2sub": lambda a, b: a - b,
+           "f2mul": lambda a, b: a * b, "f2fma": lambda a, b, c: a * b + c,
+           "K": lambda c: float(c), "I": lambda v: 1j * v, "MI": lambda v: -1j * v,
+           "NEG": lambda v: -v, "v": list(x), "out": {}}
+    py = []
+    for line in body.split("\n"):
+        line = re.sub(r"\((-?[0-9.e+-]+)f\)", r"(\1)", line.strip().rstrip(";"))
+        if line.startswith("const float2 "):
+            py.append(line[len("const float2 "):])
+        elif line.startswith("v["):
+            mm = re.match(r"v\[(\d+)\] = (.*)", line)
+            py.append(f"out[{mm.group(1)}] = {mm.group(2)}")
+        else:
+            assert not line or line.startswith("//"), line
+    exec("\n".join(py), env)
+    return np.array([env["out"][k] for k in range(len(x))])
+
+
 def test_generated_codelets_are_dfts():
+    """fp32 codelets (packed complex operations) evaluate to the DFT; each costs about half
+    the instructions of its scalar fp64 twin (one packed operation per complex step)."""
     src = open(os.path.join(ROOT, "paper_conf_icpp_blattnerkcsbz14_b200", "csrc",
                             "codelets.cuh")).read()
     funcs = re.findall(r"void dft(\d+)([mp])\(float2\* __restrict__ v\) \{\n(.*?)\n\}", src, re.S)
     assert len(funcs) >= 20
+    twins = dict(((n, t), b) for n, t, b in re.findall(
+        r"void dft(\d+)([mp])_d\(double2\* __restrict__ v\) \{\n(.*?)\n\}", src, re.S))
     rng = np.random.default_rng(0)
     for n, tag, body in funcs:
+        assert "float " not in body and "fmaf" not in body, (n, tag)
+        packed_ops = body.count("const float2 t")
+        scalar_ops = twins[(n, tag)].count("const double t")
+        assert packed_ops <= 0.55 * scalar_ops + 2, (n, tag, packed_ops, scalar_ops)
         n = int(n)
         sign = -1 if tag == "m" else 1
         x = rng.standard_normal(n) + 1j * rng.standard_normal(n)
-        got = _eval_codelet(body, x)
+        got = _eval_packed_codelet(body, x)
         j = np.arange(n)
         ref = np.exp(sign * 2j * math.pi * np.outer(j, j) / n) @ x
         assert np.abs(got - ref).max() <= 1e-6 * np.abs(ref).max(), (n, tag)
