@@ -141,6 +141,8 @@ struct FftRunPfa<Radix<N, R0, R1>, SIGN, L, T, C> {
                     if constexpr (SLOT_OUT) {
 #pragma unroll
                         for (int j = 0; j < R1; ++j) xc.at(line, k1, j) = v[j];
+                    } else if constexpr (Dst::PFA_BATCH) {
+                        dst.template store_pfa<R1, C1, C2, N>(line, k1, v);
                     } else {
                         int n = (C1 * k1) % N;
 #pragma unroll
@@ -590,6 +592,29 @@ struct ArgmaxDstD {  // step 5 in double: running (max |x|, smallest index at th
     double best_v;     // -1 before the first value
     uint32_t best_i;
     int row_base, W;
+    // A whole prime-factor butterfly at once (output j at n = (C1 k1 + C2 j) mod N): its max
+    // |x| by DSETP.MAX, and only when that reaches the running best (rare once a block is under
+    // way) the smallest index holding it -- the same (value, index) as `store` value by value.
+    static constexpr bool PFA_BATCH = true;
+    template <int R1, int C1, int C2, int N>
+    __device__ __forceinline__ void store_pfa(int line, int k1, const double2 (&v)[R1]) {
+        double m = fmax(fabs(v[0].x), fabs(v[0].y));
+#pragma unroll
+        for (int j = 1; j < R1; ++j) m = fmax(m, fmax(fabs(v[j].x), fabs(v[j].y)));
+        if (m >= best_v) {
+            const uint32_t base = (uint32_t)(row_base + line) * W;
+            uint32_t idx = 0xFFFFFFFFu, n = (uint32_t)((C1 * k1) % N);
+#pragma unroll
+            for (int j = 0; j < R1; ++j) {
+                if (fabs(v[j].x) == m) idx = min(idx, base + 2 * n);
+                if (fabs(v[j].y) == m) idx = min(idx, base + 2 * n + 1);
+                n += C2;
+                if (n >= (uint32_t)N) n -= N;
+            }
+            best_i = m > best_v ? idx : min(idx, best_i);
+            best_v = m;
+        }
+    }
     __device__ __forceinline__ void take(double a, uint32_t idx) {
         if (a > best_v || (a == best_v && idx < best_i)) {
             best_v = a;
