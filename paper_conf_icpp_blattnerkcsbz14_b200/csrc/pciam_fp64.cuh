@@ -696,6 +696,121 @@ __global__ void __launch_bounds__(PL::ROW_T, 3) d4_pair_rows(const double2* __re
     }
 }
 
+// ------------------------------------------------------------------ D4w ---
+// D4 as a warp-per-row kernel (the fp32 K4w design in double): each warp walks a contiguous run
+// of ROW_L-row blocks, the next row landing by bulk copy (per-warp mbarrier) as soon as stage 1
+// has read the current one, with no CTA-wide barrier; the C2R pre-pass runs in place on the
+// landed row, the prime-factor 29 x 24 transform on the warp (WarpFftPfa in double), and each
+// stage-2 lane keeps a running (max |x|, smallest index) over the block's rows; at the block's
+// end one warp reduction writes the block partial D5 reduces.  (The CTA version lost a third of
+// its stall samples to the landing wait and its two barriers, ncu r02_ncu_d4.txt.)
+constexpr int D4W_WARPS = 10;   // 10 x 22.4 KB of landing + exchange: one CTA per SM
+
+template <class PL>
+struct D4w {
+    using RI = typename PL::RI;
+    static constexpr size_t QROW = sizeof(double2) * PL::WP;          // a landed Q row
+    static constexpr size_t XCH = sizeof(double2) * RI::R1 * RI::R0;   // exchange (PAD 0)
+    static constexpr size_t WARP = QROW + XCH;
+    static constexpr size_t OFF_WARP = 128;                            // after the mbarriers
+    static constexpr size_t SMEM = OFF_WARP + D4W_WARPS * WARP;
+    static constexpr bool OK = RI::STAGES == 2 && gcd_c(RI::R0, RI::R1) == 1 && RI::R0 % 2 == 1 &&
+                               RI::R0 <= 32 && RI::R1 <= 32 && PL::H % PL::ROW_L == 0 &&
+                               QROW % 16 == 0 && SMEM <= 227 * 1024;
+};
+
+template <int R1, int C1, int C2, int N>
+struct WarpArgmaxD {   // a lane's running (max |x|, smallest index) over the rows of a block
+    double best_v;
+    uint32_t best_i;
+    int row_base, W;
+    __device__ __forceinline__ void store_pfa(int k1, const double2 (&v)[R1]) {
+        double m = fmax(fabs(v[0].x), fabs(v[0].y));
+#pragma unroll
+        for (int j = 1; j < R1; ++j) m = fmax(m, fmax(fabs(v[j].x), fabs(v[j].y)));
+        if (m >= best_v) {
+            const uint32_t base = (uint32_t)row_base * W;
+            uint32_t idx = 0xFFFFFFFFu, n = (uint32_t)((C1 * k1) % N);
+#pragma unroll
+            for (int j = 0; j < R1; ++j) {
+                if (fabs(v[j].x) == m) idx = min(idx, base + 2 * n);
+                if (fabs(v[j].y) == m) idx = min(idx, base + 2 * n + 1);
+                n += C2;
+                if (n >= (uint32_t)N) n -= N;
+            }
+            best_i = m > best_v ? idx : min(idx, best_i);
+            best_v = m;
+        }
+    }
+};
+
+template <class PL>
+__global__ void __launch_bounds__(32 * D4W_WARPS, 1)
+    d4w_pair_rows(const double2* __restrict__ Q, double* __restrict__ part_v,
+                  uint32_t* __restrict__ part_i, int pair0, int npairs,
+                  const double2* __restrict__ twW) {
+    using DW = D4w<PL>;
+    using RI = typename PL::RI;
+    constexpr int M = PL::M, H = PL::H, L = PL::ROW_L, NBLK = Plan64<PL>::NBLK;
+    extern __shared__ __align__(128) unsigned char smem_d4w[];
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_d4w) + (threadIdx.x >> 5);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned char* mine = smem_d4w + DW::OFF_WARP + warp * DW::WARP;
+    double2* landw = reinterpret_cast<double2*>(mine);
+    const WarpXchg<RI::R0, RI::R1, 0, double2> xc{reinterpret_cast<double2*>(mine + DW::QROW)};
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+    }
+    __syncwarp();
+    const long long nb = (long long)npairs * NBLK;
+    const long long gw = (long long)blockIdx.x * D4W_WARPS + warp, nw = (long long)gridDim.x * D4W_WARPS;
+    const int r0 = (int)(nb * gw / nw) * L, r1 = (int)(nb * (gw + 1) / nw) * L;
+    auto issue = [&](int r) {
+        mbar_arrive_expect_tx(bar, (uint32_t)DW::QROW);
+        bulk_g2s(mine, Q + (size_t)r * PL::WP, (uint32_t)DW::QROW, bar);
+    };
+    if (lane == 0 && r0 < r1) issue(r0);
+    using Pfa = WarpFftPfa<typename PL::Row, +1, double2>;
+    WarpArgmaxD<RI::R1, Pfa::C1, Pfa::C2, M> acc{-1.0, 0xFFFFFFFFu, 0, PL::W};
+    int k = 0;
+    for (int r = r0; r < r1; ++r, ++k) {
+        const int pl = r / H, y = r - pl * H;
+        acc.row_base = y;
+        mbar_wait(bar, k & 1);
+        // C2R pre-processing in place (as K4w): Z[q] = X[q] + conj X[M-q] + i o,
+        // Z[M-q] = conj(X[q] + conj X[M-q]) + i conj(o), o = (X[q] - conj X[M-q]) conj(w_W^q)
+        for (int q = lane; 2 * q <= M; q += 32) {
+            const double2 xn = landw[q], xm = landw[M - q];
+            const double2 o = cmulc(make_double2(xn.x - xm.x, xn.y + xm.y), __ldg(&twW[q]));
+            const double sx = xn.x + xm.x, dy = xn.y - xm.y;
+            landw[q] = make_double2(sx - o.y, dy + o.x);
+            if (q != 0 && 2 * q != M) landw[M - q] = make_double2(sx + o.y, o.x - dy);
+        }
+        __syncwarp();
+        auto prefetch = [&]() {
+            if (lane == 0 && r + 1 < r1) {
+                fence_proxy_async();
+                issue(r + 1);
+            }
+        };
+        Pfa::run(landw, xc, acc, lane, prefetch);
+        __syncwarp();                          // exchange free for the next row
+        if ((y + 1) % L == 0) {                // block end: one partial per ROW_L rows
+            double v = acc.best_v;
+            uint32_t i = acc.best_i;
+            warp_argmax(v, i);
+            if (lane == 0) {
+                const size_t o = (size_t)(pair0 + pl) * NBLK + y / L;
+                part_v[o] = v;
+                part_i[o] = i;
+            }
+            acc.best_v = -1.0;
+            acc.best_i = 0xFFFFFFFFu;
+        }
+    }
+}
+
 // ------------------------------------------------------------------ D5 ----
 // One warp per pair: reduce the NBLK block partials and emit the K5/K6 key
 // (bits(float(max)) << 32 | (2^32 - 1 - index)); the index is the exact double argmax.

@@ -200,6 +200,7 @@ cudaError_t d_setup() {
     using P64 = Plan64<PL>;
     CKE(max_smem(d1_fwd_rows<PL>, P64::ROW_SMEM));
     CKE(max_smem(d4_pair_rows<PL>, P64::D4_SMEM));
+    if constexpr (D4w<PL>::OK) CKE(max_smem(d4w_pair_rows<PL>, D4w<PL>::SMEM));
     CKE(max_smem(d2_fwd_cols<PL, true>, P64::D2_SMEM));
     CKE(max_smem(d2_fwd_cols<PL, false>, P64::D2_SMEM));
     if constexpr (D3P<PL>::F::OK) {
@@ -249,6 +250,18 @@ template <class PL>
 void launch_d4(const double2* Q, double* pv, uint32_t* pi, int p0, int np, const double2* tw2,
                const double2* twW, cudaStream_t s) {
     using P64 = Plan64<PL>;
+    if constexpr (D4w<PL>::OK) {   // warp per row, one CTA per SM
+        static int sms = 0;
+        if (!sms) {
+            int dev = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        }
+        const int need = (int)(((long long)np * P64::NBLK + D4W_WARPS - 1) / D4W_WARPS);
+        d4w_pair_rows<PL><<<need < sms ? need : sms, 32 * D4W_WARPS, D4w<PL>::SMEM, s>>>(
+            Q, pv, pi, p0, np, twW);
+        return;
+    }
     d4_pair_rows<PL><<<dim3(P64::NBLK, np), P64::ROW_T, P64::D4_SMEM, s>>>(Q, pv, pi, p0, tw2,
                                                                             twW);
 }

@@ -19,18 +19,18 @@
 namespace stitch {
 
 // Exchange slot of element (u < R0, v < R1): v*(R0+PAD) + u; natural index n = v*R0 + u.
-template <int R0, int R1, int PAD>
+template <int R0, int R1, int PAD, class C = float2>
 struct WarpXchg {
-    float2* s;
+    C* s;
     static constexpr int SIZE = R1 * (R0 + PAD);
-    __device__ __forceinline__ float2& at(int u, int v) const { return s[v * (R0 + PAD) + u]; }
-    __device__ __forceinline__ float2& nat(int n) const {
+    __device__ __forceinline__ C& at(int u, int v) const { return s[v * (R0 + PAD) + u]; }
+    __device__ __forceinline__ C& nat(int n) const {
         if constexpr (PAD == 0)
             return s[n];
         else
             return at(n % R0, n / R0);
     }
-    __device__ __forceinline__ void store(int, int n, float2 v) const { nat(n) = v; }
+    __device__ __forceinline__ void store(int, int n, C v) const { nat(n) = v; }
 };
 
 template <class RX, int SIGN, int PAD>
@@ -75,22 +75,22 @@ struct WarpFft2<Radix<N, R0, R1>, SIGN, PAD> {
 // butterfly, at a lane-dependent a, so each load picks one of two base pointers; the
 // destination receives whole butterflies (store_pfa) and maps indices itself.
 
-template <class RX, int SIGN>
+template <class RX, int SIGN, class C = float2>
 struct WarpFftPfa;
 
-template <int N, int R0, int R1, int SIGN>
-struct WarpFftPfa<Radix<N, R0, R1>, SIGN> {
+template <int N, int R0, int R1, int SIGN, class C>
+struct WarpFftPfa<Radix<N, R0, R1>, SIGN, C> {
     static constexpr bool OK = gcd_c(R0, R1) == 1 && R0 <= 32 && R1 <= 32;
     static constexpr int C1 = (R1 * modinv(R1 % R0, R0)) % N;
     static constexpr int C2 = (R0 * modinv(R0 % R1, R1)) % N;
     template <class Xc, class Dst, class Mid>
-    static __device__ __forceinline__ void run(const float2* z, const Xc& xc, Dst& dst, int lane,
+    static __device__ __forceinline__ void run(const C* z, const Xc& xc, Dst& dst, int lane,
                                                const Mid& mid) {
         if (lane < R1) {                       // stage 1: radix R0, butterfly b = lane
-            const float2* p1 = z + R0 * lane;  // n = R0 b + R1 a, minus N once it passes N
-            const float2* p2 = p1 - N;
+            const C* p1 = z + R0 * lane;       // n = R0 b + R1 a, minus N once it passes N
+            const C* p2 = p1 - N;
             const int aw = (N - R0 * lane + R1 - 1) / R1;
-            float2 v[R0];
+            C v[R0];
 #pragma unroll
             for (int a = 0; a < R0; ++a) v[a] = (a < aw ? p1 : p2)[a * R1];
             Dft<R0, SIGN>::run(v);
@@ -100,7 +100,7 @@ struct WarpFftPfa<Radix<N, R0, R1>, SIGN> {
         __syncwarp();
         mid();
         if (lane < R0) {                       // stage 2: radix R1, butterfly k1 = lane
-            float2 v[R1];
+            C v[R1];
 #pragma unroll
             for (int j = 0; j < R1; ++j) v[j] = xc.at(lane, j);
             Dft<R1, SIGN>::run(v);
