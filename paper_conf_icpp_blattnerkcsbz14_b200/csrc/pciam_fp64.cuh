@@ -811,6 +811,99 @@ __global__ void __launch_bounds__(32 * D4W_WARPS, 1)
     }
 }
 
+// ------------------------------------------------------------------ D1w ---
+// D1 as a warp-per-row kernel (the K1w design in double): the raw uint16 row lands by bulk
+// copy (the next one prefetched after stage 1), the prime-factor 29 x 24 transform runs on the
+// warp with its outputs left in their exchange slots (Z[q] at (q mod R0, q mod R1)), and the
+// R2C post-pass writes the mirror pairs into the panel-blocked Gd.
+constexpr int D1W_WARPS = 12;   // 168 registers: at most three warps per SM sub-partition
+
+struct U16WordSrcD {   // z[n] = x[2n] + i x[2n+1] of a landed uint16 row (exact in double)
+    const uint32_t* p;
+    __device__ __forceinline__ double2 load(int n) const {
+        const uint32_t u = p[n];
+        return make_double2((double)(u & 0xFFFFu), (double)(u >> 16));
+    }
+};
+template <class Xc, int R1>
+struct PfaSlotDstD {   // a warp PFA's stage-2 outputs back into the slots they were read from
+    Xc x;
+    __device__ __forceinline__ void store_pfa(int k1, const double2 (&v)[R1]) const {
+#pragma unroll
+        for (int j = 0; j < R1; ++j) x.at(k1, j) = v[j];
+    }
+};
+
+template <class PL>
+struct D1w {
+    using RI = typename PL::RI;
+    static constexpr size_t RAWB = (size_t)PL::W * 2;                  // a raw row
+    static constexpr size_t XCH = sizeof(double2) * RI::R1 * RI::R0;   // exchange (PAD 0)
+    static constexpr size_t WARP = (RAWB + 15) / 16 * 16 + XCH;
+    static constexpr size_t OFF_WARP = 128;
+    static constexpr size_t SMEM = OFF_WARP + D1W_WARPS * WARP;
+    static constexpr bool OK = D4w<PL>::OK && RAWB % 16 == 0 && SMEM <= 227 * 1024;
+};
+
+template <class PL>
+__global__ void __launch_bounds__(32 * D1W_WARPS, 1)
+    d1w_fwd_rows(const uint16_t* __restrict__ raw, double2* __restrict__ G, int tile0, int ntiles,
+                 const double2* __restrict__ twW) {
+    using DW = D1w<PL>;
+    using RI = typename PL::RI;
+    constexpr int M = PL::M, H = PL::H, R0 = RI::R0, R1 = RI::R1;
+    extern __shared__ __align__(128) unsigned char smem_d1w[];
+    uint64_t* bar = reinterpret_cast<uint64_t*>(smem_d1w) + (threadIdx.x >> 5);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    unsigned char* mine = smem_d1w + DW::OFF_WARP + warp * DW::WARP;
+    const uint32_t* land = reinterpret_cast<const uint32_t*>(mine);
+    using Xc = WarpXchg<R0, R1, 0, double2>;
+    const Xc xc{reinterpret_cast<double2*>(mine + (DW::WARP - DW::XCH))};
+    if (lane == 0) {
+        mbar_init(bar, 1);
+        fence_mbar_init();
+    }
+    __syncwarp();
+    const long long nrows = (long long)ntiles * H;
+    const long long gw = (long long)blockIdx.x * D1W_WARPS + warp, nw = (long long)gridDim.x * D1W_WARPS;
+    const int r0 = (int)(nrows * gw / nw), r1 = (int)(nrows * (gw + 1) / nw);
+    auto issue = [&](int r) {                  // row r = tl * H + y of this chunk's tiles
+        mbar_arrive_expect_tx(bar, (uint32_t)DW::RAWB);
+        bulk_g2s(mine, raw + ((size_t)tile0 * H + r) * PL::W, (uint32_t)DW::RAWB, bar);
+    };
+    if (lane == 0 && r0 < r1) issue(r0);
+    using Src = U16WordSrcD;
+    using SlotDst = PfaSlotDstD<Xc, R1>;
+    using Pfa = WarpFftPfa<typename PL::Row, -1, double2>;
+    int k = 0;
+    for (int r = r0; r < r1; ++r, ++k) {
+        mbar_wait(bar, k & 1);
+        auto prefetch = [&]() {
+            if (lane == 0 && r + 1 < r1) {
+                fence_proxy_async();
+                issue(r + 1);
+            }
+        };
+        SlotDst dst{xc};
+        Pfa::run_src(Src{land}, xc, dst, lane, prefetch);
+        __syncwarp();
+        const int tl = r / H;
+        const GRowD<PL> out{G + (size_t)tl * H * PL::WP, r - tl * H};
+        for (int q = lane; q <= M / 2; q += 32) {
+            const int qm = q == 0 ? 0 : M - q;
+            const double2 zq = xc.at(q % R0, q % R1);
+            const double2 zm = xc.at(qm % R0, qm % R1);
+            const double2 E = make_double2(0.5 * (zq.x + zm.x), 0.5 * (zq.y - zm.y));
+            const double2 O = make_double2(0.5 * (zq.y + zm.y), -0.5 * (zq.x - zm.x));
+            const double2 wo = cmul(__ldg(&twW[q]), O);
+            out[q] = make_double2(E.x + wo.x, E.y + wo.y);
+            if (2 * q != M) out[M - q] = make_double2(E.x - wo.x, wo.y - E.y);
+        }
+        for (int q = M + 1 + lane; q < PL::WP; q += 32) out[q] = make_double2(0.0, 0.0);
+        __syncwarp();                          // exchange free for the next row
+    }
+}
+
 // ------------------------------------------------------------------ D5 ----
 // One warp per pair: reduce the NBLK block partials and emit the K5/K6 key
 // (bits(float(max)) << 32 | (2^32 - 1 - index)); the index is the exact double argmax.

@@ -199,6 +199,7 @@ template <class PL>
 cudaError_t d_setup() {
     using P64 = Plan64<PL>;
     CKE(max_smem(d1_fwd_rows<PL>, P64::ROW_SMEM));
+    if constexpr (D1w<PL>::OK) CKE(max_smem(d1w_fwd_rows<PL>, D1w<PL>::SMEM));
     CKE(max_smem(d4_pair_rows<PL>, P64::D4_SMEM));
     if constexpr (D4w<PL>::OK) CKE(max_smem(d4w_pair_rows<PL>, D4w<PL>::SMEM));
     CKE(max_smem(d2_fwd_cols<PL, true>, P64::D2_SMEM));
@@ -214,6 +215,18 @@ template <class PL>
 void launch_d1(const uint16_t* raw, double2* G, int t0, int nt, const double2* tw2,
                const double2* twW, cudaStream_t s) {
     using P64 = Plan64<PL>;
+    if constexpr (D1w<PL>::OK) {   // warp per row, one CTA per SM
+        static int sms = 0;
+        if (!sms) {
+            int dev = 0;
+            cudaGetDevice(&dev);
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        }
+        const int need = (int)(((long long)nt * PL::H + D1W_WARPS - 1) / D1W_WARPS);
+        d1w_fwd_rows<PL><<<need < sms ? need : sms, 32 * D1W_WARPS, D1w<PL>::SMEM, s>>>(
+            raw, G, t0, nt, twW);
+        return;
+    }
     d1_fwd_rows<PL><<<dim3(P64::NBLK, nt), P64::ROW_T, P64::ROW_SMEM, s>>>(raw, G, t0, tw2, twW);
 }
 template <class PL>

@@ -86,13 +86,22 @@ struct WarpFftPfa<Radix<N, R0, R1>, SIGN, C> {
     template <class Xc, class Dst, class Mid>
     static __device__ __forceinline__ void run(const C* z, const Xc& xc, Dst& dst, int lane,
                                                const Mid& mid) {
+        struct Ptr {
+            const C* z;
+            __device__ __forceinline__ C load(int n) const { return z[n]; }
+        };
+        run_src(Ptr{z}, xc, dst, lane, mid);
+    }
+    // the same with a source functor src.load(n) (element n of the sequence)
+    template <class Src, class Xc, class Dst, class Mid>
+    static __device__ __forceinline__ void run_src(const Src& src, const Xc& xc, Dst& dst,
+                                                   int lane, const Mid& mid) {
         if (lane < R1) {                       // stage 1: radix R0, butterfly b = lane
-            const C* p1 = z + R0 * lane;       // n = R0 b + R1 a, minus N once it passes N
-            const C* p2 = p1 - N;
+            const int n1 = R0 * lane;          // n = R0 b + R1 a, minus N once it passes N
             const int aw = (N - R0 * lane + R1 - 1) / R1;
             C v[R0];
 #pragma unroll
-            for (int a = 0; a < R0; ++a) v[a] = (a < aw ? p1 : p2)[a * R1];
+            for (int a = 0; a < R0; ++a) v[a] = src.load(n1 + a * R1 - (a < aw ? 0 : N));
             Dft<R0, SIGN>::run(v);
 #pragma unroll
             for (int a = 0; a < R0; ++a) xc.at(a, lane) = v[a];
