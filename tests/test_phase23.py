@@ -213,3 +213,25 @@ def test_compose_overlay_stays_inside_the_canvas():
         assert (b[:pad] == 0xBEEF).all() and (b[pad + ch * cw:] == 0xBEEF).all(), (n, m, H, W)
         got = b[pad:pad + ch * cw].reshape(ch, cw)
         assert np.array_equal(got, numpy_overlay(g.tiles, g.origins)), (n, m, H, W)
+
+
+@pytest.mark.gpu
+def test_compose_overlay_async_is_stream_ordered():
+    """stitch_compose_overlay_async returns once enqueued: on a side stream, after work that
+    fills the tiles on that same stream, the canvas equals the synchronous call's."""
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("needs a CUDA device")
+    from paper_conf_icpp_blattnerkcsbz14_b200 import compose_overlay
+    g = synthgrid.make_grid(3, 4, 192, 256, overlap=0.2, delta=4, seed=54)
+    ref_tiles = torch.from_numpy(g.tiles.view(np.int16)).view(torch.uint16).cuda()
+    want = compose_overlay(ref_tiles, g.origins)
+    torch.cuda.synchronize()
+    side = torch.cuda.Stream()
+    with torch.cuda.stream(side):
+        tiles = torch.zeros_like(ref_tiles)
+        tiles.copy_(ref_tiles)                  # the producer, on the same stream
+        canvas = torch.zeros_like(want)
+        compose_overlay(tiles, g.origins, canvas, sync=False)
+    side.synchronize()
+    assert torch.equal(canvas, want)
