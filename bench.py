@@ -310,7 +310,8 @@ def run_pooled(args, cfg):
     line = {"metric": metric_name(cfg), "value": pairs / (ms / 1e3), "unit": "pairs/s",
             "n_gpus": 1, "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms,
             "higher_is_better": True, "scaling": "strong", "vs_baseline": None,
-            "dtype": "f32 (Q15 resident phasor)", "data": "synthetic", "config": conf,
+            "dtype": "f32 (Q15 resident phasor, fp16 Q intermediate)" if W >= 1024
+                     else "f32 (Q15 resident phasor)", "data": "synthetic", "config": conf,
             "e2e": {"value": pairs / e2e_s, "unit": "pairs/s",
                     "h2d_bytes_per_step": n * m * H * W * 2, "d2h_bytes_per_step": pairs * 64,
                     "grid_wall_ms": e2e_s * 1e3},
@@ -473,6 +474,9 @@ def main():
         "k4_pair_rows": S,             # Q in (the surface is never stored)
         "k5_ccf_moments": 2 * T,       # the four candidate overlaps of A and B (HW pixels each)
         "k6_finalize": 8 + 160 + 64}
+    q_half = W >= 1024 and args.precision != "f64"   # Plan::Q_HALF: Q as scaled fp16 pairs
+    if q_half:
+        alg_bytes_per_unit.update({"k3_pair_cols": S // 2 * 2 + S // 2, "k4_pair_rows": S // 2})
     if args.precision == "f64":
         # fp64 path (D1..D4, pciam_fp64.cuh): complex intermediates are 2S (complex128), the
         # resident unit phasor is S (Q31, 8 B per bin); D4's per-block argmax partials are ~0
@@ -495,8 +499,9 @@ def main():
                 "peak_source": pk_kind, "avg_launch_ms": avg_launch_ms,
                 "alg_bytes_per_launch": bytes_per_launch,
                 "byte_model": ("design: bytes each kernel must move with the resident spectrum "
-                               "as a Q15 unit phasor (S/2 per tile) and complex64 G/Q chunks "
-                               "(S); DESIGN.md section 6"),
+                               "as a Q15 unit phasor (S/2 per tile), complex64 G chunks (S) and "
+                               + ("fp16 Q chunks (S/2)" if q_half else "complex64 Q chunks (S)")
+                               + "; DESIGN.md section 6"),
                 "share_of_step": kd["ms"] / step_kernel_ms,
                 "kernels_ms_per_step": kms,
                 "kernels_launches_per_step": klaunch,
@@ -636,6 +641,7 @@ def main():
                                "(Table II, P:L1208) = 97.7 pairs/s; other hardware, end to end "
                                "incl. TIFF reads",
             "dtype": ("f64 (Q31 resident phasor)" if args.precision == "f64"
+                      else "f32 (Q15 resident phasor, fp16 Q intermediate)" if W >= 1024
                       else "f32 (Q15 resident phasor)"),
             "data": "synthetic",
             "config": conf,

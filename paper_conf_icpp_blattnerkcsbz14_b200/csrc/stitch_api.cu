@@ -67,6 +67,7 @@ struct PlanOps {
                int, cudaStream_t);
     // fp64 path (f2, pciam_fp64.cuh)
     int nblk64;
+    double q_scale;   // the scale K3 applies to Q (carried to the reported peak height)
     cudaError_t (*d_setup)();
     void (*d1)(const uint16_t*, double2*, int, int, const double2*, const double2*, cudaStream_t);
     void (*d2)(const double2*, int2*, double2*, int, int, const double2*, bool, cudaStream_t);
@@ -115,13 +116,14 @@ cudaError_t plan_setup(int* grid_k1, int* grid_k4) {
         using RW = RowWarp<PL>;
         constexpr bool PFA = k4_pfa_ok<PL>();
         CKE(max_smem(k1w_fwd_rows<PL>, RW::SMEM_K1));
-        CKE(max_smem(k4w_pair_rows<PL, PFA>, RW::SMEM_K4));
-        CKE(max_smem(k4w_pair_rows<PL, PFA, true>, RW::SMEM_K4));
+        CKE(max_smem(k4w_pair_rows<PL, PFA>, RW::template SMEM_K4<PFA>));
+        CKE(max_smem(k4w_pair_rows<PL, PFA, true>, RW::template SMEM_K4<PFA>));
         CKE(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k1w_fwd_rows<PL>, 32 * ROWW_WARPS,
                                                           RW::SMEM_K1));
         *grid_k1 = nb * sms;
         CKE(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, k4w_pair_rows<PL, PFA>,
-                                                          32 * ROWW_WARPS, RW::SMEM_K4));
+                                                          32 * ROWW_WARPS,
+                                                          RW::template SMEM_K4<PFA>));
         *grid_k4 = nb * sms;
     } else {
         CKE(max_smem(k1_fwd_rows<PL>, PL::ROW_SMEM));
@@ -168,7 +170,8 @@ void launch_k4(const float2* Q, unsigned long long* keys, int p0, int np, const 
     if constexpr (RowWarp<PL>::OK) {
         const int need = (np * PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
         k4w_pair_rows<PL, k4_pfa_ok<PL>()><<<grid < need ? grid : need, 32 * ROWW_WARPS,
-                                             RowWarp<PL>::SMEM_K4, s>>>(Q, keys, p0, np, tw2, twW);
+                                             RowWarp<PL>::template SMEM_K4<k4_pfa_ok<PL>()>, s>>>(
+            Q, keys, p0, np, tw2, twW);
     } else {
         k4_pair_rows<PL><<<dim3(PL::H / PL::ROW_L, np), PL::ROW_T, PL::ROW_SMEM, s>>>(Q, keys, p0,
                                                                                       tw2, twW);
@@ -180,7 +183,7 @@ void launch_k4s(const float2* Q, float* surf, float scale, const float2* tw2, co
     if constexpr (RowWarp<PL>::OK) {
         const int need = (PL::H + ROWW_WARPS - 1) / ROWW_WARPS;
         k4w_pair_rows<PL, k4_pfa_ok<PL>(), true><<<grid < need ? grid : need, 32 * ROWW_WARPS,
-                                                   RowWarp<PL>::SMEM_K4, s>>>(
+                                                   RowWarp<PL>::template SMEM_K4<k4_pfa_ok<PL>()>, s>>>(
             Q, nullptr, 0, 1, tw2, twW, surf, scale);
     } else {
         k4_pair_rows<PL, true><<<dim3(PL::H / PL::ROW_L, 1), PL::ROW_T, PL::ROW_SMEM, s>>>(
@@ -284,6 +287,7 @@ PlanOps make_ops() {
     PlanOps o;
     o.W = PL::W; o.H = PL::H; o.M = PL::M; o.WC = PL::WC; o.WP = PL::WP; o.HP = PL::HP; o.HP64 = Plan64<PL>::HP64;
     o.col_p = PL::COL_P;
+    o.q_scale = PL::Q_SCALE;
     o.row_r0 = PL::RI::R0; o.row_r1 = PL::RI::R1; o.col_r0 = PL::CI::R0; o.col_r1 = PL::CI::R1;
     o.setup = plan_setup<PL>;
     o.k1 = launch_k1<PL>; o.k2 = launch_k2<PL>; o.k3 = launch_k3<PL>; o.k4 = launch_k4<PL>;
@@ -1016,7 +1020,7 @@ static stitch_status enqueue_ops(stitch_ctx* ctx, const std::vector<Op>& ops, co
             // the key's value is max |c| (fp64 path) or max |c| x 32767^2 (Q15 phasor NCPS)
             k6_finalize<<<(unsigned)((np + 127) / 128), 128, 0, sk>>>(
                 ctx->keys + pa, ctx->mom + pa * 20, ctx->res + pa, ctx->H, ctx->W, (int)np,
-                (double)ctx->W * ctx->H * (ctx->prec ? Q31_S * Q31_S : NCPS_Q15_SCALE));
+                (double)ctx->W * ctx->H * (ctx->prec ? Q31_S * Q31_S : NCPS_Q15_SCALE * o->q_scale));
         });
         mark(ctx, 5);
         ctx->launches += 1;
@@ -1679,7 +1683,7 @@ stitch_status stitch_debug_surface(stitch_ctx* ctx, int32_t tile, int32_t kind, 
     GUARD(ctx);
     const PlanOps* o = ctx->ops;
     float* surf = reinterpret_cast<float*>(ctx->G);   // H*W floats fit one chunk slot of G
-    const float scale = (float)(1.0 / ((double)ctx->W * ctx->H * NCPS_Q15_SCALE));
+    const float scale = (float)(1.0 / ((double)ctx->W * ctx->H * NCPS_Q15_SCALE * ctx->ops->q_scale));
     o->k3(ctx->spec, ctx->Q, ctx->pairs, (int)p, 1, ctx->twH, ctx->stream);
     o->k4s(ctx->Q, surf, scale, ctx->twM, ctx->twW, ctx->grid_k4, ctx->stream);
     CK(cudaGetLastError(), "surface launch");

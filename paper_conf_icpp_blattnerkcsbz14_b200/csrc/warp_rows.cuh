@@ -13,6 +13,8 @@
 
 #include <type_traits>
 
+#include <cuda_fp16.h>
+
 #include "async_copy.cuh"
 #include "fft_engine.cuh"
 
@@ -139,9 +141,18 @@ struct RowWarp {
     static constexpr size_t OFF_TWW = OFF_TW2 + (size_t)(PL::ROW_TW2 > 0 ? PL::ROW_TW2 : 1) * 8;
     static constexpr size_t OFF_WARP = (OFF_TWW + (size_t)(PL::M + 1) * 8 + 127) / 128 * 128;
     static constexpr size_t WARP_K1 = ((size_t)RAWB + 15) / 16 * 16 + (size_t)XCH * 8;
-    static constexpr size_t WARP_K4 = (size_t)QROW + (size_t)XCH * 8;
     static constexpr size_t SMEM_K1 = OFF_WARP + ROWW_WARPS * WARP_K1;
-    static constexpr size_t SMEM_K4 = OFF_WARP + ROWW_WARPS * WARP_K4;
+    // K4: the landed Q row (fp16 pairs, or float2), the C2R-processed row Z (float2), the exchange; the
+    // stage-2 twiddle table only for the Stockham rows (the prime-factor rows need none); w_W
+    // is read through L1
+    static constexpr int QROWH = PL::WP * (PL::Q_HALF ? 4 : 8);   // a landed Q row
+    static constexpr size_t ZROW = ((size_t)PL::M * 8 + 15) / 16 * 16;
+    static constexpr size_t WARP_K4 = (size_t)QROWH + ZROW + (size_t)XCH * 8;
+    template <bool PFA>
+    static constexpr size_t OFF_WARP4 =
+        (OFF_TW2 + (PFA ? 0 : (size_t)(PL::ROW_TW2 > 0 ? PL::ROW_TW2 : 1) * 8) + 127) / 128 * 128;
+    template <bool PFA>
+    static constexpr size_t SMEM_K4 = OFF_WARP4<PFA> + ROWW_WARPS * WARP_K4;
     static constexpr bool OK = RI::STAGES == 2 && RAWB % 16 == 0;
 };
 
@@ -338,33 +349,35 @@ struct WarpSurfacePfa {
 // SURF: the test hook's surface output (one pair, `surf` [H][W]) instead of the argmax.
 template <class PL, bool PFA = false, bool SURF = false>
 __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
-    k4w_pair_rows(const float2* __restrict__ Q, unsigned long long* __restrict__ keys, int pair0,
+    k4w_pair_rows(const float2* __restrict__ Qf, unsigned long long* __restrict__ keys, int pair0,
                   int npairs, const float2* __restrict__ tw2, const float2* __restrict__ twW,
                   float* __restrict__ surf = nullptr, float scale = 0.f) {
     using RW = RowWarp<PL>;
     constexpr int M = PL::M, H = PL::H;
+    using QT = std::conditional_t<PL::Q_HALF, __half2, float2>;   // scaled fp16 pairs, or float2
+    const QT* Q = reinterpret_cast<const QT*>(Qf);
     extern __shared__ __align__(128) unsigned char smem_w[];
     uint64_t* bars = reinterpret_cast<uint64_t*>(smem_w);
     float2* tw2s = reinterpret_cast<float2*>(smem_w + RW::OFF_TW2);
-    float2* twWs = reinterpret_cast<float2*>(smem_w + RW::OFF_TWW);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    unsigned char* mine = smem_w + RW::OFF_WARP + warp * RW::WARP_K4;
-    float2* landw = reinterpret_cast<float2*>(mine);
-    const float2* land = landw;
-    typename RW::IFft::Xc xc{reinterpret_cast<float2*>(mine + RW::QROW)};
+    unsigned char* mine = smem_w + RW::template OFF_WARP4<PFA> + warp * RW::WARP_K4;
+    const QT* landh = reinterpret_cast<const QT*>(mine);
+    float2* zrow = reinterpret_cast<float2*>(mine + RW::QROWH);
+    typename RW::IFft::Xc xc{reinterpret_cast<float2*>(mine + RW::QROWH + RW::ZROW)};
     uint64_t* bar = &bars[warp];
     if (lane == 0) {
         mbar_init(bar, 1);
         fence_mbar_init();
     }
-    rowwarp_tables<PL>(tw2s, twWs, tw2, twW);
+    if constexpr (!PFA)
+        for (int i = threadIdx.x; i < PL::ROW_TW2; i += 32 * ROWW_WARPS) tw2s[i] = __ldg(tw2 + i);
     __syncthreads();                           // the only CTA-wide barrier
     const long long nrows = (long long)npairs * H;
     const long long gw = (long long)blockIdx.x * ROWW_WARPS + warp, nw = (long long)gridDim.x * ROWW_WARPS;
     const int r0 = (int)(nrows * gw / nw), r1 = (int)(nrows * (gw + 1) / nw);
     auto issue = [&](int r) {
-        mbar_arrive_expect_tx(bar, RW::QROW);
-        bulk_g2s(mine, Q + (size_t)r * PL::WP, RW::QROW, bar);
+        mbar_arrive_expect_tx(bar, RW::QROWH);
+        bulk_g2s(mine, Q + (size_t)r * PL::WP, RW::QROWH, bar);
     };
     auto flush = [&](int pair, float bv, uint32_t bi) {
         unsigned long long key =
@@ -397,35 +410,40 @@ __global__ void __launch_bounds__(32 * ROWW_WARPS, ROWW_MINB4)
         }
         acc.row_base = y;
         mbar_wait(bar, k & 1);
-        // C2R pre-processing in place, one mirror pair (q, M-q) per lane and iteration (all 32
-        // lanes; the radix-R0 stage below keeps only R1 of them busy):
+        // C2R pre-processing from the landed row into the float row Z, one mirror pair
+        // (q, M-q) per lane and iteration:
         //   d = X[q] - conj X[M-q],  o = d conj(w_W^q),  Z[q] = X[q] + conj X[M-q] + i o,
         //   Z[M-q] = conj(X[q] + conj X[M-q]) + i conj(o)      (w_W^{M-q} = -conj w_W^q)
-        // so Z (the length-M complex sequence whose inverse FFT interleaves the real row)
-        // replaces the landed Hermitian row; Z[0] pairs X[0] with X[M].
+        // so Z (the length-M complex sequence whose inverse FFT interleaves the real row) is
+        // ready and the landing buffer free: the next row is requested right away.
         for (int q = lane; 2 * q <= M; q += 32) {
-            const float2 xn = landw[q], xm = landw[M - q];
-            const float2 o = cmulc(make_float2(xn.x - xm.x, xn.y + xm.y), twWs[q]);
+            float2 xn, xm;
+            if constexpr (PL::Q_HALF) {
+                xn = __half22float2(landh[q]);
+                xm = __half22float2(landh[M - q]);
+            } else {
+                xn = landh[q];
+                xm = landh[M - q];
+            }
+            const float2 o = cmulc(make_float2(xn.x - xm.x, xn.y + xm.y), __ldg(&twW[q]));
             const float sx = xn.x + xm.x, dy = xn.y - xm.y;
-            landw[q] = make_float2(sx - o.y, dy + o.x);
-            if (q != 0 && 2 * q != M) landw[M - q] = make_float2(sx + o.y, o.x - dy);
+            zrow[q] = make_float2(sx - o.y, dy + o.x);
+            if (q != 0 && 2 * q != M) zrow[M - q] = make_float2(sx + o.y, o.x - dy);
         }
         __syncwarp();
+        if (lane == 0 && r + 1 < r1) {
+            fence_proxy_async();
+            issue(r + 1);
+        }
         struct Src {
             const float2* z;
             __device__ __forceinline__ float2 load(int, int n) const { return z[n]; }
-        } src{land};
-        auto prefetch = [&]() {
-            if (lane == 0 && r + 1 < r1) {
-                fence_proxy_async();
-                issue(r + 1);
-            }
-        };
+        } src{zrow};
         if constexpr (PFA)
-            Pfa::run(land, xc, acc, lane, prefetch);
+            Pfa::run(zrow, xc, acc, lane, NoMid());
         else
-            RW::IFft::run(src, xc, acc, tw2s, lane, prefetch);
-        __syncwarp();                          // exchange free for the next row
+            RW::IFft::run(src, xc, acc, tw2s, lane, NoMid());
+        __syncwarp();                          // Z and the exchange free for the next row
     }
     if constexpr (!SURF)
         if (cur >= 0) flush(cur, acc.best_v, acc.best_i);

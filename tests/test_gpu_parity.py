@@ -374,7 +374,10 @@ def test_correlation_surface_matches_oracle(H, W, seed):
     """Reading C11 measured: the step's own K3 + K4 transforms (K4 storing the surface instead
     of reducing it) from the resident Q15 unit phasors give the normalised correlation surface
     |iFFT2(NCC)|/(HW) of the oracle (fp64, exact phasors) element by element; the error is a
-    small fraction of the 1e-4 peak-height contract.  Measured max errors are printed."""
+    small fraction of the 1e-4 peak-height / near-tie margin.  Bound: 1e-5 of the peak with a
+    float2 intermediate Q (small plans), 5e-5 with the scaled fp16 Q of the 1392x1040 plan
+    (reading C11-Q: measured ~2e-5, still 2x inside the 1e-4 margin that decides
+    near-ties, C17).  Measured max errors are printed."""
     g = synthgrid.make_grid(2, 2, H, W, seed=seed)
     with PciamGrid(2, 2, H, W) as pg:
         pg.load_grid(g.tiles)
@@ -388,6 +391,6 @@ def test_correlation_surface_matches_oracle(H, W, seed):
             rms = np.sqrt(np.mean(ref ** 2))
             print(f"surface {H}x{W} pair ({r},{c},{kind}): peak {peak:.4g}, max abs err "
                   f"{err:.3g} = {err / peak:.3g} of the peak, {err / rms:.3g} of the rms")
-            assert err <= 1e-5 * peak, (err, peak)
+            assert err <= (5e-5 if W >= 1024 else 1e-5) * peak, (err, peak)
             assert np.unravel_index(np.argmax(got), got.shape) == np.unravel_index(
                 np.argmax(ref), ref.shape)
