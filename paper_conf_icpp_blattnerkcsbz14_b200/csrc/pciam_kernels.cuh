@@ -109,6 +109,8 @@ struct Plan {
     // float2 for the small test plans, whose fewer samples leave less averaging
     static constexpr bool Q_HALF = W >= 1024;
     static constexpr double Q_SCALE = Q_HALF ? 1.0 / 33554432.0 : 1.0;
+    static_assert(!Q_HALF || H * 32767.0 * 32767.0 * 1.0001 / 33554432.0 < 65504.0,
+                  "scaled fp16 Q would overflow: |Q| <= H 32767^2");
     static_assert(W % 2 == 0, "W must be even");
     static_assert(Row::N == M && Col::N == H, "plan radices do not match the tile");
     static_assert(H % ROW_L == 0, "rows per CTA must divide H");
