@@ -11,10 +11,12 @@
 //                                        4 mod 8 words), stored as its Q15 unit phasor F/|F|
 //                                        (2 x int16), reused by <= 4 pairs: K3's
 //                                        column panel of a tile is one contiguous run
-//   Q     float2 [chunk][H][WP]          per-pair column-inverse intermediate
+//   Q     half2 / float2 [chunk][H][WP]  per-pair column-inverse intermediate (scaled fp16
+//                                        pairs for the 1392x1040 plan, reading C11-Q)
 //   fslot i32    [local tiles]           slot of each local tile (K1/K2 write there)
 //   pairs {a, b} [pairs]                 slots of the pair's tiles (K3/K5 read there)
-// (G and Q chunks are 0.38 / 0.94 GB at the default 64 / 160 chunks: they round-trip HBM,
+// (G and Q chunks are 0.38 / 0.47 GB at the default 64 / 160 chunks -- Q as scaled fp16 pairs
+// for the 1392x1040 plan, Plan::Q_HALF -- and they round-trip HBM,
 // DESIGN.md section 6.)
 //   keys  u64    [pairs]                 packed (|c| bits << 32 | ~index) argmax per pair
 //   mom   u64    [pairs][4][5]           exact integer CCF moments per candidate

@@ -4,7 +4,7 @@
 //   * plan table: the compiled FFT plans per tile size (radices, CTA shapes);
 //   * layout: raw pixels and Q15 phasor spectra by SLOT (slot = local tile in the resident
 //     mode; a recycled pool slot in the bounded mode), the forward-chunk G
-//     and pair-chunk Q intermediates (0.38 / 0.94 GB at the default 64 / 160 chunks: they
+//     and pair-chunk Q intermediates (0.38 / 0.47 GB at the default 64 / 160 chunks: they
 //     round-trip HBM), the pair list (Fig. 4), argmax keys, CCF moments, results;
 //   * schedule: a static list of forward chunks (K1 + K2, an H2D copy first when the tiles come
 //     from the host) and pair chunks (K3 + K4, then K5), decided at stitch_init and enqueued on
