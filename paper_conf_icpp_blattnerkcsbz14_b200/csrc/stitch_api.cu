@@ -423,10 +423,13 @@ stitch_status make_layout(const stitch_config* c, const PlanOps* ops, Layout* L)
     // default chunks (both precisions): 160 pairs / 64 tiles -- the intermediates round-trip
     // HBM either way, and larger launches lose less to their tail wave (fp64 sweep: 8/8 75.7 ms,
     // 32/16 68.5 ms, 160/64 67.8 ms per 42x59 step, DESIGN.md variant 40)
-    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs : 160;
-    L->chunk_tiles = c->chunk_tiles > 0
-                         ? c->chunk_tiles
-                         : (L->pool ? std::max(1, std::min(64, L->nslots / 4)) : 64);
+    // bounded mode: chunks of about an eighth of the pool (and ~3 pairs per tile), so slots
+    // turn over while the H2D stream runs ahead (pool 160 at 42x59: 20 / 60 -> 132 ms end to
+    // end, PCIe-bound like the resident mode; 40 / 160: 154 ms)
+    const int ct_pool = std::max(1, std::min(64, L->nslots / 8));
+    L->chunk_tiles = c->chunk_tiles > 0 ? c->chunk_tiles : (L->pool ? ct_pool : 64);
+    L->chunk_pairs = c->chunk_pairs > 0 ? c->chunk_pairs
+                                        : (L->pool ? std::min(160, 3 * L->chunk_tiles) : 160);
     if (L->chunk_pairs > 65535 || L->chunk_tiles > 65535) return STITCH_ERR_INVALID_ARG;
     const size_t H = ops->H, W = ops->W, WP = ops->WP;
     // spectrum by slot: u32 Q15 unit phasor [WP][HP] (fp32) or double2 unit phasor [H][WP] (fp64)
@@ -737,7 +740,7 @@ static bool build_pooled(stitch_ctx* ctx, std::string* why) {
     std::vector<int> tag_pair(L.nslots, -1), tag_fwd(L.nslots, -1);
     struct P { int a, b, t; int8_t kind; };   // local tiles
     std::deque<P> pending;
-    int cur_f = -1;
+    int cur_f = -1, next_slot = 0;
     auto release = [&](int lt, int tp, int tf) {
         const int s = ctx->fslot_h[lt];
         tag_pair[s] = tp;
@@ -770,8 +773,14 @@ static bool build_pooled(stitch_ctx* ctx, std::string* why) {
         }
         FwdChunk fc{t0, nt};
         for (int i = 0; i < nt; ++i) {
-            const int s = *free_slots.begin();
-            free_slots.erase(free_slots.begin());
+            // next fit around the ring: slots are freed roughly in the order they were taken,
+            // so continuing after the last one keeps a chunk's slots in long runs (one H2D copy
+            // per run, copy_chunk_in) instead of refilling scattered low slots
+            auto it = free_slots.lower_bound(next_slot);
+            if (it == free_slots.end()) it = free_slots.begin();
+            const int s = *it;
+            free_slots.erase(it);
+            next_slot = s + 1;
             ctx->fslot_h[t0 + i] = s;
             fc.wait_pair = std::max(fc.wait_pair, tag_pair[s]);
             fc.wait_fwd = std::max(fc.wait_fwd, tag_fwd[s]);
